@@ -1,0 +1,269 @@
+/*
+ * bless.h -- C ABI of the B200-native BLESS hot path.
+ *
+ * BLESS = "Improving GPU Sharing Performance through Adaptive Bubbleless
+ * Spatial-Temporal Sharing" (Zhang et al., EuroSys '25).  Citations "L<n>" are
+ * lines of that paper's text; "R<n>" are the readings of the paper
+ * recorded in DESIGN.md §3.
+ *
+ * The calls follow the paper's problem statement (L143, L145, L157, L259,
+ * L276): an application registers with a GPU quota, its kernels are profiled
+ * offline at every SM count, requests are submitted into per-application FIFO
+ * queues, a scheduler groups kernels of concurrent requests into kernel squads,
+ * picks an execution configuration (no restriction, or a spatial SM split) from
+ * the profile, launches the kernels confined to their SM ranges, and the
+ * caller polls for completion.
+ *
+ * Conventions
+ *  - One bl_ctx per GPU ("replicating its runtime components for each active
+ *    GPU", L171).  device = BL_DEVICE_NONE builds a CUDA-free context that runs
+ *    the same C++ scheduler on a virtual clock (CPU parity tests).
+ *  - Every call returns bl_status; on failure bl_last_error() returns a
+ *    thread-local message.  No C++ exception crosses this boundary.
+ *  - All times are int64 nanoseconds.  Host times use bl_now_ns()
+ *    (CLOCK_MONOTONIC).  Quotas are converted once to integer parts-per-million;
+ *    no floating point enters a scheduling decision.
+ *  - Pointers inside bl_op are DEVICE pointers, allocated by the caller
+ *    (PyTorch) and BORROWED: they must stay valid until bl_destroy.  All other
+ *    pointer arguments are host pointers owned by the caller and only read or
+ *    written during the call.
+ *  - Thread safety: bl_submit / bl_poll / bl_now_ns may be called from any
+ *    thread after bl_start (bl_submit: at most one producer per tenant).
+ *    Everything else is single-threaded setup/teardown.
+ */
+#ifndef BLESS_BLESS_H
+#define BLESS_BLESS_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define BL_MAX_TENANTS 16   /* per GPU */
+#define BL_MAX_SQUAD 128    /* squad_max upper bound */
+#define BL_DEVICE_NONE (-1)
+
+typedef struct bl_ctx bl_ctx;
+
+typedef enum {
+  BL_OK = 0,
+  BL_PENDING = 1,       /* bl_poll: request not finished yet */
+  BL_E_INVALID = -1,    /* bad argument (null pointer, out-of-range index, bad op) */
+  BL_E_QUOTA = -2,      /* quota <= 0, > 1, sum > 1 + 1e-9, or < 1 SM after apportionment */
+  BL_E_STATE = -3,      /* call not allowed in the current state (see each call) */
+  BL_E_CUDA = -4,       /* a CUDA call failed; the ctx is unusable afterwards */
+  BL_E_OOM = -5,        /* host/device allocation failed or workspace too small */
+  BL_E_FULL = -6,       /* request table / ring full */
+  BL_E_NOTFOUND = -7,   /* unknown request id / file */
+  BL_E_TIMEOUT = -8     /* bl_drain timed out */
+} bl_status;
+
+/* Scheduling policies.  BLESS is the paper's method (§4.3-§4.5).  The others
+ * are the in-run baselines of §6.1 (L300-L304) on the same executor/kernels:
+ *  ISO/STATIC - each tenant confined to its quota SM range, whole request
+ *               launched at arrival (ISO = run with one tenant's sub-trace);
+ *  TEMPORAL   - time slices of quota*period on the full GPU (L41, R22);
+ *  UNBOUND    - every request launched at arrival on [0,S) (native CUDA
+ *               stream concurrency, L103). */
+typedef enum {
+  BL_POLICY_BLESS = 0,
+  BL_POLICY_ISO = 1,
+  BL_POLICY_STATIC = 2,
+  BL_POLICY_TEMPORAL = 3,
+  BL_POLICY_UNBOUND = 4
+} bl_policy;
+
+/* R17.  VIRTUAL: 'now' of each decision is the predicted-time chain (exactly
+ * the oracle DES); all requests must be submitted before bl_start; on a GPU a
+ * squad is never launched before the wall time of its newest arrival.
+ * WALL: 'now' = max(host time, predicted end of the in-flight squad); every
+ * decision's inputs are logged so the oracle can replay it. */
+typedef enum { BL_CLOCK_WALL = 0, BL_CLOCK_VIRTUAL = 1 } bl_clock;
+
+typedef struct {
+  int32_t sm_unit;            /* g: SMs per partition (R8; default 4 -> N = 37 on B200) */
+  int32_t squad_max;          /* max kernels per squad (L181, L408; R5; default 50) */
+  int32_t split_pct;          /* Semi-SP ratio c% (L255; R16; default 50) */
+  int32_t seed_all;           /* R6: seed every active request first (default 1) */
+  int32_t policy;             /* bl_policy */
+  int32_t clock;              /* bl_clock */
+  int64_t squad_overhead_ns;  /* VIRTUAL clock: added to 'now' after each squad (L432) */
+  int64_t temporal_period_ns; /* TEMPORAL period P (R22; default 2 ms) */
+  int32_t temporal_work_conserving; /* 0 = T-cap, 1 = T-wc (R22) */
+  int32_t max_inflight_squads;      /* WALL: squads queued on the GPU ahead (default 2) */
+  int64_t lookahead_ns;       /* WALL: decide the next squad this long before the
+                                 predicted end of the in-flight one (default 20 us) */
+  int64_t max_requests;       /* request-table capacity (default 1<<20) */
+} bl_params;
+
+/* Fill *p with the defaults listed above. */
+void bl_params_default(bl_params* p);
+
+/* ---- tenant layers (the applications' kernels, L143 "invoke GPU functions at
+ * the granularity of GPU kernels") ------------------------------------------ */
+typedef enum {
+  BL_OP_GEMM = 0,    /* Y[M,N] = act((X[M,K] W[N,K]^T) * scale + shift + R)          */
+  BL_OP_CONV = 1,    /* NHWC conv, KRSC weights, same epilogue                        */
+  BL_OP_POOL = 2,    /* max / avg / global-avg pooling, NHWC                          */
+  BL_OP_ELTWISE = 3, /* Y = act(X * scale + shift (+ R)), per-channel, any layout      */
+  BL_OP_VIRTUAL = 15 /* no device work (BL_DEVICE_NONE contexts / profile-only)       */
+} bl_op_kind;
+
+typedef enum { BL_F32 = 0, BL_BF16 = 1 } bl_dtype;
+typedef enum { BL_ACT_NONE = 0, BL_ACT_RELU = 1, BL_ACT_RELU6 = 2, BL_ACT_GELU = 3 } bl_act;
+typedef enum { BL_POOL_MAX = 0, BL_POOL_AVG = 1, BL_POOL_GLOBAL_AVG = 2 } bl_pool_mode;
+
+/* Operation descriptor.  Layouts are row-major, contiguous unless an ld* is
+ * given.  Element types: X/W/R/Y in 'dtype'; scale/shift are always fp32
+ * per-output-channel vectors (nullable: scale = 1, shift = 0).
+ *
+ *  GEMM  dims = {M, N, K, ldx(0=K), ldy(0=N), ldr(0=N), split_k(0=auto)}
+ *        ptr  = {X, W, scale, shift, R, Y}
+ *  CONV  dims = {Nb, H, W, C, K, R, S, stride, pad, groups, ldx(0=C), ldy(0=K)}
+ *        ptr  = {X, W(KRSC), scale, shift, R(ld = ldy), Y}
+ *        (channel slices: offset the pointers, give ld*)
+ *  POOL  dims = {Nb, H, W, C, k, stride, pad, mode(bl_pool_mode)}
+ *        ptr  = {X, Y}
+ *  ELTWISE dims = {rows, C}  ptr = {X, scale, shift, R, Y}
+ */
+typedef struct {
+  int32_t kind;     /* bl_op_kind */
+  int32_t dtype;    /* bl_dtype */
+  int32_t act;      /* bl_act */
+  int32_t flags;    /* reserved, 0 */
+  int64_t dims[12];
+  void* ptr[8];
+  float fparam[4];
+} bl_op;
+
+typedef struct {
+  uint64_t req;
+  int32_t tenant;
+  int32_t status;     /* BL_OK or BL_PENDING */
+  int64_t arrival_ns; /* as submitted (host clock, or trace time in VIRTUAL) */
+  int64_t start_ns;   /* first kernel's first CTA (host clock), or model time */
+  int64_t finish_ns;  /* last kernel's last CTA (host clock), or model time */
+} bl_req_info;
+
+/* One scheduling decision (BLESS policy), for bit-exact replay by the oracle.
+ * config_sp = 0 -> NSP (no spatial restriction), 1 -> SP split p[0..K-1]
+ * (partitions of g SMs per participant, participants in tenant-id order). */
+typedef struct {
+  int64_t now;
+  int64_t t_hat;   /* chosen predicted squad duration */
+  int64_t t_nsp;   /* Eq. 2 prediction (NSP) */
+  int32_t n_active;
+  int32_t n_part;
+  int32_t config_sp;
+  int32_t n_picks;
+  int32_t act_tenant[BL_MAX_TENANTS];
+  int32_t act_next[BL_MAX_TENANTS];
+  int64_t act_arrival[BL_MAX_TENANTS];
+  int32_t part_tenant[BL_MAX_TENANTS];
+  int32_t part_p[BL_MAX_TENANTS];
+  int32_t pick_tenant[BL_MAX_SQUAD];
+  int32_t pick_kernel[BL_MAX_SQUAD];
+  int16_t pick_lo[BL_MAX_SQUAD];
+  int16_t pick_hi[BL_MAX_SQUAD];
+} bl_decision;
+
+/* One executed kernel launch (device timestamps converted to host clock). */
+typedef struct {
+  uint64_t seq;
+  int32_t tenant;
+  int32_t kernel;
+  int16_t lo, hi;     /* logical SM range */
+  int32_t nsm;        /* distinct SMs that processed >= 1 tile */
+  int32_t fallback;   /* 1 if no in-range CTA ran and the last CTA did the work */
+  int64_t start_ns;   /* first tile claimed */
+  int64_t end_ns;     /* last CTA exit */
+  uint64_t req;
+} bl_launch_rec;
+
+/* Device facts from the probe kernel (A1). */
+typedef struct {
+  int32_t device;
+  int32_t sm_count;        /* S */
+  int32_t max_smid;        /* %nsmid - 1 */
+  int32_t cc_major, cc_minor;
+  int32_t tpc_pairs_found; /* cluster-2 probe: pairs whose smids differ by 1 */
+  int64_t globaltimer_res_ns; /* smallest observed globaltimer step */
+  int64_t clock_offset_ns;    /* globaltimer - host clock */
+  int64_t l2_bytes;
+  int64_t smem_per_block_optin;
+  uint8_t smid_to_lid[256];   /* 255 = not a usable SM */
+} bl_device_info;
+
+/* ---- lifecycle ---------------------------------------------------------------
+ * bl_create: device >= 0 selects a CUDA device and runs the SM probe (A1);
+ * BL_DEVICE_NONE makes a CUDA-free ctx (S, g come from bl_load_profile).
+ * workspace/ws_bytes: optional caller-owned device buffer for the launch-slot
+ * ring (>= 4 MiB); NULL lets the library cudaMalloc it.  Errors: BL_E_INVALID,
+ * BL_E_CUDA, BL_E_OOM. */
+bl_status bl_create(int device, const bl_params* params, void* workspace, size_t ws_bytes, bl_ctx** out);
+bl_status bl_destroy(bl_ctx* ctx);               /* stops threads, frees library memory */
+bl_status bl_device_info_get(bl_ctx* ctx, bl_device_info* out);
+
+/* Register an application with a GPU quota in (0, 1] (L143, L157).  Before
+ * bl_start only.  Sum of quotas must be <= 1 + 1e-9 (BL_E_QUOTA). */
+bl_status bl_register_tenant(bl_ctx* ctx, double quota, const char* name, int* tenant_out);
+/* Optional: run tenant's kernels on a caller-owned cudaStream_t (torch stream). */
+bl_status bl_set_stream(bl_ctx* ctx, int tenant, void* cuda_stream);
+/* Append one kernel to the tenant's per-request kernel sequence.  Validates
+ * the op and builds its launch descriptor (tiles, grid, TMA maps).  Before
+ * bl_start; BL_E_INVALID on a malformed op. */
+bl_status bl_append_kernel(bl_ctx* ctx, int tenant, const bl_op* op, int* kernel_idx_out);
+/* Run one kernel (not a request) once, unrestricted, on the tenant's stream and
+ * wait: parity tests use it to compare a single layer with the oracle. */
+bl_status bl_run_kernel(bl_ctx* ctx, int tenant, int kernel_idx, int lo, int hi);
+
+/* ---- offline profiler (L155-L161 §4.2.1; A2) ------------------------------------
+ * bl_profile_kernel: time kernel on logical SMs [0, sm_count) with CUDA events:
+ * median over 3 batches of the mean of 'reps' back-to-back launches; *d_out =
+ * distinct SMs used in an unrestricted run (R19).  bl_profile_tenant fills
+ * t[k][s] for every kernel and every s = 1..S.  Before bl_start. */
+bl_status bl_profile_kernel(bl_ctx* ctx, int tenant, int kernel_idx, int sm_count, int reps,
+                            int64_t* ns_out, int* d_out);
+bl_status bl_profile_tenant(bl_ctx* ctx, int tenant, int reps);
+/* Direct access to the table: t_ns has S entries (s = 1..S). */
+bl_status bl_set_profile_row(bl_ctx* ctx, int tenant, int kernel_idx, const int64_t* t_ns, int d);
+bl_status bl_get_profile_row(bl_ctx* ctx, int tenant, int kernel_idx, int64_t* t_ns, int* d);
+/* Text format documented in synth/profile.py.  bl_load_profile on a
+ * BL_DEVICE_NONE ctx with no tenants also registers the tenants and virtual
+ * kernels it describes. */
+bl_status bl_save_profile(bl_ctx* ctx, const char* path);
+bl_status bl_load_profile(bl_ctx* ctx, const char* path);
+/* Derived quantities (R18): SMs per tenant and tau/T (tau[k] at quota SMs). */
+bl_status bl_tenant_info(bl_ctx* ctx, int tenant, int* quota_sms, int* n_kernels, int64_t* T_iso_ns);
+
+/* ---- runtime ----------------------------------------------------------------------- */
+bl_status bl_start(bl_ctx* ctx);   /* spawns the scheduler/launch thread; requires a full profile */
+/* Submit one request (one pass over the tenant's kernel sequence).  WALL: any
+ * time after bl_start, arrival_ns = host clock of the arrival.  VIRTUAL: before
+ * bl_start, arrival_ns = trace time (non-decreasing per tenant). */
+bl_status bl_submit(bl_ctx* ctx, int tenant, int64_t arrival_ns, uint64_t* req_out);
+bl_status bl_poll(bl_ctx* ctx, uint64_t req, bl_req_info* out);    /* BL_OK / BL_PENDING */
+bl_status bl_drain(bl_ctx* ctx, int64_t timeout_ns);               /* all submitted finished */
+bl_status bl_stop(bl_ctx* ctx);
+/* Copy out decision records / launch records (from index 'first'). */
+bl_status bl_decisions(bl_ctx* ctx, size_t first, bl_decision* buf, size_t cap, size_t* n_out);
+bl_status bl_launches(bl_ctx* ctx, size_t first, bl_launch_rec* buf, size_t cap, size_t* n_out);
+/* Reset request table, logs and queues (between runs with the same tenants). */
+bl_status bl_reset(bl_ctx* ctx, const bl_params* params);
+
+/* ---- pure scheduler entry point (no ctx state; CPU parity) --------------------------
+ * decide() of the C++ scheduler on a loaded profile: active arrays of length
+ * n_active (tenant ids, arrivals, next kernel indices). */
+bl_status bl_decide(bl_ctx* ctx, int64_t now, int n_active, const int32_t* tenants,
+                    const int64_t* arrivals, const int32_t* next_kernel, bl_decision* out);
+
+int64_t bl_now_ns(void);
+const char* bl_last_error(void);
+const char* bl_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BLESS_BLESS_H */

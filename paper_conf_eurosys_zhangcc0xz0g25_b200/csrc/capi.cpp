@@ -1,0 +1,176 @@
+// capi.cpp -- extern "C" boundary (include/bless/bless.h).  Argument checks,
+// error strings and exception containment only; all logic is in Engine.
+#include <chrono>
+#include <exception>
+#include <string>
+
+#include "../../include/bless/bless.h"
+#include "runtime/engine.hpp"
+
+struct bl_ctx {
+  bless::Engine* eng;
+};
+
+static thread_local std::string g_err;
+
+#define GUARD(ctx)                                      \
+  if (!(ctx) || !(ctx)->eng) {                          \
+    g_err = "null ctx";                                 \
+    return BL_E_INVALID;                                \
+  }
+
+template <class F>
+static bl_status wrap(F&& f) {
+  try {
+    std::string err;
+    bl_status st = f(err);
+    if (st != BL_OK && st != BL_PENDING) g_err = err;
+    return st;
+  } catch (const std::bad_alloc&) {
+    g_err = "out of host memory";
+    return BL_E_OOM;
+  } catch (const std::exception& e) {
+    g_err = e.what();
+    return BL_E_INVALID;
+  } catch (...) {
+    g_err = "unknown exception";
+    return BL_E_INVALID;
+  }
+}
+
+extern "C" {
+
+void bl_params_default(bl_params* p) {
+  if (!p) return;
+  *p = bl_params{};
+  p->sm_unit = 4;
+  p->squad_max = 50;
+  p->split_pct = 50;
+  p->seed_all = 1;
+  p->policy = BL_POLICY_BLESS;
+  p->clock = BL_CLOCK_WALL;
+  p->squad_overhead_ns = 0;
+  p->temporal_period_ns = 2000000;
+  p->temporal_work_conserving = 0;
+  p->max_inflight_squads = 2;
+  p->lookahead_ns = 20000;
+  p->max_requests = 1 << 20;
+}
+
+bl_status bl_create(int device, const bl_params* params, void* ws, size_t ws_bytes, bl_ctx** out) {
+  if (!out) { g_err = "null out"; return BL_E_INVALID; }
+  *out = nullptr;
+  bl_params p;
+  bl_params_default(&p);
+  if (params) p = *params;
+  return wrap([&](std::string& err) {
+    bless::Engine* e = new bless::Engine(device, p);
+    bl_status st = e->init(ws, ws_bytes, err);
+    if (st != BL_OK) { delete e; return st; }
+    *out = new bl_ctx{e};
+    return BL_OK;
+  });
+}
+
+bl_status bl_destroy(bl_ctx* ctx) {
+  GUARD(ctx);
+  delete ctx->eng;
+  ctx->eng = nullptr;
+  delete ctx;
+  return BL_OK;
+}
+
+bl_status bl_device_info_get(bl_ctx* ctx, bl_device_info* out) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->device_info(out, e); });
+}
+bl_status bl_register_tenant(bl_ctx* ctx, double quota, const char* name, int* tenant_out) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->register_tenant(quota, name, tenant_out, e); });
+}
+bl_status bl_set_stream(bl_ctx* ctx, int tenant, void* s) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->set_stream(tenant, s, e); });
+}
+bl_status bl_append_kernel(bl_ctx* ctx, int tenant, const bl_op* op, int* k) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->append_kernel(tenant, op, k, e); });
+}
+bl_status bl_run_kernel(bl_ctx* ctx, int tenant, int k, int lo, int hi) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->run_kernel(tenant, k, lo, hi, e); });
+}
+bl_status bl_profile_kernel(bl_ctx* ctx, int tenant, int k, int sm_count, int reps, int64_t* ns, int* d) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->profile_kernel(tenant, k, sm_count, reps, ns, d, e); });
+}
+bl_status bl_profile_tenant(bl_ctx* ctx, int tenant, int reps) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->profile_tenant(tenant, reps, e); });
+}
+bl_status bl_set_profile_row(bl_ctx* ctx, int tenant, int k, const int64_t* t, int d) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->set_profile_row(tenant, k, t, d, e); });
+}
+bl_status bl_get_profile_row(bl_ctx* ctx, int tenant, int k, int64_t* t, int* d) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->get_profile_row(tenant, k, t, d, e); });
+}
+bl_status bl_save_profile(bl_ctx* ctx, const char* path) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->save_profile(path, e); });
+}
+bl_status bl_load_profile(bl_ctx* ctx, const char* path) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->load_profile(path, e); });
+}
+bl_status bl_tenant_info(bl_ctx* ctx, int tenant, int* qsms, int* m, int64_t* T) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->tenant_info(tenant, qsms, m, T, e); });
+}
+bl_status bl_start(bl_ctx* ctx) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->start(e); });
+}
+bl_status bl_submit(bl_ctx* ctx, int tenant, int64_t arrival_ns, uint64_t* req_out) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->submit(tenant, arrival_ns, req_out, e); });
+}
+bl_status bl_poll(bl_ctx* ctx, uint64_t req, bl_req_info* out) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->poll(req, out, e); });
+}
+bl_status bl_drain(bl_ctx* ctx, int64_t timeout_ns) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->drain(timeout_ns, e); });
+}
+bl_status bl_stop(bl_ctx* ctx) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->stop(e); });
+}
+bl_status bl_decisions(bl_ctx* ctx, size_t first, bl_decision* buf, size_t cap, size_t* n) {
+  GUARD(ctx);
+  return ctx->eng->decisions(first, buf, cap, n);
+}
+bl_status bl_launches(bl_ctx* ctx, size_t first, bl_launch_rec* buf, size_t cap, size_t* n) {
+  GUARD(ctx);
+  return ctx->eng->launches(first, buf, cap, n);
+}
+bl_status bl_reset(bl_ctx* ctx, const bl_params* p) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->reset(p, e); });
+}
+bl_status bl_decide(bl_ctx* ctx, int64_t now, int n, const int32_t* t, const int64_t* a, const int32_t* k,
+                    bl_decision* out) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->decide_pure(now, n, t, a, k, out, e); });
+}
+
+int64_t bl_now_ns(void) {
+  return std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now().time_since_epoch())
+      .count();
+}
+const char* bl_last_error(void) { return g_err.c_str(); }
+const char* bl_version(void) { return "blessb200 0.1 (sm_100a)"; }
+
+}  // extern "C"

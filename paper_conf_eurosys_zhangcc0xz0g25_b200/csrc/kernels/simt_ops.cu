@@ -1,0 +1,462 @@
+// simt_ops.cu -- CUDA-core tenant kernels under the SM-gated executor.
+//
+//  * SimtMM: tiled fp32-accumulate GEMM / implicit-GEMM convolution (NHWC
+//    input, KRSC weights) with the fused epilogue act(acc*scale+shift+R).
+//    This is the fp32 path of config C1 (1e-4 parity) and
+//    the generic fallback for shapes the tcgen05 path does not take.
+//  * Pool: max / avg / global-average pooling, NHWC (K8).
+//  * Eltwise: per-channel affine + activation (+ residual) (K7/K12).
+//  * Gemv: M <= 8 rows (batch-1 FC layers): HBM-bound, 16-byte vector loads,
+//    split over N rows and K chunks (K2 GEMV shapes).
+// The tenants' layers come from the paper's applications (PAPER.md L259,
+// L284); semantics as in oracle/layers_ref.py.
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+
+#include "../runtime/kdesc.hpp"
+#include "executor.cuh"
+
+namespace bless {
+
+template <typename T>
+__device__ __forceinline__ float ldf(const T* p);
+template <>
+__device__ __forceinline__ float ldf<float>(const float* p) { return __ldg(p); }
+template <>
+__device__ __forceinline__ float ldf<__nv_bfloat16>(const __nv_bfloat16* p) { return __bfloat162float(*p); }
+template <typename T>
+__device__ __forceinline__ void stf(T* p, float v);
+template <>
+__device__ __forceinline__ void stf<float>(float* p, float v) { *p = v; }
+template <>
+__device__ __forceinline__ void stf<__nv_bfloat16>(__nv_bfloat16* p, float v) { *p = __float2bfloat16_rn(v); }
+
+__device__ __forceinline__ float apply_act(float y, int act) {
+  switch (act) {
+    case BL_ACT_RELU: return fmaxf(y, 0.f);
+    case BL_ACT_RELU6: return fminf(fmaxf(y, 0.f), 6.f);
+    case BL_ACT_GELU: return 0.5f * y * (1.f + erff(y * 0.70710678118654752f));
+    default: return y;
+  }
+}
+
+// ---------------------------------------------------------------------------
+// SimtMM
+// ---------------------------------------------------------------------------
+struct SimtMMParams {
+  const void* X;
+  const void* W;
+  const float* scale;
+  const float* shift;
+  const void* R;
+  void* Y;
+  int M, N, K;
+  int ldx, ldy, ldr;
+  int act, conv;
+  int H, Wd, C, OH, OW, R_, S_, stride, pad;
+  int tiles_n;
+};
+
+constexpr int kMMB = 32;      // BM = BN = BK
+constexpr int kMMThreads = 256;
+
+template <typename T>
+struct SimtMM {
+  using Params = SimtMMParams;
+  __device__ static float loadA(const Params& p, int m, int k) {
+    const T* X = (const T*)p.X;
+    if (!p.conv) return ldf(X + (size_t)m * p.ldx + k);
+    const int hw = p.OH * p.OW;
+    const int n = m / hw, pix = m - n * hw;
+    const int oh = pix / p.OW, ow = pix - oh * p.OW;
+    const int sc = p.S_ * p.C;
+    const int r = k / sc, rem = k - r * sc;
+    const int s = rem / p.C, c = rem - s * p.C;
+    const int ih = oh * p.stride - p.pad + r, iw = ow * p.stride - p.pad + s;
+    if (ih < 0 || ih >= p.H || iw < 0 || iw >= p.Wd) return 0.f;
+    return ldf(X + ((size_t)(n * p.H + ih) * p.Wd + iw) * p.ldx + c);
+  }
+  __device__ static void tile(const Params& p, int t, unsigned char* smem) {
+    float(*As)[kMMB + 1] = reinterpret_cast<float(*)[kMMB + 1]>(smem);
+    float(*Bs)[kMMB + 1] = reinterpret_cast<float(*)[kMMB + 1]>(smem + sizeof(float) * kMMB * (kMMB + 1));
+    const int tm = t / p.tiles_n, tn = t - tm * p.tiles_n;
+    const int m0 = tm * kMMB, n0 = tn * kMMB;
+    const int tid = threadIdx.x, ty = tid >> 4, tx = tid & 15;
+    const T* W = (const T*)p.W;
+    float acc[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
+    for (int k0 = 0; k0 < p.K; k0 += kMMB) {
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int idx = tid + i * kMMThreads;
+        const int r = idx >> 5, c = idx & 31;
+        const int m = m0 + r, n = n0 + r, k = k0 + c;
+        As[c][r] = (m < p.M && k < p.K) ? loadA(p, m, k) : 0.f;
+        Bs[c][r] = (n < p.N && k < p.K) ? ldf(W + (size_t)n * p.K + k) : 0.f;
+      }
+      __syncthreads();
+#pragma unroll 8
+      for (int kk = 0; kk < kMMB; ++kk) {
+        const float a0 = As[kk][ty * 2], a1 = As[kk][ty * 2 + 1];
+        const float b0 = Bs[kk][tx * 2], b1 = Bs[kk][tx * 2 + 1];
+        acc[0][0] = fmaf(a0, b0, acc[0][0]);
+        acc[0][1] = fmaf(a0, b1, acc[0][1]);
+        acc[1][0] = fmaf(a1, b0, acc[1][0]);
+        acc[1][1] = fmaf(a1, b1, acc[1][1]);
+      }
+      __syncthreads();
+    }
+    T* Y = (T*)p.Y;
+    const T* Rr = (const T*)p.R;
+#pragma unroll
+    for (int i = 0; i < 2; ++i)
+#pragma unroll
+      for (int j = 0; j < 2; ++j) {
+        const int m = m0 + ty * 2 + i, n = n0 + tx * 2 + j;
+        if (m >= p.M || n >= p.N) continue;
+        float y = acc[i][j];
+        if (p.scale) y *= __ldg(p.scale + n);
+        if (p.shift) y += __ldg(p.shift + n);
+        if (Rr) y += ldf(Rr + (size_t)m * p.ldr + n);
+        stf(Y + (size_t)m * p.ldy + n, apply_act(y, p.act));
+      }
+  }
+};
+
+// ---------------------------------------------------------------------------
+// Pool
+// ---------------------------------------------------------------------------
+struct PoolParams {
+  const void* X;
+  void* Y;
+  int Nb, H, W, C, OH, OW, k, stride, pad, mode;
+  int pix_per_tile, total_pix;
+};
+
+template <typename T>
+struct Pool {
+  using Params = PoolParams;
+  __device__ static void tile(const Params& p, int t, unsigned char*) {
+    const T* X = (const T*)p.X;
+    T* Y = (T*)p.Y;
+    if (p.mode == BL_POOL_GLOBAL_AVG) {
+      // tile = (image, 256-channel chunk)
+      const int cchunks = (p.C + 255) / 256;
+      const int n = t / cchunks, c = (t - n * cchunks) * 256 + threadIdx.x;
+      if (c >= p.C || threadIdx.x >= 256) return;
+      float s = 0.f;
+      const int hw = p.H * p.W;
+      for (int i = 0; i < hw; ++i) s += ldf(X + ((size_t)n * hw + i) * p.C + c);
+      stf(Y + (size_t)n * p.C + c, s / (float)hw);
+      return;
+    }
+    const int p0 = t * p.pix_per_tile;
+    const int npix = min(p.pix_per_tile, p.total_pix - p0);
+    for (int idx = threadIdx.x; idx < npix * p.C; idx += blockDim.x) {
+      const int pl = idx / p.C, c = idx - pl * p.C;
+      const int pix = p0 + pl;
+      const int n = pix / (p.OH * p.OW), q = pix - n * p.OH * p.OW;
+      const int oh = q / p.OW, ow = q - oh * p.OW;
+      float acc = (p.mode == BL_POOL_MAX) ? -INFINITY : 0.f;
+      for (int r = 0; r < p.k; ++r) {
+        const int ih = oh * p.stride - p.pad + r;
+        for (int s = 0; s < p.k; ++s) {
+          const int iw = ow * p.stride - p.pad + s;
+          if (ih < 0 || ih >= p.H || iw < 0 || iw >= p.W) continue;  // max: -inf pad; avg: 0 pad
+          const float v = ldf(X + ((size_t)(n * p.H + ih) * p.W + iw) * p.C + c);
+          acc = (p.mode == BL_POOL_MAX) ? fmaxf(acc, v) : acc + v;
+        }
+      }
+      if (p.mode == BL_POOL_AVG) acc /= (float)(p.k * p.k);  // count_include_pad
+      stf(Y + (size_t)pix * p.C + c, acc);
+    }
+  }
+};
+
+// ---------------------------------------------------------------------------
+// Eltwise: Y[r, c] = act(X*scale[c] + shift[c] + R)
+// ---------------------------------------------------------------------------
+struct EltParams {
+  const void* X;
+  const float* scale;
+  const float* shift;
+  const void* R;
+  void* Y;
+  long long total;
+  int C, act, per_tile;
+};
+
+template <typename T>
+struct Eltwise {
+  using Params = EltParams;
+  __device__ static void tile(const Params& p, int t, unsigned char*) {
+    const long long e0 = (long long)t * p.per_tile;
+    const long long e1 = min(e0 + p.per_tile, p.total);
+    const T* X = (const T*)p.X;
+    const T* R = (const T*)p.R;
+    T* Y = (T*)p.Y;
+    for (long long e = e0 + threadIdx.x; e < e1; e += blockDim.x) {
+      const int c = (int)(e % p.C);
+      float y = ldf(X + e);
+      if (p.scale) y *= __ldg(p.scale + c);
+      if (p.shift) y += __ldg(p.shift + c);
+      if (R) y += ldf(R + e);
+      stf(Y + e, apply_act(y, p.act));
+    }
+  }
+};
+
+// ---------------------------------------------------------------------------
+// Gemv: Y[m, n] for m < M <= 8; tile = (row block of 8 outputs, K split).
+// Each warp owns one output row n and streams W[n, k-chunk] with 16-byte
+// loads; partial sums of a split-K tile are combined by atomics into an fp32
+// workspace and the last split applies the epilogue (counter per row block).
+// ---------------------------------------------------------------------------
+struct GemvParams {
+  const void* X;
+  const void* W;
+  const float* scale;
+  const float* shift;
+  const void* R;
+  void* Y;
+  int M, N, K, ldx, ldy, ldr, act;
+  int rows_per_tile, ksplit, kchunk;
+  float* ws;          // [M, N] fp32 partial sums (zeroed)
+  unsigned* cnt;      // [row blocks] arrival counters (zeroed)
+};
+
+template <typename T>
+struct Gemv {
+  using Params = GemvParams;
+  static constexpr int kVec = 16 / sizeof(T);
+  __device__ static void tile(const Params& p, int t, unsigned char*) {
+    const int rb = t / p.ksplit, ks = t - rb * p.ksplit;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int nwarps = blockDim.x >> 5;
+    const int k0 = ks * p.kchunk, k1 = min(p.K, k0 + p.kchunk);
+    const T* X = (const T*)p.X;
+    const T* W = (const T*)p.W;
+    for (int rr = warp; rr < p.rows_per_tile; rr += nwarps) {
+      const int n = rb * p.rows_per_tile + rr;
+      if (n >= p.N) break;
+      float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+      const T* wrow = W + (size_t)n * p.K;
+      int k = k0 + lane * kVec;
+      const bool vec_ok = ((p.K % kVec) == 0) && ((k0 % kVec) == 0);
+      if (vec_ok) {
+        for (; k + kVec <= k1; k += 32 * kVec) {
+          const uint4 wv = __ldg(reinterpret_cast<const uint4*>(wrow + k));
+          const T* we = reinterpret_cast<const T*>(&wv);
+#pragma unroll
+          for (int m = 0; m < 8; ++m) {
+            if (m >= p.M) break;
+            const T* xr = X + (size_t)m * p.ldx + k;
+            float s = 0.f;
+#pragma unroll
+            for (int v = 0; v < kVec; ++v) s = fmaf(ldf(we + v), ldf(xr + v), s);
+            acc[m] += s;
+          }
+        }
+      } else {
+        for (k = k0 + lane; k < k1; k += 32) {
+          const float w = ldf(wrow + k);
+          for (int m = 0; m < p.M && m < 8; ++m) acc[m] = fmaf(w, ldf(X + (size_t)m * p.ldx + k), acc[m]);
+        }
+      }
+      for (int m = 0; m < p.M && m < 8; ++m) {
+        float v = acc[m];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        acc[m] = v;
+      }
+      if (p.ksplit == 1) {
+        if (lane == 0) {
+          for (int m = 0; m < p.M; ++m) {
+            float y = acc[m];
+            if (p.scale) y *= __ldg(p.scale + n);
+            if (p.shift) y += __ldg(p.shift + n);
+            if (p.R) y += ldf((const T*)p.R + (size_t)m * p.ldr + n);
+            stf((T*)p.Y + (size_t)m * p.ldy + n, apply_act(y, p.act));
+          }
+        }
+      } else if (lane == 0) {
+        for (int m = 0; m < p.M; ++m) atomicAdd(p.ws + (size_t)m * p.N + n, acc[m]);
+      }
+    }
+    if (p.ksplit > 1) {
+      __shared__ unsigned s_last;
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        __threadfence();
+        s_last = (atomicAdd(p.cnt + rb, 1u) == (unsigned)p.ksplit - 1);
+      }
+      __syncthreads();
+      if (s_last) {
+        __threadfence();
+        const int nb0 = rb * p.rows_per_tile;
+        for (int i = threadIdx.x; i < p.rows_per_tile * p.M; i += blockDim.x) {
+          const int rr = i % p.rows_per_tile, m = i / p.rows_per_tile;
+          const int n = nb0 + rr;
+          if (n >= p.N) continue;
+          volatile float* wsv = p.ws + (size_t)m * p.N + n;
+          float y = *wsv;
+          *wsv = 0.f;  // leave the workspace zeroed for the next launch
+          if (p.scale) y *= __ldg(p.scale + n);
+          if (p.shift) y += __ldg(p.shift + n);
+          if (p.R) y += ldf((const T*)p.R + (size_t)m * p.ldr + n);
+          stf((T*)p.Y + (size_t)m * p.ldy + n, apply_act(y, p.act));
+        }
+        if (threadIdx.x == 0) p.cnt[rb] = 0;
+      }
+    }
+  }
+};
+
+// ---------------------------------------------------------------------------
+// gated kernels + launchers
+// ---------------------------------------------------------------------------
+template <class Op>
+__global__ void __launch_bounds__(256) k_gated(const typename Op::Params p, const GateArgs g) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  gated_run<Op>(p, g, smem);
+}
+
+template <class Op>
+static cudaError_t launch_gated(const KernelDesc& d, const GateArgs& g, cudaStream_t st) {
+  void* args[2] = {(void*)d.params, (void*)&g};
+  return cudaLaunchKernel((const void*)k_gated<Op>, dim3(d.grid), dim3(d.block), args, (size_t)d.smem, st);
+}
+
+static inline size_t esize(int dt) { return dt == BL_BF16 ? 2 : 4; }
+
+// Gemv split-K workspace: one static pool per process (zero-initialised, each
+// launch leaves it zeroed).  Kernels of the same tenant never run
+// concurrently (one stream), but different tenants may: give every Gemv
+// kernel its own region.
+static float* gemv_ws_alloc(size_t floats, size_t counters, unsigned** cnt_out) {
+  void* p = nullptr;
+  if (cudaMalloc(&p, floats * 4 + counters * 4) != cudaSuccess) return nullptr;
+  cudaMemset(p, 0, floats * 4 + counters * 4);
+  *cnt_out = reinterpret_cast<unsigned*>(reinterpret_cast<char*>(p) + floats * 4);
+  return reinterpret_cast<float*>(p);
+}
+
+bool build_simt(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::string& err) {
+  const bool bf = op.dtype == BL_BF16;
+  if (op.dtype != BL_F32 && op.dtype != BL_BF16) { err = "dtype"; return false; }
+  const int occ = 2;
+  d.block = 256;
+  d.grid = caps.S * occ;
+  d.op = op;
+  if (op.kind == BL_OP_GEMM || op.kind == BL_OP_CONV) {
+    SimtMMParams p{};
+    p.X = op.ptr[0]; p.W = op.ptr[1]; p.scale = (const float*)op.ptr[2]; p.shift = (const float*)op.ptr[3];
+    p.R = op.ptr[4]; p.Y = op.ptr[5]; p.act = op.act;
+    if (op.kind == BL_OP_GEMM) {
+      p.M = (int)op.dims[0]; p.N = (int)op.dims[1]; p.K = (int)op.dims[2];
+      p.ldx = op.dims[3] ? (int)op.dims[3] : p.K;
+      p.ldy = op.dims[4] ? (int)op.dims[4] : p.N;
+      p.ldr = op.dims[5] ? (int)op.dims[5] : p.N;
+      p.conv = 0;
+      if (p.M <= 8 && p.M >= 1) {
+        // batch-1 FC layer: HBM-bound GEMV path
+        GemvParams q{};
+        q.X = p.X; q.W = p.W; q.scale = p.scale; q.shift = p.shift; q.R = p.R; q.Y = p.Y;
+        q.M = p.M; q.N = p.N; q.K = p.K; q.ldx = p.ldx; q.ldy = p.ldy; q.ldr = p.ldr; q.act = p.act;
+        q.rows_per_tile = 8;
+        const int rblocks = (q.N + 7) / 8;
+        // split K so there are >= ~2 tiles per SM when K is long
+        int ks = 1;
+        while ((long long)rblocks * ks < 2LL * caps.S && q.K / (ks * 2) >= 1024) ks *= 2;
+        q.ksplit = ks;
+        const int vec = bf ? 8 : 4;
+        q.kchunk = ((q.K + ks - 1) / ks + vec - 1) / vec * vec;
+        if (ks > 1) {
+          q.ws = gemv_ws_alloc((size_t)q.M * q.N, rblocks, &q.cnt);
+          if (!q.ws) { err = "gemv workspace alloc"; return false; }
+        }
+        d.tiles = (uint32_t)(rblocks * ks);
+        d.smem = 0;
+        std::memcpy(d.params, &q, sizeof(q));
+        d.launch = bf ? launch_gated<Gemv<__nv_bfloat16>> : launch_gated<Gemv<float>>;
+        d.family = bf ? "gemv_bf16" : "gemv_f32";
+        d.flops = 2.0 * q.M * q.N * q.K;
+        d.bytes = esize(op.dtype) * ((double)q.N * q.K + (double)q.M * q.K + (double)q.M * q.N);
+        return true;
+      }
+    } else {
+      const int Nb = (int)op.dims[0], H = (int)op.dims[1], Wd = (int)op.dims[2], C = (int)op.dims[3];
+      const int K = (int)op.dims[4], R = (int)op.dims[5], S = (int)op.dims[6];
+      const int stride = (int)op.dims[7], pad = (int)op.dims[8], groups = (int)op.dims[9];
+      if (groups != 1) { err = "simt conv supports groups == 1 only"; return false; }
+      if (stride < 1 || R < 1 || S < 1 || C < 1 || K < 1 || Nb < 1) { err = "conv dims"; return false; }
+      p.H = H; p.Wd = Wd; p.C = C; p.R_ = R; p.S_ = S; p.stride = stride; p.pad = pad;
+      p.OH = (H + 2 * pad - R) / stride + 1;
+      p.OW = (Wd + 2 * pad - S) / stride + 1;
+      p.M = Nb * p.OH * p.OW; p.N = K; p.K = R * S * C;
+      p.ldx = op.dims[10] ? (int)op.dims[10] : C;
+      p.ldy = op.dims[11] ? (int)op.dims[11] : K;
+      p.ldr = p.ldy;
+      p.conv = 1;
+    }
+    if (p.M < 0 || p.N < 1 || p.K < 1) { err = "gemm dims"; return false; }
+    p.tiles_n = (p.N + kMMB - 1) / kMMB;
+    d.tiles = (uint32_t)(((p.M + kMMB - 1) / kMMB) * p.tiles_n);
+    d.smem = 2 * sizeof(float) * kMMB * (kMMB + 1);
+    std::memcpy(d.params, &p, sizeof(p));
+    d.launch = bf ? launch_gated<SimtMM<__nv_bfloat16>> : launch_gated<SimtMM<float>>;
+    d.family = bf ? "simt_mm_bf16" : "simt_mm_f32";
+    d.flops = 2.0 * p.M * p.N * p.K;
+    d.bytes = esize(op.dtype) * ((double)p.N * p.K + (double)p.M * p.N * (p.R ? 2 : 1) +
+                                 (op.kind == BL_OP_CONV ? (double)op.dims[0] * op.dims[1] * op.dims[2] * op.dims[3]
+                                                        : (double)p.M * p.K));
+    return true;
+  }
+  if (op.kind == BL_OP_POOL) {
+    PoolParams p{};
+    p.X = op.ptr[0]; p.Y = op.ptr[1];
+    p.Nb = (int)op.dims[0]; p.H = (int)op.dims[1]; p.W = (int)op.dims[2]; p.C = (int)op.dims[3];
+    p.k = (int)op.dims[4]; p.stride = (int)op.dims[5]; p.pad = (int)op.dims[6]; p.mode = (int)op.dims[7];
+    if (p.mode == BL_POOL_GLOBAL_AVG) {
+      p.OH = p.OW = 1;
+      d.tiles = (uint32_t)(p.Nb * ((p.C + 255) / 256));
+    } else {
+      if (p.k < 1 || p.stride < 1) { err = "pool dims"; return false; }
+      p.OH = (p.H + 2 * p.pad - p.k) / p.stride + 1;
+      p.OW = (p.W + 2 * p.pad - p.k) / p.stride + 1;
+      p.total_pix = p.Nb * p.OH * p.OW;
+      p.pix_per_tile = std::max(1, 4096 / std::max(1, p.C));
+      d.tiles = (uint32_t)((p.total_pix + p.pix_per_tile - 1) / p.pix_per_tile);
+    }
+    d.smem = 0;
+    std::memcpy(d.params, &p, sizeof(p));
+    d.launch = bf ? launch_gated<Pool<__nv_bfloat16>> : launch_gated<Pool<float>>;
+    d.family = bf ? "pool_bf16" : "pool_f32";
+    d.bytes = esize(op.dtype) * ((double)p.Nb * p.H * p.W * p.C + (double)p.Nb * p.OH * p.OW * p.C);
+    return true;
+  }
+  if (op.kind == BL_OP_ELTWISE) {
+    EltParams p{};
+    p.X = op.ptr[0]; p.scale = (const float*)op.ptr[1]; p.shift = (const float*)op.ptr[2]; p.R = op.ptr[3];
+    p.Y = op.ptr[4];
+    p.total = op.dims[0] * op.dims[1];
+    p.C = (int)op.dims[1];
+    p.act = op.act;
+    p.per_tile = 8192;
+    if (p.C < 1) { err = "eltwise dims"; return false; }
+    d.tiles = (uint32_t)((p.total + p.per_tile - 1) / p.per_tile);
+    d.smem = 0;
+    std::memcpy(d.params, &p, sizeof(p));
+    d.launch = bf ? launch_gated<Eltwise<__nv_bfloat16>> : launch_gated<Eltwise<float>>;
+    d.family = bf ? "eltwise_bf16" : "eltwise_f32";
+    d.bytes = esize(op.dtype) * (double)p.total * (p.R ? 3 : 2);
+    return true;
+  }
+  err = "unsupported op kind";
+  return false;
+}
+
+}  // namespace bless

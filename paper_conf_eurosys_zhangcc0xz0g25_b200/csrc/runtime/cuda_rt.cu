@@ -1,0 +1,316 @@
+// cuda_rt.cu -- see cuda_rt.hpp.
+#include "cuda_rt.hpp"
+
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <cstring>
+#include <thread>
+
+#include "../kernels/executor.cuh"
+
+namespace bless {
+
+static int64_t host_now_ns() {
+  return std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now().time_since_epoch())
+      .count();
+}
+
+#define RT_CHECK(call)                                                          \
+  do {                                                                          \
+    cudaError_t e_ = (call);                                                    \
+    if (e_ != cudaSuccess) {                                                    \
+      err = std::string(#call) + ": " + cudaGetErrorString(e_);                 \
+      return false;                                                             \
+    }                                                                           \
+  } while (0)
+
+// ---------------------------------------------------------------- probe kernels (A1)
+__global__ void k_probe_smid(unsigned* seen, unsigned* nsmid_out) {
+  const uint32_t sm = ptx_smid();
+  if (threadIdx.x == 0) {
+    atomicOr(&seen[(sm >> 5) & 7], 1u << (sm & 31));
+    uint32_t n;
+    asm volatile("mov.u32 %0, %%nsmid;" : "=r"(n));
+    atomicMax(nsmid_out, n);
+  }
+}
+
+__global__ void __cluster_dims__(2, 1, 1) k_probe_pairs(int* out) {
+  if (threadIdx.x == 0) out[blockIdx.x] = (int)ptx_smid();
+}
+
+__global__ void k_clock(unsigned long long* out) {
+  if (threadIdx.x == 0) {
+    const unsigned long long t = ptx_globaltimer();
+    *(volatile unsigned long long*)out = t;
+    __threadfence_system();
+  }
+}
+
+__global__ void k_gt_res(long long* out) {
+  uint64_t prev = ptx_globaltimer();
+  long long best = 1LL << 40;
+  for (int i = 0; i < 20000; ++i) {
+    const uint64_t t = ptx_globaltimer();
+    if (t != prev) {
+      best = min(best, (long long)(t - prev));
+      prev = t;
+    }
+  }
+  *out = best;
+}
+
+// ---------------------------------------------------------------- kernel dispatch
+bool build_kernel(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err) {
+  if (op.kind == BL_OP_VIRTUAL) { err = "virtual op on a device ctx"; return false; }
+  std::string e2;
+  if (op.dtype == BL_BF16 && (op.kind == BL_OP_GEMM || op.kind == BL_OP_CONV)) {
+    if (build_tc_gemm(op, caps, out, e2)) return true;
+    if (!e2.empty()) { err = e2; return false; }
+  }
+  return build_simt(op, caps, out, err);
+}
+
+// ---------------------------------------------------------------- DeviceRT
+std::unique_ptr<DeviceRT> DeviceRT::create(int device, void* ws, size_t ws_bytes, std::string& err) {
+  std::unique_ptr<DeviceRT> rt(new DeviceRT());
+  rt->device_ = device;
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || device < 0 || device >= ndev) {
+    err = std::string("no CUDA device ") + std::to_string(device) + " (" + cudaGetErrorString(e) + ")";
+    return nullptr;
+  }
+  if (cudaSetDevice(device) != cudaSuccess) { err = "cudaSetDevice"; return nullptr; }
+  cudaDeviceProp prop{};
+  cudaGetDeviceProperties(&prop, device);
+  rt->info_.device = device;
+  rt->info_.sm_count = prop.multiProcessorCount;
+  rt->info_.cc_major = prop.major;
+  rt->info_.cc_minor = prop.minor;
+  rt->info_.l2_bytes = prop.l2CacheSize;
+  rt->info_.smem_per_block_optin = (int64_t)prop.sharedMemPerBlockOptin;
+  rt->caps_.S = prop.multiProcessorCount;
+  rt->caps_.cc_major = prop.major;
+  rt->caps_.cc_minor = prop.minor;
+  rt->caps_.smem_optin = (int)prop.sharedMemPerBlockOptin;
+  const size_t slot_bytes = kSlotRing * sizeof(DevSlot);
+  if (ws && ws_bytes >= slot_bytes) {
+    rt->slots_ = ws;
+    rt->own_slots_ = false;
+  } else {
+    if (cudaMalloc(&rt->slots_, slot_bytes) != cudaSuccess) { err = "cudaMalloc slots"; return nullptr; }
+    rt->own_slots_ = true;
+  }
+  if (cudaMemset(rt->slots_, 0, slot_bytes) != cudaSuccess) { err = "memset slots"; return nullptr; }
+  if (cudaHostAlloc(&rt->stats_host_, kSlotRing * sizeof(SlotStats), cudaHostAllocMapped) != cudaSuccess) {
+    err = "cudaHostAlloc stats";
+    return nullptr;
+  }
+  std::memset(rt->stats_host_, 0, kSlotRing * sizeof(SlotStats));
+  if (cudaHostGetDevicePointer(&rt->stats_dev_, rt->stats_host_, 0) != cudaSuccess) {
+    err = "cudaHostGetDevicePointer";
+    return nullptr;
+  }
+  if (!rt->probe(err)) return nullptr;
+  if (!rt->calibrate_clock(err)) return nullptr;
+  return rt;
+}
+
+DeviceRT::~DeviceRT() {
+  cudaSetDevice(device_);
+  cudaDeviceSynchronize();
+  if (own_slots_ && slots_) cudaFree(slots_);
+  if (stats_host_) cudaFreeHost(stats_host_);
+  if (lid_map_dev_) cudaFree(lid_map_dev_);
+}
+
+bool DeviceRT::set_device() { return cudaSetDevice(device_) == cudaSuccess; }
+
+bool DeviceRT::probe(std::string& err) {
+  unsigned* d = nullptr;
+  RT_CHECK(cudaMalloc(&d, 64));
+  RT_CHECK(cudaMemset(d, 0, 64));
+  const int S = info_.sm_count;
+  k_probe_smid<<<S * 16, 64>>>(d, d + 8);
+  RT_CHECK(cudaGetLastError());
+  unsigned h[9];
+  RT_CHECK(cudaMemcpy(h, d, 36, cudaMemcpyDeviceToHost));
+  std::vector<int> smids;
+  for (int i = 0; i < 256; ++i)
+    if (h[i >> 5] & (1u << (i & 31))) smids.push_back(i);
+  info_.max_smid = (int)h[8] - 1;
+  std::memset(info_.smid_to_lid, 255, 256);
+  // Logical order = ascending %smid (TPC siblings are adjacent ids).
+  for (size_t i = 0; i < smids.size(); ++i) info_.smid_to_lid[smids[i]] = (uint8_t)i;
+  identity_map_ = true;
+  for (size_t i = 0; i < smids.size(); ++i)
+    if (smids[i] != (int)i) identity_map_ = false;
+  if ((int)smids.size() != S) {
+    err = "probe saw " + std::to_string(smids.size()) + " SMs, expected " + std::to_string(S);
+    cudaFree(d);
+    return false;
+  }
+  RT_CHECK(cudaMalloc(&lid_map_dev_, 256));
+  RT_CHECK(cudaMemcpy(lid_map_dev_, info_.smid_to_lid, 256, cudaMemcpyHostToDevice));
+  // TPC pairs via 2-CTA clusters (informational: siblings whose ids differ by one).
+  int* pr = nullptr;
+  const int npairs = (S / 2) * 2;
+  RT_CHECK(cudaMalloc(&pr, sizeof(int) * npairs));
+  k_probe_pairs<<<npairs, 32>>>(pr);
+  if (cudaGetLastError() == cudaSuccess) {
+    std::vector<int> hp(npairs);
+    cudaMemcpy(hp.data(), pr, sizeof(int) * npairs, cudaMemcpyDeviceToHost);
+    int ok = 0;
+    for (int i = 0; i + 1 < npairs; i += 2)
+      if ((hp[i] ^ hp[i + 1]) == 1) ok++;
+    info_.tpc_pairs_found = ok;
+  }
+  cudaFree(pr);
+  long long* r = nullptr;
+  RT_CHECK(cudaMalloc(&r, 8));
+  k_gt_res<<<1, 1>>>(r);
+  long long res = 0;
+  RT_CHECK(cudaMemcpy(&res, r, 8, cudaMemcpyDeviceToHost));
+  info_.globaltimer_res_ns = res;
+  cudaFree(r);
+  cudaFree(d);
+  return true;
+}
+
+bool DeviceRT::calibrate_clock(std::string& err) {
+  unsigned long long* hp = nullptr;
+  RT_CHECK(cudaHostAlloc((void**)&hp, 64, cudaHostAllocMapped));
+  unsigned long long* dp = nullptr;
+  RT_CHECK(cudaHostGetDevicePointer((void**)&dp, hp, 0));
+  cudaStream_t s;
+  RT_CHECK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  int64_t best_span = INT64_MAX, best_off = 0;
+  for (int it = 0; it < 9; ++it) {
+    *(volatile unsigned long long*)hp = 0;
+    const int64_t t0 = host_now_ns();
+    k_clock<<<1, 32, 0, s>>>(dp);
+    while (*(volatile unsigned long long*)hp == 0) {
+    }
+    const int64_t t1 = host_now_ns();
+    const int64_t gt = (int64_t) * (volatile unsigned long long*)hp;
+    // the kernel ran between t0 + launch latency and t1 - visibility latency;
+    // attribute the stamp to 3/4 of the span (launch latency dominates).
+    const int64_t est = t0 + (t1 - t0) * 3 / 4;
+    if (t1 - t0 < best_span) {
+      best_span = t1 - t0;
+      best_off = gt - est;
+    }
+  }
+  cudaStreamSynchronize(s);
+  cudaStreamDestroy(s);
+  cudaFreeHost(hp);
+  info_.clock_offset_ns = best_off;
+  return true;
+}
+
+int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
+  std::unique_ptr<KernelDesc> kd(new KernelDesc());
+  if (!build_kernel(op, caps_, *kd, err)) return -1;
+  kernels_.push_back(std::move(kd));
+  return (int)kernels_.size() - 1;
+}
+
+uint64_t DeviceRT::launch(int h, int lo, int hi, void* stream, std::string& err) {
+  const KernelDesc& kd = *kernels_[h];
+  const uint64_t seq = ++seq_;
+  const uint64_t slot = seq % kSlotRing;
+  GateArgs g;
+  g.slot = reinterpret_cast<DevSlot*>(slots_) + slot;
+  g.stats = reinterpret_cast<SlotStats*>(stats_dev_) + slot;
+  g.lid_map = identity_map_ ? nullptr : lid_map_dev_;
+  g.seq = seq;
+  g.tiles = kd.tiles;
+  g.lo = lo;
+  g.hi = hi;
+  const cudaError_t e = kd.launch(kd, g, (cudaStream_t)stream);
+  if (e != cudaSuccess) {
+    err = std::string("launch ") + kd.family + ": " + cudaGetErrorString(e);
+    return 0;
+  }
+  return seq;
+}
+
+bool DeviceRT::poll(uint64_t seq, LaunchStats* out) const {
+  const volatile SlotStats* s = reinterpret_cast<const volatile SlotStats*>(stats_host_) + (seq % kSlotRing);
+  if (s->seq != seq) return false;
+  std::atomic_thread_fence(std::memory_order_acquire);
+  if (out) {
+    out->start_host = gt_to_host(s->start_gt);
+    out->end_host = gt_to_host(s->end_gt);
+    out->nsm = (int)s->nsm;
+    out->fallback = (int)(s->flags & 1u);
+  }
+  return true;
+}
+
+void* DeviceRT::stream_create() {
+  cudaStream_t s = nullptr;
+  cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
+  return s;
+}
+void DeviceRT::stream_destroy(void* s) { cudaStreamDestroy((cudaStream_t)s); }
+void* DeviceRT::event_create() {
+  cudaEvent_t e = nullptr;
+  cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+  return e;
+}
+void DeviceRT::event_destroy(void* e) { cudaEventDestroy((cudaEvent_t)e); }
+bool DeviceRT::event_record(void* e, void* s) { return cudaEventRecord((cudaEvent_t)e, (cudaStream_t)s) == cudaSuccess; }
+bool DeviceRT::stream_wait(void* s, void* e) {
+  return cudaStreamWaitEvent((cudaStream_t)s, (cudaEvent_t)e, 0) == cudaSuccess;
+}
+int DeviceRT::event_query(void* e) {
+  const cudaError_t r = cudaEventQuery((cudaEvent_t)e);
+  if (r == cudaSuccess) return 1;
+  if (r == cudaErrorNotReady) return 0;
+  return -1;
+}
+bool DeviceRT::stream_sync(void* s) { return cudaStreamSynchronize((cudaStream_t)s) == cudaSuccess; }
+bool DeviceRT::device_sync() { return cudaDeviceSynchronize() == cudaSuccess; }
+
+bool DeviceRT::profile(int h, int sm_count, int reps, void* stream, int64_t* ns_out, int* d_out, std::string& err) {
+  cudaStream_t s = (cudaStream_t)stream;
+  cudaEvent_t e0, e1;
+  RT_CHECK(cudaEventCreate(&e0));
+  RT_CHECK(cudaEventCreate(&e1));
+  const int S = info_.sm_count;
+  sm_count = std::max(1, std::min(sm_count, S));
+  reps = std::max(1, reps);
+  if (d_out) {
+    const uint64_t q = launch(h, 0, S, s, err);
+    if (!q) return false;
+    RT_CHECK(cudaStreamSynchronize(s));
+    LaunchStats st{};
+    int spins = 0;
+    while (!poll(q, &st) && spins++ < 1000000) {
+    }
+    *d_out = std::max(1, st.nsm);
+  }
+  for (int w = 0; w < 2; ++w)
+    if (!launch(h, 0, sm_count, s, err)) return false;
+  float ms[3];
+  for (int b = 0; b < 3; ++b) {
+    RT_CHECK(cudaEventRecord(e0, s));
+    for (int r = 0; r < reps; ++r)
+      if (!launch(h, 0, sm_count, s, err)) return false;
+    RT_CHECK(cudaEventRecord(e1, s));
+    RT_CHECK(cudaEventSynchronize(e1));
+    RT_CHECK(cudaEventElapsedTime(&ms[b], e0, e1));
+  }
+  std::sort(ms, ms + 3);
+  *ns_out = std::max<int64_t>(1, (int64_t)(ms[1] * 1.0e6 / reps + 0.5));
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  return true;
+}
+
+}  // namespace bless

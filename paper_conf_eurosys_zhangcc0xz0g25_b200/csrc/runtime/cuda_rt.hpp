@@ -1,0 +1,77 @@
+// cuda_rt.hpp -- the CUDA side of one bl_ctx: SM probe (A1), launch-slot
+// ring, gated launches (A9/A10), completion stamps (A12), offline profiler
+// (A2).  Host-only declarations; implemented in cuda_rt.cu.
+#pragma once
+#include <cstdint>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "../../../include/bless/bless.h"
+#include "kdesc.hpp"
+
+namespace bless {
+
+struct LaunchStats {
+  int64_t start_host, end_host;  // host clock (CLOCK_MONOTONIC ns)
+  int nsm;
+  int fallback;
+};
+
+class DeviceRT {
+ public:
+  static std::unique_ptr<DeviceRT> create(int device, void* ws, size_t ws_bytes, std::string& err);
+  ~DeviceRT();
+
+  const bl_device_info& info() const { return info_; }
+  const DeviceCaps& caps() const { return caps_; }
+
+  // Build a launch descriptor; returns its handle (index) or -1.
+  int add_kernel(const bl_op& op, std::string& err);
+  const KernelDesc& kernel(int h) const { return *kernels_[h]; }
+
+  // Launch kernel h confined to logical SMs [lo, hi) on stream; returns seq (>0) or 0 on error.
+  uint64_t launch(int h, int lo, int hi, void* stream, std::string& err);
+  // Non-blocking: true if launch seq has published its stats.
+  bool poll(uint64_t seq, LaunchStats* out) const;
+
+  // Streams / events (thin wrappers so the engine does not include CUDA headers).
+  void* stream_create();
+  void stream_destroy(void* s);
+  void* event_create();
+  void event_destroy(void* e);
+  bool event_record(void* e, void* s);
+  bool stream_wait(void* s, void* e);
+  int event_query(void* e);  // 1 done, 0 pending, -1 error
+  bool stream_sync(void* s);
+  bool device_sync();
+  bool set_device();
+
+  // Offline profiler: median over 3 batches of the per-launch mean of 'reps'
+  // back-to-back launches on [0, sm_count).  d_out (if non-null): distinct SMs
+  // used in one unrestricted run.
+  bool profile(int h, int sm_count, int reps, void* stream, int64_t* ns_out, int* d_out, std::string& err);
+
+  int64_t gt_to_host(int64_t gt) const { return gt - info_.clock_offset_ns; }
+  bool calibrate_clock(std::string& err);
+
+ private:
+  DeviceRT() = default;
+  bool probe(std::string& err);
+
+  int device_ = 0;
+  bl_device_info info_{};
+  DeviceCaps caps_{};
+  void* slots_ = nullptr;        // DevSlot ring (device)
+  bool own_slots_ = false;
+  void* stats_host_ = nullptr;   // SlotStats ring (host-mapped)
+  void* stats_dev_ = nullptr;
+  uint8_t* lid_map_dev_ = nullptr;
+  bool identity_map_ = true;
+  uint64_t seq_ = 0;
+  std::vector<std::unique_ptr<KernelDesc>> kernels_;
+};
+
+constexpr uint64_t kSlotRing = 65536;
+
+}  // namespace bless

@@ -1,0 +1,777 @@
+// engine.cpp -- see engine.hpp.  Paper citations are PAPER.md lines; readings
+// R<n> are DESIGN.md §3.
+#include "engine.hpp"
+
+#include <algorithm>
+#include <chrono>
+#include <climits>
+#include <cmath>
+#include <cstring>
+
+#include "cuda_rt.hpp"
+
+namespace bless {
+
+static int64_t now_ns() {
+  return std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now().time_since_epoch())
+      .count();
+}
+
+static inline void cpu_relax() {
+#if defined(__x86_64__)
+  __builtin_ia32_pause();
+#endif
+}
+
+Engine::Engine(int device, const bl_params& p) : device_(device), prm_(p) {}
+
+Engine::~Engine() {
+  std::string e;
+  stop(e);
+  if (rt_) {
+    rt_->set_device();
+    rt_->device_sync();
+    for (auto& t : ten_) {
+      for (void* ev : t.events) rt_->event_destroy(ev);
+      if (t.own_stream && t.stream) rt_->stream_destroy(t.stream);
+    }
+    if (temporal_stream_) rt_->stream_destroy(temporal_stream_);
+  }
+}
+
+bl_status Engine::init(void* ws, size_t ws_bytes, std::string& err) {
+  if (prm_.sm_unit < 1 || prm_.squad_max < 1 || prm_.squad_max > BL_MAX_SQUAD || prm_.split_pct < 0 ||
+      prm_.split_pct > 100 || prm_.max_requests < 1) {
+    err = "invalid bl_params";
+    return BL_E_INVALID;
+  }
+  if (device_ != BL_DEVICE_NONE) {
+    rt_ = DeviceRT::create(device_, ws, ws_bytes, err);
+    if (!rt_) return BL_E_CUDA;
+    prof_.S = rt_->info().sm_count;
+  }
+  prof_.g = prm_.sm_unit;
+  cap_ = prm_.max_requests;
+  reqs_.reset(new (std::nothrow) Req[cap_]);
+  if (!reqs_) { err = "request table alloc"; return BL_E_OOM; }
+  return BL_OK;
+}
+
+void Engine::fail(const std::string& msg) {
+  if (!failed_.exchange(true)) fail_msg_ = msg;
+  stop_ = true;
+}
+
+// ------------------------------------------------------------------ setup
+bl_status Engine::register_tenant(double quota, const char* name, int* out, std::string& err) {
+  if (started_) { err = "register after bl_start"; return BL_E_STATE; }
+  if (!(quota > 0.0) || quota > 1.0) { err = "quota must be in (0, 1]"; return BL_E_QUOTA; }
+  if (quota_sum_ + quota > 1.0 + 1e-9) { err = "sum of quotas exceeds 1"; return BL_E_QUOTA; }
+  if (nten() >= BL_MAX_TENANTS) { err = "too many tenants"; return BL_E_FULL; }
+  TenantRT t;
+  t.name = name && *name ? name : ("tenant" + std::to_string(nten()));
+  for (char& c : t.name)
+    if (c == ' ' || c == '\t' || c == '\n') c = '_';
+  t.ppm = std::llround(quota * 1e6);
+  if (rt_) {
+    rt_->set_device();
+    t.stream = rt_->stream_create();
+    t.own_stream = true;
+    for (int i = 0; i < 64; ++i) t.events.push_back(rt_->event_create());
+  }
+  quota_sum_ += quota;
+  TenantProfile tp;
+  tp.name = t.name;
+  tp.quota_ppm = t.ppm;
+  prof_.ten.push_back(tp);
+  ten_.push_back(std::move(t));
+  if (out) *out = nten() - 1;
+  return BL_OK;
+}
+
+bl_status Engine::set_stream(int t, void* s, std::string& err) {
+  if (t < 0 || t >= nten() || !s) { err = "bad tenant/stream"; return BL_E_INVALID; }
+  if (started_) { err = "set_stream after bl_start"; return BL_E_STATE; }
+  if (!rt_) { err = "no device"; return BL_E_STATE; }
+  if (ten_[t].own_stream) rt_->stream_destroy(ten_[t].stream);
+  ten_[t].stream = s;
+  ten_[t].own_stream = false;
+  return BL_OK;
+}
+
+bl_status Engine::append_kernel(int t, const bl_op* op, int* out, std::string& err) {
+  if (t < 0 || t >= nten() || !op) { err = "bad tenant/op"; return BL_E_INVALID; }
+  if (started_) { err = "append after bl_start"; return BL_E_STATE; }
+  KernelProfile kp;
+  if (rt_) {
+    rt_->set_device();
+    const int h = rt_->add_kernel(*op, err);
+    if (h < 0) return BL_E_INVALID;
+    ten_[t].handles.push_back(h);
+    kp.name = std::string(rt_->kernel(h).family) + "_" + std::to_string(prof_.ten[t].k.size());
+  } else {
+    if (op->kind != BL_OP_VIRTUAL) { err = "device-less ctx accepts BL_OP_VIRTUAL only"; return BL_E_INVALID; }
+    ten_[t].handles.push_back(-1);
+    kp.name = "virtual_" + std::to_string(prof_.ten[t].k.size());
+  }
+  prof_.ten[t].k.push_back(kp);
+  if (out) *out = (int)prof_.ten[t].k.size() - 1;
+  return BL_OK;
+}
+
+bl_status Engine::run_kernel(int t, int k, int lo, int hi, std::string& err) {
+  if (!rt_) { err = "no device"; return BL_E_STATE; }
+  if (t < 0 || t >= nten() || k < 0 || k >= (int)ten_[t].handles.size()) { err = "bad index"; return BL_E_INVALID; }
+  if (started_) { err = "run_kernel while running"; return BL_E_STATE; }
+  rt_->set_device();
+  lo = std::max(0, lo);
+  hi = std::min(S(), hi);
+  if (lo >= hi) { err = "empty SM range"; return BL_E_INVALID; }
+  const uint64_t seq = rt_->launch(ten_[t].handles[k], lo, hi, ten_[t].stream, err);
+  if (!seq) return BL_E_CUDA;
+  if (!rt_->stream_sync(ten_[t].stream)) { err = "stream sync failed (kernel fault?)"; return BL_E_CUDA; }
+  return BL_OK;
+}
+
+bl_status Engine::profile_kernel(int t, int k, int sm_count, int reps, int64_t* ns, int* d, std::string& err) {
+  if (!rt_) { err = "no device"; return BL_E_STATE; }
+  if (started_) { err = "profile while running"; return BL_E_STATE; }
+  if (t < 0 || t >= nten() || k < 0 || k >= (int)ten_[t].handles.size() || !ns) { err = "bad index"; return BL_E_INVALID; }
+  rt_->set_device();
+  if (!rt_->profile(ten_[t].handles[k], sm_count, reps, ten_[t].stream, ns, d, err)) return BL_E_CUDA;
+  return BL_OK;
+}
+
+bl_status Engine::profile_tenant(int t, int reps, std::string& err) {
+  if (!rt_) { err = "no device"; return BL_E_STATE; }
+  if (t < 0 || t >= nten()) { err = "bad tenant"; return BL_E_INVALID; }
+  const int Sx = S();
+  for (size_t k = 0; k < ten_[t].handles.size(); ++k) {
+    KernelProfile& kp = prof_.ten[t].k[k];
+    kp.t.assign(Sx, 0);
+    int d = 0;
+    int64_t ns = 0;
+    bl_status st = profile_kernel(t, (int)k, Sx, reps, &ns, &d, err);
+    if (st != BL_OK) return st;
+    kp.d = d;
+    kp.t[Sx - 1] = ns;
+    for (int s = 1; s < Sx; ++s) {
+      st = profile_kernel(t, (int)k, s, reps, &kp.t[s - 1], nullptr, err);
+      if (st != BL_OK) return st;
+    }
+  }
+  prof_.derive();
+  return BL_OK;
+}
+
+bl_status Engine::set_profile_row(int t, int k, const int64_t* tns, int d, std::string& err) {
+  if (t < 0 || t >= nten() || k < 0 || k >= (int)prof_.ten[t].k.size() || !tns || d < 1 || d > S()) {
+    err = "bad profile row";
+    return BL_E_INVALID;
+  }
+  if (started_) { err = "profile change while running"; return BL_E_STATE; }
+  prof_.ten[t].k[k].t.assign(tns, tns + S());
+  prof_.ten[t].k[k].d = d;
+  prof_.derive();
+  return BL_OK;
+}
+
+bl_status Engine::get_profile_row(int t, int k, int64_t* tns, int* d, std::string& err) {
+  if (t < 0 || t >= nten() || k < 0 || k >= (int)prof_.ten[t].k.size()) { err = "bad index"; return BL_E_INVALID; }
+  const auto& kp = prof_.ten[t].k[k];
+  if ((int)kp.t.size() != S()) { err = "kernel not profiled"; return BL_E_STATE; }
+  if (tns) std::memcpy(tns, kp.t.data(), sizeof(int64_t) * S());
+  if (d) *d = kp.d;
+  return BL_OK;
+}
+
+bl_status Engine::save_profile(const char* path, std::string& err) {
+  if (!path) { err = "null path"; return BL_E_INVALID; }
+  if (!prof_.complete()) { err = "profile incomplete"; return BL_E_STATE; }
+  return save_profile_text(path, prof_, err) ? BL_OK : BL_E_INVALID;
+}
+
+bl_status Engine::load_profile(const char* path, std::string& err) {
+  if (!path) { err = "null path"; return BL_E_INVALID; }
+  if (started_) { err = "load after bl_start"; return BL_E_STATE; }
+  Profile p;
+  if (!load_profile_text(path, p, err)) return BL_E_NOTFOUND;
+  if (!rt_ && nten() == 0) {
+    // device-less ctx: adopt the whole description
+    prm_.sm_unit = p.g;
+    for (auto& tn : p.ten) {
+      int id = 0;
+      bl_status st = register_tenant((double)tn.quota_ppm / 1e6, tn.name.c_str(), &id, err);
+      if (st != BL_OK) return st;
+      ten_[id].ppm = tn.quota_ppm;  // exact
+      for (size_t k = 0; k < tn.k.size(); ++k) ten_[id].handles.push_back(-1);
+    }
+    prof_ = p;
+    prof_.derive();
+    return BL_OK;
+  }
+  if (p.S != S() || (int)p.ten.size() != nten()) { err = "profile does not match this ctx (S or tenants)"; return BL_E_INVALID; }
+  for (int j = 0; j < nten(); ++j) {
+    if (p.ten[j].k.size() != prof_.ten[j].k.size() || p.ten[j].quota_ppm != prof_.ten[j].quota_ppm) {
+      err = "profile does not match tenant " + std::to_string(j);
+      return BL_E_INVALID;
+    }
+    for (size_t k = 0; k < p.ten[j].k.size(); ++k) {
+      prof_.ten[j].k[k].t = p.ten[j].k[k].t;
+      prof_.ten[j].k[k].d = p.ten[j].k[k].d;
+    }
+  }
+  prof_.g = p.g;
+  prm_.sm_unit = p.g;
+  prof_.derive();
+  return BL_OK;
+}
+
+bl_status Engine::tenant_info(int t, int* qsms, int* m, int64_t* T, std::string& err) {
+  if (t < 0 || t >= nten()) { err = "bad tenant"; return BL_E_INVALID; }
+  prof_.derive();
+  if (qsms) *qsms = prof_.ten[t].quota_sms;
+  if (m) *m = (int)prof_.ten[t].k.size();
+  if (T) *T = prof_.ten[t].T;
+  return BL_OK;
+}
+
+bl_status Engine::device_info(bl_device_info* out, std::string& err) {
+  if (!out) { err = "null"; return BL_E_INVALID; }
+  if (!rt_) { err = "no device"; return BL_E_STATE; }
+  *out = rt_->info();
+  return BL_OK;
+}
+
+// ------------------------------------------------------------------ runtime
+bl_status Engine::start(std::string& err) {
+  if (started_) { err = "already started"; return BL_E_STATE; }
+  if (nten() == 0) { err = "no tenants"; return BL_E_STATE; }
+  if (!prof_.complete()) { err = "submit/start before a complete profile (PAPER.md L155: no profile, no BLESS)"; return BL_E_STATE; }
+  prof_.g = prm_.sm_unit;
+  prof_.derive();
+  if (prof_.N < 1) { err = "sm_unit larger than S"; return BL_E_INVALID; }
+  int lo = 0;
+  for (int j = 0; j < nten(); ++j) {
+    if (prof_.ten[j].quota_sms < 1) { err = "tenant " + std::to_string(j) + " gets 0 SMs"; return BL_E_QUOTA; }
+    if (prof_.ten[j].k.empty()) { err = "tenant without kernels"; return BL_E_STATE; }
+    ten_[j].lo = lo;
+    ten_[j].hi = lo + prof_.ten[j].quota_sms;
+    lo = ten_[j].hi;
+  }
+  if (!rt_ && prm_.policy != BL_POLICY_BLESS) { err = "device-less ctx runs the BLESS policy only"; return BL_E_STATE; }
+  if (!rt_ && prm_.clock != BL_CLOCK_VIRTUAL) { err = "device-less ctx needs the VIRTUAL clock"; return BL_E_STATE; }
+  if (rt_) {
+    rt_->set_device();
+    if (!temporal_stream_) temporal_stream_ = rt_->stream_create();
+    rt_->calibrate_clock(err);
+  }
+  fifo_.assign(nten(), {});
+  scan_ = 0;
+  pending_.clear();
+  inflight_.clear();
+  prev_events_.clear();
+  stop_ = false;
+  failed_ = false;
+  t0_ = now_ns() + 1000000;  // VIRTUAL on a device: wall anchor of trace time 0
+  started_ = true;
+  th_ = std::thread([this] { thread_main(); });
+  return BL_OK;
+}
+
+bl_status Engine::submit(int t, int64_t arrival, uint64_t* out, std::string& err) {
+  if (t < 0 || t >= nten()) { err = "bad tenant"; return BL_E_INVALID; }
+  if (prm_.clock == BL_CLOCK_VIRTUAL && started_) { err = "VIRTUAL clock: submit the whole trace before bl_start"; return BL_E_STATE; }
+  if (!prof_.complete()) { err = "submit before a complete profile"; return BL_E_STATE; }
+  if (prm_.clock == BL_CLOCK_VIRTUAL) {
+    if ((int)last_submit_arrival_.size() < nten()) last_submit_arrival_.resize(nten(), INT64_MIN);
+    if (arrival < last_submit_arrival_[t]) { err = "VIRTUAL: arrivals must be non-decreasing per tenant"; return BL_E_INVALID; }
+    last_submit_arrival_[t] = arrival;
+  }
+  const uint64_t id = next_id_.fetch_add(1);
+  if ((int64_t)id >= cap_) { err = "request table full"; return BL_E_FULL; }
+  Req& r = reqs_[id];
+  r.tenant = t;
+  r.arrival = arrival;
+  r.arrival_host = arrival;
+  r.start = r.finish = 0;
+  r.done.store(0, std::memory_order_relaxed);
+  r.published.store(1, std::memory_order_release);
+  if (out) *out = id;
+  return BL_OK;
+}
+
+bl_status Engine::poll(uint64_t id, bl_req_info* out, std::string& err) {
+  if (id >= next_id_.load() || (int64_t)id >= cap_) { err = "unknown request"; return BL_E_NOTFOUND; }
+  Req& r = reqs_[id];
+  if (out) {
+    out->req = id;
+    out->tenant = r.tenant;
+    out->arrival_ns = r.arrival_host;
+  }
+  if (!r.done.load(std::memory_order_acquire)) {
+    if (out) out->status = BL_PENDING;
+    if (failed_) { err = "engine failed: " + fail_msg_; return BL_E_CUDA; }
+    return BL_PENDING;
+  }
+  if (out) {
+    out->status = BL_OK;
+    out->start_ns = r.start;
+    out->finish_ns = r.finish;
+  }
+  return BL_OK;
+}
+
+bl_status Engine::drain(int64_t timeout_ns, std::string& err) {
+  const int64_t deadline = now_ns() + timeout_ns;
+  while (n_done_.load() < next_id_.load()) {
+    if (failed_) { err = "engine failed: " + fail_msg_; return BL_E_CUDA; }
+    if (!started_) { err = "not started"; return BL_E_STATE; }
+    if (timeout_ns >= 0 && now_ns() > deadline) { err = "drain timeout"; return BL_E_TIMEOUT; }
+    std::this_thread::sleep_for(std::chrono::microseconds(50));
+  }
+  return BL_OK;
+}
+
+bl_status Engine::stop(std::string& err) {
+  stop_ = true;
+  if (th_.joinable()) th_.join();
+  if (rt_ && started_) {
+    rt_->set_device();
+    if (!rt_->device_sync()) { err = "device error at stop"; started_ = false; return BL_E_CUDA; }
+    harvest();
+  }
+  started_ = false;
+  if (failed_) { err = fail_msg_; return BL_E_CUDA; }
+  return BL_OK;
+}
+
+bl_status Engine::reset(const bl_params* p, std::string& err) {
+  bl_status st = stop(err);
+  if (st != BL_OK && st != BL_E_CUDA) return st;
+  if (p) {
+    if (p->max_requests != prm_.max_requests) { err = "max_requests cannot change on reset"; return BL_E_INVALID; }
+    prm_ = *p;
+    prof_.g = prm_.sm_unit;
+    prof_.derive();
+  }
+  const uint64_t n = next_id_.load();
+  for (uint64_t i = 0; i < n && (int64_t)i < cap_; ++i) {
+    reqs_[i].published.store(0);
+    reqs_[i].done.store(0);
+  }
+  next_id_ = 0;
+  n_done_ = 0;
+  last_submit_arrival_.clear();
+  failed_ = false;
+  fail_msg_.clear();
+  std::lock_guard<std::mutex> lk(log_mu_);
+  dlog_.clear();
+  llog_.clear();
+  return BL_OK;
+}
+
+bl_status Engine::decisions(size_t first, bl_decision* buf, size_t cap, size_t* n) {
+  std::lock_guard<std::mutex> lk(log_mu_);
+  size_t c = 0;
+  for (size_t i = first; i < dlog_.size() && c < cap; ++i) buf[c++] = dlog_[i];
+  if (n) *n = (buf == nullptr) ? dlog_.size() : c;
+  return BL_OK;
+}
+
+bl_status Engine::launches(size_t first, bl_launch_rec* buf, size_t cap, size_t* n) {
+  std::lock_guard<std::mutex> lk(log_mu_);
+  size_t c = 0;
+  for (size_t i = first; i < llog_.size() && c < cap; ++i) buf[c++] = llog_[i];
+  if (n) *n = (buf == nullptr) ? llog_.size() : c;
+  return BL_OK;
+}
+
+static void to_record(const Decision& d, bl_decision& r) {
+  std::memset(&r, 0, sizeof(r));
+  r.now = d.now;
+  r.t_hat = d.t_hat;
+  r.t_nsp = d.t_nsp;
+  r.n_active = (int32_t)d.active.size();
+  for (size_t i = 0; i < d.active.size() && i < BL_MAX_TENANTS; ++i) {
+    r.act_tenant[i] = d.active[i].tenant;
+    r.act_arrival[i] = d.active[i].arrival;
+    r.act_next[i] = d.active[i].next;
+  }
+  r.n_part = (int32_t)d.parts.size();
+  r.config_sp = d.sp ? 1 : 0;
+  for (size_t i = 0; i < d.parts.size(); ++i) {
+    r.part_tenant[i] = d.parts[i];
+    r.part_p[i] = d.sp ? d.p[i] : 0;
+  }
+  r.n_picks = (int32_t)d.picks.size();
+  for (size_t i = 0; i < d.picks.size() && i < BL_MAX_SQUAD; ++i) {
+    r.pick_tenant[i] = d.picks[i].tenant;
+    r.pick_kernel[i] = d.picks[i].kernel;
+    r.pick_lo[i] = (int16_t)d.picks[i].lo;
+    r.pick_hi[i] = (int16_t)d.picks[i].hi;
+  }
+}
+
+bl_status Engine::decide_pure(int64_t now, int n, const int32_t* ten, const int64_t* arr, const int32_t* nxt,
+                              bl_decision* out, std::string& err) {
+  if (n < 1 || n > nten() || !ten || !arr || !nxt || !out) { err = "bad active set"; return BL_E_INVALID; }
+  if (!prof_.complete()) { err = "profile incomplete"; return BL_E_STATE; }
+  prof_.g = prm_.sm_unit;
+  prof_.derive();
+  std::vector<ActiveReq> a(n);
+  std::vector<int> seen(nten(), 0);
+  for (int i = 0; i < n; ++i) {
+    if (ten[i] < 0 || ten[i] >= nten() || seen[ten[i]]++ || nxt[i] < 0 || nxt[i] >= (int)prof_.ten[ten[i]].k.size()) {
+      err = "bad active entry";
+      return BL_E_INVALID;
+    }
+    a[i] = {ten[i], arr[i], nxt[i]};
+  }
+  SchedParams sp{prm_.squad_max, prm_.split_pct, prm_.seed_all != 0};
+  Decision d;
+  DecideScratch sc;
+  decide(now, a.data(), n, prof_, sp, d, sc);
+  to_record(d, *out);
+  return BL_OK;
+}
+
+void Engine::log_decision(const Decision& d) {
+  bl_decision r;
+  to_record(d, r);
+  std::lock_guard<std::mutex> lk(log_mu_);
+  dlog_.push_back(r);
+}
+
+// ------------------------------------------------------------------ scheduler thread
+void Engine::scan_submissions() {
+  const uint64_t hi = next_id_.load(std::memory_order_acquire);
+  while (scan_ < hi && (int64_t)scan_ < cap_ && reqs_[scan_].published.load(std::memory_order_acquire)) {
+    fifo_[reqs_[scan_].tenant].push_back(scan_);
+    ++scan_;
+  }
+}
+
+uint64_t Engine::launch_one(int t, int k, int lo, int hi, void* stream, int64_t req, bool last) {
+  std::string err;
+  const uint64_t seq = rt_->launch(ten_[t].handles[k], lo, hi, stream, err);
+  if (!seq) {
+    fail(err);
+    return 0;
+  }
+  bl_launch_rec rec{};
+  rec.seq = seq;
+  rec.tenant = t;
+  rec.kernel = k;
+  rec.lo = (int16_t)lo;
+  rec.hi = (int16_t)hi;
+  rec.req = req >= 0 ? (uint64_t)req : ~0ull;
+  size_t idx;
+  {
+    std::lock_guard<std::mutex> lk(log_mu_);
+    idx = llog_.size();
+    llog_.push_back(rec);
+  }
+  pending_.push_back({seq, idx, req, k, last ? 1 : 0});
+  return seq;
+}
+
+void Engine::harvest() {
+  if (!rt_ || pending_.empty()) return;
+  size_t w = 0;
+  for (size_t i = 0; i < pending_.size(); ++i) {
+    PendingLaunch& p = pending_[i];
+    LaunchStats st;
+    if (!rt_->poll(p.seq, &st)) {
+      pending_[w++] = p;
+      continue;
+    }
+    {
+      std::lock_guard<std::mutex> lk(log_mu_);
+      bl_launch_rec& r = llog_[p.log_idx];
+      r.start_ns = st.start_host;
+      r.end_ns = st.end_host;
+      r.nsm = st.nsm;
+      r.fallback = st.fallback;
+    }
+    if (p.req >= 0) {
+      Req& q = reqs_[p.req];
+      if (p.kernel == 0) q.start = st.start_host;
+      if (p.last) {
+        q.finish = st.end_host;
+        q.done.store(1, std::memory_order_release);
+        n_done_.fetch_add(1);
+      }
+    }
+  }
+  pending_.resize(w);
+}
+
+void Engine::retire_inflight() {
+  while (!inflight_.empty()) {
+    bool all = true;
+    for (void* e : inflight_.front().events) {
+      const int q = rt_->event_query(e);
+      if (q < 0) {
+        fail("device error (event query)");
+        return;
+      }
+      if (q == 0) { all = false; break; }
+    }
+    if (!all) return;
+    inflight_.pop_front();
+  }
+}
+
+void Engine::thread_main() {
+  if (rt_) rt_->set_device();
+  switch (prm_.policy) {
+    case BL_POLICY_BLESS: loop_bless(); break;
+    case BL_POLICY_ISO:
+    case BL_POLICY_STATIC: loop_at_arrival(false); break;
+    case BL_POLICY_UNBOUND: loop_at_arrival(true); break;
+    case BL_POLICY_TEMPORAL: loop_temporal(); break;
+    default: fail("unknown policy");
+  }
+  // keep harvesting completions until stopped
+  while (!stop_) {
+    if (rt_) harvest();
+    std::this_thread::sleep_for(std::chrono::microseconds(20));
+  }
+}
+
+// BLESS: squads on the event-barriered tenant streams (§4.3-§4.5).
+void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req, const std::vector<int>& act_next) {
+  // Squad barrier: every participant waits for the previous squad's kernels
+  // (the paper synchronises after each squad, L276; here a GPU-side event
+  // wait instead of a host synchronisation, L432's 20 us switch).
+  for (int j : d.parts)
+    for (void* ev : prev_events_) rt_->stream_wait(ten_[j].stream, ev);
+  std::vector<int> cnt(nten(), 0);
+  for (const Pick& p : d.picks) {
+    const int j = p.tenant;
+    const int k = p.kernel;
+    const bool last = k == (int)prof_.ten[j].k.size() - 1;
+    const bool first = k == 0;
+    (void)act_next;
+    (void)cnt;
+    if (!launch_one(j, k, p.lo, p.hi, ten_[j].stream, (first || last) ? act_req[j] : -1, last)) return;
+  }
+  Inflight inf;
+  for (int j : d.parts) {
+    TenantRT& t = ten_[j];
+    void* ev = t.events[t.ev_next++ % t.events.size()];
+    rt_->event_record(ev, t.stream);
+    inf.events.push_back(ev);
+  }
+  prev_events_ = inf.events;
+  inflight_.push_back(std::move(inf));
+}
+
+void Engine::loop_bless() {
+  const bool virt = prm_.clock == BL_CLOCK_VIRTUAL;
+  const int nt = nten();
+  std::vector<int64_t> act_req(nt, -1);
+  std::vector<int> act_next(nt, 0);
+  std::vector<ActiveReq> av;
+  SchedParams sp{prm_.squad_max, prm_.split_pct, prm_.seed_all != 0};
+  int64_t vnow = 0;   // VIRTUAL clock
+  int64_t E = 0;      // WALL: predicted end of the last launched squad
+  const size_t max_inflight = (size_t)std::max(1, prm_.max_inflight_squads);
+  while (!stop_) {
+    if (rt_) {
+      harvest();
+      retire_inflight();
+      if (failed_) return;
+    }
+    scan_submissions();
+    int64_t now;
+    if (virt) {
+      for (int j = 0; j < nt; ++j)
+        if (act_req[j] < 0 && !fifo_[j].empty() && reqs_[fifo_[j].front()].arrival <= vnow) {
+          act_req[j] = (int64_t)fifo_[j].front();
+          act_next[j] = 0;
+          fifo_[j].pop_front();
+        }
+      bool any = false;
+      for (int j = 0; j < nt; ++j) any |= act_req[j] >= 0;
+      if (!any) {
+        int64_t nxt = INT64_MAX;
+        for (int j = 0; j < nt; ++j)
+          if (!fifo_[j].empty()) nxt = std::min(nxt, reqs_[fifo_[j].front()].arrival);
+        if (nxt == INT64_MAX) return;  // trace finished (all submitted before start)
+        vnow = nxt;
+        continue;
+      }
+      now = vnow;
+    } else {
+      const int64_t host = now_ns();
+      const bool gpu_idle = inflight_.empty();
+      if (!gpu_idle && (inflight_.size() >= max_inflight || host < E - prm_.lookahead_ns)) {
+        cpu_relax();
+        continue;
+      }
+      for (int j = 0; j < nt; ++j)
+        if (act_req[j] < 0 && !fifo_[j].empty() && reqs_[fifo_[j].front()].arrival <= host) {
+          act_req[j] = (int64_t)fifo_[j].front();
+          act_next[j] = 0;
+          fifo_[j].pop_front();
+        }
+      bool any = false;
+      for (int j = 0; j < nt; ++j) any |= act_req[j] >= 0;
+      if (!any) {
+        cpu_relax();
+        continue;
+      }
+      now = gpu_idle ? host : std::max(host, E);
+    }
+    av.clear();
+    for (int j = 0; j < nt; ++j)
+      if (act_req[j] >= 0) av.push_back({j, reqs_[act_req[j]].arrival, act_next[j]});
+    decide(now, av.data(), (int)av.size(), prof_, sp, dec_, scratch_);
+    log_decision(dec_);
+    if (rt_) {
+      if (virt) {
+        // a squad is not launched before the wall time of its newest arrival (R17)
+        int64_t newest = INT64_MIN;
+        for (int j : dec_.parts) newest = std::max(newest, reqs_[act_req[j]].arrival);
+        for (int j : dec_.parts) reqs_[act_req[j]].arrival_host = t0_ + reqs_[act_req[j]].arrival;
+        while (!stop_ && (now_ns() < t0_ + newest || inflight_.size() >= max_inflight)) {
+          harvest();
+          retire_inflight();
+          if (failed_) return;
+          cpu_relax();
+        }
+      }
+      launch_squad(dec_, act_req, act_next);
+      if (failed_) return;
+    }
+    // advance the requests
+    for (size_t i = 0; i < dec_.parts.size(); ++i) {
+      const int j = dec_.parts[i];
+      int c = 0;
+      for (const Pick& p : dec_.picks) c += p.tenant == j;
+      Req& r = reqs_[act_req[j]];
+      if (!rt_ && act_next[j] == 0) r.start = now;
+      act_next[j] += c;
+      if (act_next[j] == (int)prof_.ten[j].k.size()) {
+        if (!rt_) {  // model completion (device-less ctx): SURVEY C-3
+          r.finish = now + dec_.chain_end[i];
+          r.done.store(1, std::memory_order_release);
+          n_done_.fetch_add(1);
+        }
+        act_req[j] = -1;
+        act_next[j] = 0;
+      }
+    }
+    if (virt) vnow = now + dec_.t_hat + prm_.squad_overhead_ns;
+    else E = now + dec_.t_hat;
+  }
+}
+
+// ISO / STATIC / UNBOUND: the whole request is launched at arrival on the
+// tenant's stream, confined to its quota range or unrestricted (L103, L300).
+void Engine::loop_at_arrival(bool unbound) {
+  const int nt = nten();
+  while (!stop_) {
+    harvest();
+    if (failed_) return;
+    scan_submissions();
+    const int64_t host = now_ns();
+    bool launched = false;
+    for (int j = 0; j < nt; ++j) {
+      while (!fifo_[j].empty() && reqs_[fifo_[j].front()].arrival <= host) {
+        const int64_t r = (int64_t)fifo_[j].front();
+        fifo_[j].pop_front();
+        const int m = (int)prof_.ten[j].k.size();
+        const int lo = unbound ? 0 : ten_[j].lo, hi = unbound ? S() : ten_[j].hi;
+        for (int k = 0; k < m; ++k)
+          if (!launch_one(j, k, lo, hi, ten_[j].stream, (k == 0 || k == m - 1) ? r : -1, k == m - 1)) return;
+        launched = true;
+      }
+    }
+    if (!launched) cpu_relax();
+  }
+}
+
+// TEMPORAL (R22): slices of quota*P on the full GPU, one kernel at a time on a
+// shared stream; non-preemptive, a kernel starts only if it is predicted to end
+// inside the slice (except the slice's first kernel).  T-cap: fixed cyclic
+// slices (idle slices stay idle).  T-wc: round robin skipping idle tenants.
+void Engine::loop_temporal() {
+  const int nt = nten();
+  const int64_t P = std::max<int64_t>(1000, prm_.temporal_period_ns);
+  std::vector<int64_t> len(nt), off(nt);
+  int64_t acc = 0;
+  for (int j = 0; j < nt; ++j) {
+    len[j] = P * ten_[j].ppm / 1000000;
+    off[j] = acc;
+    acc += len[j];
+  }
+  std::vector<int64_t> act_req(nt, -1);
+  std::vector<int> act_next(nt, 0);
+  const int64_t base = now_ns();
+  int64_t F = 0;                 // predicted time the GPU becomes free
+  int64_t last_sid = -1;
+  // T-wc turn state
+  int turn = -1;
+  int64_t turn_end = 0, sid_wc = 0;
+  auto activate = [&](int j, int64_t host) {
+    if (act_req[j] < 0 && !fifo_[j].empty() && reqs_[fifo_[j].front()].arrival <= host) {
+      act_req[j] = (int64_t)fifo_[j].front();
+      act_next[j] = 0;
+      fifo_[j].pop_front();
+    }
+    return act_req[j] >= 0;
+  };
+  while (!stop_) {
+    harvest();
+    if (failed_) return;
+    scan_submissions();
+    const int64_t host = now_ns();
+    int j = -1;
+    int64_t slice_end = 0, sid = 0;
+    if (!prm_.temporal_work_conserving) {
+      const int64_t cyc = (host - base) / P, pos = (host - base) % P;
+      for (int q = 0; q < nt; ++q)
+        if (pos >= off[q] && pos < off[q] + len[q]) j = q;
+      if (j < 0) { cpu_relax(); continue; }
+      slice_end = base + cyc * P + off[j] + len[j];
+      sid = cyc * nt + j;
+      if (!activate(j, host)) { cpu_relax(); continue; }
+    } else {
+      if (turn < 0 || host >= turn_end || !activate(turn, host)) {
+        int pick = -1;
+        for (int s = 1; s <= nt; ++s) {
+          const int q = ((turn < 0 ? -1 : turn) + s + nt) % nt;
+          if (activate(q, host)) { pick = q; break; }
+        }
+        if (pick < 0) { turn = -1; cpu_relax(); continue; }
+        turn = pick;
+        turn_end = host + len[pick];
+        ++sid_wc;
+      }
+      j = turn;
+      slice_end = turn_end;
+      sid = sid_wc;
+    }
+    const int k = act_next[j];
+    const int m = (int)prof_.ten[j].k.size();
+    const int64_t dur = prof_.t(j, k, S());
+    const int64_t st = std::max(F, host);
+    const bool first = sid != last_sid;
+    if (st < slice_end && (first || st + dur <= slice_end)) {
+      if (!launch_one(j, k, 0, S(), temporal_stream_, (k == 0 || k == m - 1) ? act_req[j] : -1, k == m - 1)) return;
+      F = st + dur;
+      last_sid = sid;
+      if (++act_next[j] == m) {
+        act_req[j] = -1;
+        act_next[j] = 0;
+      }
+    } else {
+      cpu_relax();
+    }
+  }
+}
+
+}  // namespace bless

@@ -1,0 +1,135 @@
+// engine.hpp -- one bl_ctx: tenants, request table, scheduler/launch thread,
+// policies (BLESS + in-run baselines), logs.  Host C++17; device work goes
+// through DeviceRT (null for BL_DEVICE_NONE contexts, which run the same
+// scheduler on the virtual clock without CUDA).
+#pragma once
+#include <atomic>
+#include <deque>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "../../../include/bless/bless.h"
+#include "../sched/sched.hpp"
+
+namespace bless {
+
+class DeviceRT;
+
+struct Req {
+  std::atomic<int> published{0};
+  std::atomic<int> done{0};
+  int tenant = 0;
+  int64_t arrival = 0;       // as submitted
+  int64_t arrival_host = 0;  // latency origin (host clock; model time without a device)
+  int64_t start = 0, finish = 0;
+};
+
+struct TenantRT {
+  std::string name;
+  int64_t ppm = 0;
+  std::vector<int> handles;  // DeviceRT kernel handles
+  void* stream = nullptr;
+  bool own_stream = false;
+  int lo = 0, hi = 0;        // static (ISO/STATIC) range
+  std::vector<void*> events; // ring for squad barriers
+  size_t ev_next = 0;
+};
+
+struct PendingLaunch {
+  uint64_t seq;
+  size_t log_idx;
+  int64_t req;   // request whose first/last kernel this is (-1 otherwise)
+  int kernel;
+  int last;      // 1 if this is the request's last kernel
+};
+
+class Engine {
+ public:
+  Engine(int device, const bl_params& p);
+  ~Engine();
+  bl_status init(void* ws, size_t ws_bytes, std::string& err);
+
+  bl_status register_tenant(double quota, const char* name, int* out, std::string& err);
+  bl_status set_stream(int t, void* s, std::string& err);
+  bl_status append_kernel(int t, const bl_op* op, int* out, std::string& err);
+  bl_status run_kernel(int t, int k, int lo, int hi, std::string& err);
+  bl_status profile_kernel(int t, int k, int sm_count, int reps, int64_t* ns, int* d, std::string& err);
+  bl_status profile_tenant(int t, int reps, std::string& err);
+  bl_status set_profile_row(int t, int k, const int64_t* tns, int d, std::string& err);
+  bl_status get_profile_row(int t, int k, int64_t* tns, int* d, std::string& err);
+  bl_status save_profile(const char* path, std::string& err);
+  bl_status load_profile(const char* path, std::string& err);
+  bl_status tenant_info(int t, int* qsms, int* m, int64_t* T, std::string& err);
+  bl_status device_info(bl_device_info* out, std::string& err);
+
+  bl_status start(std::string& err);
+  bl_status submit(int t, int64_t arrival, uint64_t* out, std::string& err);
+  bl_status poll(uint64_t req, bl_req_info* out, std::string& err);
+  bl_status drain(int64_t timeout_ns, std::string& err);
+  bl_status stop(std::string& err);
+  bl_status reset(const bl_params* p, std::string& err);
+  bl_status decisions(size_t first, bl_decision* buf, size_t cap, size_t* n);
+  bl_status launches(size_t first, bl_launch_rec* buf, size_t cap, size_t* n);
+  bl_status decide_pure(int64_t now, int n, const int32_t* ten, const int64_t* arr, const int32_t* nxt,
+                        bl_decision* out, std::string& err);
+
+ private:
+  void thread_main();
+  void loop_bless();
+  void loop_at_arrival(bool unbound);
+  void loop_temporal();
+  void scan_submissions();
+  void harvest();
+  void retire_inflight();
+  void launch_squad(const Decision& d, const std::vector<int64_t>& act_req, const std::vector<int>& act_next);
+  uint64_t launch_one(int t, int k, int lo, int hi, void* stream, int64_t req, bool last);
+  void log_decision(const Decision& d);
+  void fail(const std::string& msg);
+  int nten() const { return (int)ten_.size(); }
+  int S() const { return prof_.S; }
+
+  int device_;
+  bl_params prm_;
+  std::unique_ptr<DeviceRT> rt_;
+  Profile prof_;
+  std::vector<TenantRT> ten_;
+  double quota_sum_ = 0;
+
+  // request table
+  std::unique_ptr<Req[]> reqs_;
+  int64_t cap_ = 0;
+  std::atomic<uint64_t> next_id_{0};
+  std::atomic<uint64_t> n_done_{0};
+  std::vector<int64_t> last_submit_arrival_;
+
+  // thread
+  std::thread th_;
+  std::atomic<bool> stop_{false};
+  std::atomic<bool> started_{false};
+  std::atomic<bool> failed_{false};
+  std::string fail_msg_;
+  int64_t t0_ = 0;
+
+  // scheduler-thread state
+  uint64_t scan_ = 0;
+  std::vector<std::deque<uint64_t>> fifo_;
+  DecideScratch scratch_;
+  Decision dec_;
+  std::vector<PendingLaunch> pending_;
+  struct Inflight {
+    std::vector<void*> events;
+  };
+  std::deque<Inflight> inflight_;
+  std::vector<void*> prev_events_;
+  void* temporal_stream_ = nullptr;
+
+  // logs
+  std::mutex log_mu_;
+  std::vector<bl_decision> dlog_;
+  std::vector<bl_launch_rec> llog_;
+};
+
+}  // namespace bless

@@ -1,0 +1,45 @@
+// kdesc.hpp -- launch descriptor of one tenant kernel (host side).
+//
+// Built once per kernel at bl_append_kernel (validation, tile count, grid,
+// TMA tensor maps) so that a launch on the hot path is a single
+// cudaLaunchKernel with a precomputed parameter block plus the per-launch
+// gate arguments (SM range, slot, sequence number).
+#pragma once
+#include <cuda_runtime_api.h>
+
+#include <cstdint>
+#include <string>
+
+#include "../../../include/bless/bless.h"
+#include "../kernels/executor.cuh"
+
+namespace bless {
+
+struct KernelDesc;
+typedef cudaError_t (*LaunchFn)(const KernelDesc&, const GateArgs&, cudaStream_t);
+
+struct KernelDesc {
+  bl_op op{};
+  const char* family = "";
+  uint32_t tiles = 1;
+  int grid = 0, block = 0, smem = 0;
+  double flops = 0;        // algorithmic FLOPs per launch (roofline)
+  double bytes = 0;        // algorithmic HBM bytes per launch (roofline)
+  LaunchFn launch = nullptr;
+  alignas(128) unsigned char params[4096];  // family-specific parameter block
+};
+
+struct DeviceCaps {
+  int S = 148;             // SMs
+  int cc_major = 10, cc_minor = 0;
+  int smem_optin = 232448;
+};
+
+// Validate op and fill the descriptor.  Returns false with err on a bad op.
+bool build_kernel(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
+
+// Per-family builders (return true if they took the op).
+bool build_simt(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
+bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
+
+}  // namespace bless

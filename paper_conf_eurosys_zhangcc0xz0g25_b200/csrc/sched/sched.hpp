@@ -1,0 +1,84 @@
+// sched.hpp -- BLESS runtime scheduling decision, pure C++17 (no CUDA).
+//
+// PAPER.md §4.3 (multi-task scheduler, L173-L189) and §4.4 (execution
+// configuration determiner, L191-L237), §4.5.2 (Semi-SP split, L253-L255).
+// Readings R1-R18 are listed in DESIGN.md §3.  All decision arithmetic is
+// integer (int64 / __int128) so the result is bit-exact and independent of
+// libm; the argmin over spatial splits is an exact dynamic programme over
+// suffixes instead of the oracle's plain enumeration.
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+namespace bless {
+
+// Quota -> SMs by largest remainder (R18).  ppm: quotas in parts per million.
+std::vector<int> hamilton(const std::vector<int64_t>& ppm, int S);
+
+struct KernelProfile {
+  std::string name;
+  int d = 0;                  // distinct SMs used unrestricted (L157 "d%", R19)
+  std::vector<int64_t> t;     // t[s-1]: duration on s SMs, s = 1..S (L157, R11)
+};
+
+struct TenantProfile {
+  std::string name;
+  int64_t quota_ppm = 0;
+  std::vector<KernelProfile> k;
+  // derived
+  int quota_sms = 0;
+  std::vector<int64_t> tau;   // tau[k] = sum_{i<=k} t[i][quota_sms] (L157)
+  int64_t T = 0;              // isolated latency T[n%] (L157)
+};
+
+struct Profile {
+  int S = 0, g = 4, N = 0;
+  std::vector<TenantProfile> ten;
+  void derive();              // quota_sms, tau, T, N
+  int64_t t(int j, int k, int s) const { return ten[j].k[k].t[s - 1]; }
+  bool complete() const;      // every kernel has S entries
+};
+
+bool load_profile_text(const std::string& path, Profile& out, std::string& err);
+bool save_profile_text(const std::string& path, const Profile& p, std::string& err);
+
+struct SchedParams {
+  int squad_max = 50;   // R5
+  int split_pct = 50;   // R16
+  bool seed_all = true; // R6
+};
+
+struct ActiveReq {
+  int tenant;
+  int64_t arrival;
+  int next;             // next kernel index of the request
+};
+
+struct Pick {
+  int tenant, kernel, lo, hi;
+};
+
+struct Decision {
+  int64_t now = 0, t_hat = 0, t_nsp = 0;
+  std::vector<ActiveReq> active;      // sorted by tenant
+  std::vector<Pick> picks;            // in pick order
+  std::vector<int> parts;             // participants, sorted tenant ids
+  bool sp = false;
+  std::vector<int> p;                 // partitions per participant (SP)
+  std::vector<int64_t> chain_end;     // per participant: predicted end of its picks
+};
+
+// Workspace reused across calls (no allocation on the hot path after warm-up).
+struct DecideScratch {
+  std::vector<int> nxt, order;
+  std::vector<int64_t> arr;
+  std::vector<std::vector<int>> ks;   // per participant kernel list
+  std::vector<int64_t> Sj;            // K x (N+1) chain sums
+  std::vector<int64_t> F;             // K x (N+1) DP table
+};
+
+void decide(int64_t now, const ActiveReq* act, int n_act, const Profile& prof, const SchedParams& prm,
+            Decision& out, DecideScratch& scratch);
+
+}  // namespace bless
