@@ -180,6 +180,7 @@ typedef struct {
   int64_t start_ns;   /* first tile claimed */
   int64_t end_ns;     /* last CTA exit */
   uint64_t req;
+  uint32_t sm_mask[8]; /* logical SMs that processed >= 1 tile (bit i = SM i) */
 } bl_launch_rec;
 
 /* Device facts from the probe kernel (A1). */

@@ -65,7 +65,8 @@ class bl_decision(C.Structure):
 class bl_launch_rec(C.Structure):
     _fields_ = [("seq", C.c_uint64), ("tenant", C.c_int32), ("kernel", C.c_int32),
                 ("lo", C.c_int16), ("hi", C.c_int16), ("nsm", C.c_int32), ("fallback", C.c_int32),
-                ("start_ns", C.c_int64), ("end_ns", C.c_int64), ("req", C.c_uint64)]
+                ("start_ns", C.c_int64), ("end_ns", C.c_int64), ("req", C.c_uint64),
+                ("sm_mask", C.c_uint32 * 8)]
 
 
 class bl_device_info(C.Structure):

@@ -25,12 +25,13 @@
 
 namespace bless {
 
-struct __align__(32) SlotStats {  // host-mapped, written by the last CTA
+struct __align__(64) SlotStats {  // host-mapped, written by the last CTA
   int64_t start_gt;
   int64_t end_gt;
   uint32_t nsm;
   uint32_t flags;                  // bit0: fallback executed
   uint64_t seq;                    // written last (release)
+  uint32_t mask[8];                // logical SMs that processed >= 1 tile
 };
 
 struct __align__(64) DevSlot {     // device memory, zero between launches
@@ -130,12 +131,16 @@ __device__ __forceinline__ void gate_finalize(const GateArgs& g, bool fallback) 
     __threadfence();
     DevSlot* s = g.slot;
     uint32_t nsm = 0;
+    volatile SlotStats* out = g.stats;
 #pragma unroll
-    for (int i = 0; i < 8; ++i) nsm += __popc(((volatile uint32_t*)s->mask)[i]);
+    for (int i = 0; i < 8; ++i) {
+      const uint32_t w = ((volatile uint32_t*)s->mask)[i];
+      out->mask[i] = w;
+      nsm += __popc(w);
+    }
     const uint64_t end = ptx_globaltimer();
     uint64_t st = *(volatile unsigned long long*)&s->start_gt;
     if (st == 0) st = end;
-    volatile SlotStats* out = g.stats;
     out->start_gt = (int64_t)st;
     out->end_gt = (int64_t)end;
     out->nsm = nsm;

@@ -1,10 +1,580 @@
-// tc_gemm.cu -- tcgen05/TMEM/TMA bf16 GEMM and implicit-GEMM conv (placeholder
-// until the tensor-core path lands; build_tc_gemm declines every op).
+// tc_gemm.cu -- bf16 GEMM and implicit-GEMM convolution on the 5th-generation
+// tensor cores (tcgen05.mma, fp32 accumulators in TMEM, operands staged by TMA),
+// persistent under the SM-gated executor.
+//
+//   Y[M,N] = act((A[M,K] . B[N,K]^T) * scale[n] + shift[n] + R[M,N])   (bf16 out)
+//
+// A is X (GEMM) or the implicit im2col of an NHWC input (conv): an M tile is a
+// BH x BW block of output pixels and, for every filter tap (r, s) and channel
+// chunk, one TMA box load of the shifted input window -- out-of-bounds
+// coordinates zero-fill, which implements the convolution padding.  Stride 2
+// uses a rank-5 "parity" view of the input, (c, w%2, w/2, h%2, h/2), so every
+// tap is again a dense box.  B is the KRSC weight matrix [Kout, R*S*C].
+//
+// Warp roles (192 threads): warp 0 = tile scheduler + TMA producer, warp 1 =
+// MMA issuer (one thread) and TMEM owner, warps 2-5 = epilogue (TMEM -> regs ->
+// fused epilogue -> global).  Tiles come from the executor's per-launch atomic
+// queue; the TMEM accumulator is double buffered so the epilogue of tile i
+// overlaps the main loop of tile i+1.
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <mutex>
+
 #include "../runtime/kdesc.hpp"
+#include "executor.cuh"
 
 namespace bless {
-bool build_tc_gemm(const bl_op&, const DeviceCaps&, KernelDesc&, std::string& err) {
-  err.clear();
-  return false;
+
+struct TcParams {
+  CUtensorMap tmA;  // 64-byte aligned (first member of a 128-byte aligned block)
+  CUtensorMap tmB;
+  const float* scale;
+  const float* shift;
+  const __nv_bfloat16* R;
+  __nv_bfloat16* Y;
+  int M, N, K;
+  int ldy, ldr, act;
+  int mode;          // 0 GEMM, 1 conv stride 1 (4-D map), 2 conv stride 2 (5-D parity map)
+  int tiles_n, num_kb;
+  int OH, OW, BH, BW, tiles_w, C, R_, S_, pad, kc_per_tap;
+};
+
+#ifdef __CUDACC__
+// ------------------------------------------------------------------ PTX helpers
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
 }
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(
+          smem_u32(dst)),
+      "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_4d(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1, int c2,
+                                            int c3) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6}], "
+      "[%2];" ::"r"(smem_u32(dst)),
+      "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_5d(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1, int c2,
+                                            int c3, int c4) {
+  asm volatile(
+      "cp.async.bulk.tensor.5d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6, %7}], "
+      "[%2];" ::"r"(smem_u32(dst)),
+      "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4)
+      : "memory");
+}
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void tc_mma(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc)
+      : "memory");
+}
+// 32 lanes x 32 bit, 16 consecutive columns per thread
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]), "=r"(v[8]),
+        "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+      : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_ld_wait() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+
+// UMMA shared-memory descriptor, K-major, swizzled (SW128/64/32: rows of
+// BK*2 bytes, 8-row atoms; LBO = 16 B (unused for swizzled K-major), SBO =
+// 8 rows * row bytes; version 1 = tcgen05; layout type 2/4/6).
+template <int BK>
+__device__ __forceinline__ uint64_t smem_desc(uint32_t saddr) {
+  constexpr uint64_t row_bytes = BK * 2;
+  constexpr uint64_t sbo = 8 * row_bytes;
+  constexpr uint64_t layout = (BK == 64) ? 2 : (BK == 32 ? 4 : 6);
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFF);
+  d |= (uint64_t)1 << 16;                    // LBO (16 B)
+  d |= (uint64_t)((sbo >> 4) & 0x3FFF) << 32;  // SBO
+  d |= (uint64_t)1 << 46;                    // version
+  d |= layout << 61;
+  return d;
+}
+
+// Instruction descriptor kind::f16: A, B bf16, D f32, both K-major, M = 128.
+template <int BN>
+__device__ __forceinline__ uint32_t instr_desc() {
+  uint32_t d = 0;
+  d |= 1u << 4;              // c_format = F32
+  d |= 1u << 7;              // a_format = BF16
+  d |= 1u << 10;             // b_format = BF16
+  d |= (uint32_t)(BN >> 3) << 17;
+  d |= (uint32_t)(128 >> 4) << 24;
+  return d;
+}
+
+__device__ __forceinline__ float act_f(float y, int act) {
+  switch (act) {
+    case BL_ACT_RELU: return fmaxf(y, 0.f);
+    case BL_ACT_RELU6: return fminf(fmaxf(y, 0.f), 6.f);
+    case BL_ACT_GELU: return 0.5f * y * (1.f + erff(y * 0.70710678118654752f));
+    default: return y;
+  }
+}
+
+template <int BN, int BK>
+struct TcCfg {
+  static constexpr int kStageA = 128 * BK * 2;
+  static constexpr int kStageB = BN * BK * 2;
+  static constexpr int kStageBytes = kStageA + kStageB;
+  static constexpr int kStages = std::min(6, (96 * 1024) / kStageBytes);
+  static constexpr int kTmemCols = (2 * BN) < 32 ? 32 : 2 * BN;
+  static constexpr int kSmem = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/;
+};
+
+template <int BN, int BK>
+__device__ void tc_work(const TcParams& p, const GateArgs& g) {
+  using Cfg = TcCfg<BN, BK>;
+  constexpr int ST = Cfg::kStages;
+  extern __shared__ __align__(1024) unsigned char smem_raw[];
+  unsigned char* smem = (unsigned char*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  unsigned char* sA = smem;
+  unsigned char* sB = smem + ST * Cfg::kStageA;
+  uint64_t* bars = (uint64_t*)(smem + ST * Cfg::kStageBytes);
+  uint64_t* full = bars;            // [ST]
+  uint64_t* empty = bars + ST;      // [ST]
+  uint64_t* tfull = bars + 2 * ST;  // [2] accumulator ready
+  uint64_t* tempty = tfull + 2;     // [2] accumulator drained
+  uint64_t* rfull = tempty + 2;     // [2] tile ring
+  uint64_t* rempty = rfull + 2;     // [2]
+  int* ring = (int*)(rempty + 2);   // [2]
+  uint32_t* tmem_slot = (uint32_t*)(ring + 2);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < ST; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&empty[i], 1);
+    }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&tfull[i], 1);
+      mbar_init(&tempty[i], 4);
+      mbar_init(&rfull[i], 1);
+      mbar_init(&rempty[i], 5);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "n"(Cfg::kTmemCols));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    // ---------------- tile scheduler + TMA producer
+    if (lane == 0) {
+      asm volatile("prefetch.tensormap [%0];" ::"l"(&p.tmA) : "memory");
+      asm volatile("prefetch.tensormap [%0];" ::"l"(&p.tmB) : "memory");
+      bool marked = false;
+      int stage = 0;
+      uint32_t phase = 0;
+      int rs = 0;
+      uint32_t rph = 0;
+      for (;;) {
+        const int t = gate_claim(g, marked);
+        mbar_wait(&rempty[rs], rph ^ 1);
+        ring[rs] = t;
+        mbar_arrive(&rfull[rs]);
+        if (++rs == 2) { rs = 0; rph ^= 1; }
+        if (t < 0) break;
+        const int tm = t / p.tiles_n, tn = t - tm * p.tiles_n;
+        int oh0 = 0, ow0 = 0;
+        if (p.mode != 0) {
+          const int th = tm / p.tiles_w;
+          oh0 = th * p.BH;
+          ow0 = (tm - th * p.tiles_w) * p.BW;
+        }
+        for (int kb = 0; kb < p.num_kb; ++kb) {
+          mbar_wait(&empty[stage], phase ^ 1);
+          mbar_expect_tx(&full[stage], Cfg::kStageBytes);
+          unsigned char* a = sA + stage * Cfg::kStageA;
+          unsigned char* b = sB + stage * Cfg::kStageB;
+          if (p.mode == 0) {
+            tma_load_2d(a, &p.tmA, &full[stage], kb * BK, tm * 128);
+            tma_load_2d(b, &p.tmB, &full[stage], kb * BK, tn * BN);
+          } else {
+            const int tap = kb / p.kc_per_tap, c0 = (kb - tap * p.kc_per_tap) * BK;
+            const int r = tap / p.S_, s = tap - r * p.S_;
+            if (p.mode == 1) {
+              tma_load_4d(a, &p.tmA, &full[stage], c0, ow0 - p.pad + s, oh0 - p.pad + r, 0);
+            } else {
+              const int dr = r - p.pad, ds = s - p.pad;
+              const int ph = dr & 1, pw = ds & 1;        // parity of the input row/col
+              const int qh = (dr - ph) / 2, qw = (ds - pw) / 2;
+              tma_load_5d(a, &p.tmA, &full[stage], c0, pw, ow0 + qw, ph, oh0 + qh);
+            }
+            tma_load_2d(b, &p.tmB, &full[stage], tap * p.C + c0, tn * BN);
+          }
+          if (++stage == ST) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ---------------- MMA issuer
+    const uint32_t idesc = instr_desc<BN>();
+    int stage = 0;
+    uint32_t phase = 0;
+    int rs = 0;
+    uint32_t rph = 0;
+    int acc = 0;
+    uint32_t aph = 0;
+    for (;;) {
+      mbar_wait(&rfull[rs], rph);
+      const int t = ring[rs];
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&rempty[rs]);
+      if (++rs == 2) { rs = 0; rph ^= 1; }
+      if (t < 0) break;
+      mbar_wait(&tempty[acc], aph ^ 1);
+      tc_fence_after();
+      const uint32_t d_tmem = tmem_base + acc * BN;
+      for (int kb = 0; kb < p.num_kb; ++kb) {
+        mbar_wait(&full[stage], phase);
+        tc_fence_after();
+        if (lane == 0) {
+          const uint32_t a0 = smem_u32(sA + stage * Cfg::kStageA);
+          const uint32_t b0 = smem_u32(sB + stage * Cfg::kStageB);
+#pragma unroll
+          for (int k = 0; k < BK / 16; ++k) {
+            tc_mma(d_tmem, smem_desc<BK>(a0 + k * 32), smem_desc<BK>(b0 + k * 32), idesc, (kb | k) ? 1u : 0u);
+          }
+          tc_commit(&empty[stage]);
+        }
+        __syncwarp();
+        if (++stage == ST) { stage = 0; phase ^= 1; }
+      }
+      if (lane == 0) tc_commit(&tfull[acc]);
+      __syncwarp();
+      if (++acc == 2) { acc = 0; aph ^= 1; }
+    }
+  } else {
+    // ---------------- epilogue warps 2..5 (TMEM lane quarter = warp % 4)
+    const int q = warp & 3;
+    int rs = 0;
+    uint32_t rph = 0;
+    int acc = 0;
+    uint32_t aph = 0;
+    for (;;) {
+      mbar_wait(&rfull[rs], rph);
+      const int t = ring[rs];
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&rempty[rs]);
+      if (++rs == 2) { rs = 0; rph ^= 1; }
+      if (t < 0) break;
+      const int tm = t / p.tiles_n, tn = t - tm * p.tiles_n;
+      const int row = q * 32 + lane;
+      int m;
+      bool valid;
+      if (p.mode == 0) {
+        m = tm * 128 + row;
+        valid = m < p.M;
+      } else {
+        const int th = tm / p.tiles_w;
+        const int oh = th * p.BH + row / p.BW, ow = (tm - th * p.tiles_w) * p.BW + row % p.BW;
+        valid = oh < p.OH && ow < p.OW;
+        m = oh * p.OW + ow;
+      }
+      mbar_wait(&tfull[acc], aph);
+      tc_fence_after();
+      const uint32_t tbase = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN;
+#pragma unroll 1
+      for (int c = 0; c < BN; c += 16) {
+        uint32_t v[16];
+        tmem_ld16(tbase + c, v);
+        tmem_ld_wait();
+        const int n0 = tn * BN + c;
+        if (!valid || n0 >= p.N) continue;
+        float y[16];
+#pragma unroll
+        for (int i = 0; i < 16; ++i) y[i] = __uint_as_float(v[i]);
+        const bool full16 = n0 + 16 <= p.N;
+        if (p.scale) {
+#pragma unroll
+          for (int i = 0; i < 16; ++i)
+            if (full16 || n0 + i < p.N) y[i] *= __ldg(p.scale + n0 + i);
+        }
+        if (p.shift) {
+#pragma unroll
+          for (int i = 0; i < 16; ++i)
+            if (full16 || n0 + i < p.N) y[i] += __ldg(p.shift + n0 + i);
+        }
+        if (p.R) {
+          const __nv_bfloat16* rr = p.R + (size_t)m * p.ldr + n0;
+          if (full16 && ((p.ldr & 7) == 0)) {
+            uint4 r0 = *reinterpret_cast<const uint4*>(rr);
+            uint4 r1 = *reinterpret_cast<const uint4*>(rr + 8);
+            const __nv_bfloat16* e0 = reinterpret_cast<const __nv_bfloat16*>(&r0);
+            const __nv_bfloat16* e1 = reinterpret_cast<const __nv_bfloat16*>(&r1);
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+              y[i] += __bfloat162float(e0[i]);
+              y[8 + i] += __bfloat162float(e1[i]);
+            }
+          } else {
+            for (int i = 0; i < 16; ++i)
+              if (n0 + i < p.N) y[i] += __bfloat162float(rr[i]);
+          }
+        }
+        __nv_bfloat16* yy = p.Y + (size_t)m * p.ldy + n0;
+        if (full16 && ((p.ldy & 7) == 0)) {
+          uint4 o[2];
+          __nv_bfloat162* ob = reinterpret_cast<__nv_bfloat162*>(o);
+#pragma unroll
+          for (int i = 0; i < 8; ++i) ob[i] = __floats2bfloat162_rn(act_f(y[2 * i], p.act), act_f(y[2 * i + 1], p.act));
+          *reinterpret_cast<uint4*>(yy) = o[0];
+          *reinterpret_cast<uint4*>(yy + 8) = o[1];
+        } else {
+          for (int i = 0; i < 16; ++i)
+            if (n0 + i < p.N) yy[i] = __float2bfloat16_rn(act_f(y[i], p.act));
+        }
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&tempty[acc]);
+      if (++acc == 2) { acc = 0; aph ^= 1; }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (warp == 1) {
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "n"(Cfg::kTmemCols));
+  }
+  __syncthreads();
+}
+
+template <int BN, int BK>
+__global__ void __launch_bounds__(192, 1) k_tc_gemm(const __grid_constant__ TcParams p, const GateArgs g) {
+  if (gate_in_range(g)) tc_work<BN, BK>(p, g);
+  int last = 0;
+  const bool fb = gate_leave(g, last);
+  if (fb) tc_work<BN, BK>(p, g);
+  if (last) gate_finalize(g, fb);
+}
+#endif  // __CUDACC__
+
+// ------------------------------------------------------------------ host side
+template <int BN, int BK>
+static cudaError_t launch_tc(const KernelDesc& d, const GateArgs& g, cudaStream_t st) {
+  void* args[2] = {(void*)d.params, (void*)&g};
+  return cudaLaunchKernel((const void*)k_tc_gemm<BN, BK>, dim3(d.grid), dim3(d.block), args, (size_t)d.smem, st);
+}
+
+template <int BN, int BK>
+static bool prep(KernelDesc& d, std::string& err) {
+  static std::once_flag once;
+  static cudaError_t attr_err = cudaSuccess;
+  std::call_once(once, [] {
+    attr_err = cudaFuncSetAttribute((const void*)k_tc_gemm<BN, BK>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    TcCfg<BN, BK>::kSmem);
+  });
+  if (attr_err != cudaSuccess) {
+    err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(attr_err);
+    return false;
+  }
+  d.smem = TcCfg<BN, BK>::kSmem;
+  d.launch = launch_tc<BN, BK>;
+  return true;
+}
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+static EncodeTiledFn encode_fn(std::string& err) {
+  static EncodeTiledFn fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (EncodeTiledFn)f;
+  });
+  if (!fn) err = "cuTensorMapEncodeTiled unavailable";
+  return fn;
+}
+
+static bool encode(CUtensorMap* map, int rank, const void* base, const cuuint64_t* dims, const cuuint64_t* strides,
+                   const cuuint32_t* box, int BK, std::string& err) {
+  EncodeTiledFn fn = encode_fn(err);
+  if (!fn) return false;
+  cuuint32_t es[5] = {1, 1, 1, 1, 1};
+  const CUtensorMapSwizzle sw =
+      BK == 64 ? CU_TENSOR_MAP_SWIZZLE_128B : (BK == 32 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B);
+  const CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, (cuuint32_t)rank, const_cast<void*>(base), dims,
+                        strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) {
+    err = "cuTensorMapEncodeTiled failed (" + std::to_string((int)r) + ")";
+    return false;
+  }
+  return true;
+}
+
+bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::string& err) {
+  err.clear();
+  if (op.dtype != BL_BF16 || caps.cc_major != 10) return false;
+  TcParams p;
+  std::memset(&p, 0, sizeof(p));
+  p.scale = (const float*)op.ptr[2];
+  p.shift = (const float*)op.ptr[3];
+  p.R = (const __nv_bfloat16*)op.ptr[4];
+  p.Y = (__nv_bfloat16*)op.ptr[5];
+  p.act = op.act;
+  const void* X = op.ptr[0];
+  const void* W = op.ptr[1];
+  int BK = 64;
+  if (op.kind == BL_OP_GEMM) {
+    p.M = (int)op.dims[0];
+    p.N = (int)op.dims[1];
+    p.K = (int)op.dims[2];
+    const int ldx = op.dims[3] ? (int)op.dims[3] : p.K;
+    p.ldy = op.dims[4] ? (int)op.dims[4] : p.N;
+    p.ldr = op.dims[5] ? (int)op.dims[5] : p.N;
+    if (p.M <= 8 || p.N % 16 || p.K % 8 || ldx % 8 || p.ldy % 8 || p.ldr % 8) return false;  // GEMV / SIMT
+    if (((uintptr_t)X | (uintptr_t)W) & 15) return false;
+    p.mode = 0;
+    BK = 64;
+    p.num_kb = (p.K + BK - 1) / BK;
+    cuuint64_t da[2] = {(cuuint64_t)p.K, (cuuint64_t)p.M}, sa[1] = {(cuuint64_t)ldx * 2};
+    cuuint32_t ba[2] = {(cuuint32_t)BK, 128};
+    if (!encode(&p.tmA, 2, X, da, sa, ba, BK, err)) return false;
+  } else if (op.kind == BL_OP_CONV) {
+    const int Nb = (int)op.dims[0], H = (int)op.dims[1], Wd = (int)op.dims[2], C = (int)op.dims[3];
+    const int K = (int)op.dims[4], R = (int)op.dims[5], S = (int)op.dims[6];
+    const int stride = (int)op.dims[7], pad = (int)op.dims[8], groups = (int)op.dims[9];
+    const int ldx = op.dims[10] ? (int)op.dims[10] : C;
+    p.ldy = op.dims[11] ? (int)op.dims[11] : K;
+    p.ldr = p.ldy;
+    if (Nb != 1 || groups != 1 || C % 16 || ldx % 8 || K % 16 || p.ldy % 8) return false;
+    if (stride != 1 && stride != 2) return false;
+    if (stride == 2 && ((H | Wd) & 1)) return false;
+    if (((uintptr_t)X | (uintptr_t)W) & 15) return false;
+    BK = (C % 64 == 0) ? 64 : (C % 32 == 0 ? 32 : 16);
+    p.OH = (H + 2 * pad - R) / stride + 1;
+    p.OW = (Wd + 2 * pad - S) / stride + 1;
+    p.M = p.OH * p.OW;
+    p.N = K;
+    p.K = R * S * C;
+    p.C = C;
+    p.R_ = R;
+    p.S_ = S;
+    p.pad = pad;
+    p.kc_per_tap = C / BK;
+    p.num_kb = R * S * p.kc_per_tap;
+    // M tile = BH x BW output pixels (BH*BW = 128), BW the smallest power of two >= OW (<= 128)
+    int BW = 1;
+    while (BW < p.OW && BW < 128) BW <<= 1;
+    BW = std::max(BW, 8);
+    p.BW = BW;
+    p.BH = 128 / BW;
+    p.tiles_w = (p.OW + BW - 1) / BW;
+    const int tiles_h = (p.OH + p.BH - 1) / p.BH;
+    if (R == 1 && S == 1 && stride == 1 && pad == 0 && ldx == C) {
+      // 1x1 stride-1: plain GEMM over pixels
+      p.mode = 0;
+      cuuint64_t da[2] = {(cuuint64_t)C, (cuuint64_t)(H * Wd)}, sa[1] = {(cuuint64_t)ldx * 2};
+      cuuint32_t ba[2] = {(cuuint32_t)BK, 128};
+      if (!encode(&p.tmA, 2, X, da, sa, ba, BK, err)) return false;
+    } else if (stride == 1) {
+      p.mode = 1;
+      cuuint64_t da[4] = {(cuuint64_t)C, (cuuint64_t)Wd, (cuuint64_t)H, 1};
+      cuuint64_t sa[3] = {(cuuint64_t)ldx * 2, (cuuint64_t)Wd * ldx * 2, (cuuint64_t)H * Wd * ldx * 2};
+      cuuint32_t ba[4] = {(cuuint32_t)BK, (cuuint32_t)BW, (cuuint32_t)p.BH, 1};
+      if (!encode(&p.tmA, 4, X, da, sa, ba, BK, err)) return false;
+    } else {
+      p.mode = 2;
+      cuuint64_t da[5] = {(cuuint64_t)C, 2, (cuuint64_t)(Wd / 2), 2, (cuuint64_t)(H / 2)};
+      cuuint64_t sa[4] = {(cuuint64_t)ldx * 2, (cuuint64_t)2 * ldx * 2, (cuuint64_t)Wd * ldx * 2,
+                          (cuuint64_t)2 * Wd * ldx * 2};
+      cuuint32_t ba[5] = {(cuuint32_t)BK, 1, (cuuint32_t)BW, 1, (cuuint32_t)p.BH};
+      if (!encode(&p.tmA, 5, X, da, sa, ba, BK, err)) return false;
+    }
+    if (p.mode != 0) p.tiles_n = 0;  // set below
+    (void)tiles_h;
+  } else {
+    return false;
+  }
+  // N tile: as wide as possible while keeping >= S tiles when the problem allows
+  const int tiles_m = (p.mode == 0) ? (p.M + 127) / 128 : p.tiles_w * ((p.OH + p.BH - 1) / p.BH);
+  int BN = 128;
+  if (p.N <= 16) BN = 16;
+  else if (p.N <= 32) BN = 32;
+  else if (p.N <= 64) BN = 64;
+  while (BN > 32 && (long long)tiles_m * ((p.N + BN - 1) / BN) < caps.S) BN >>= 1;
+  p.tiles_n = (p.N + BN - 1) / BN;
+  {
+    cuuint64_t db[2] = {(cuuint64_t)p.K, (cuuint64_t)p.N}, sb[1] = {(cuuint64_t)p.K * 2};
+    cuuint32_t bb[2] = {(cuuint32_t)BK, (cuuint32_t)BN};
+    if (!encode(&p.tmB, 2, W, db, sb, bb, BK, err)) return false;
+  }
+  d.op = op;
+  d.tiles = (uint32_t)(tiles_m * p.tiles_n);
+  d.block = 192;
+  d.grid = caps.S;
+  bool ok = false;
+#define TC_CASE(bn, bk) \
+  if (BN == bn && BK == bk) ok = prep<bn, bk>(d, err);
+  TC_CASE(16, 16) TC_CASE(16, 32) TC_CASE(16, 64)
+  TC_CASE(32, 16) TC_CASE(32, 32) TC_CASE(32, 64)
+  TC_CASE(64, 16) TC_CASE(64, 32) TC_CASE(64, 64)
+  TC_CASE(128, 16) TC_CASE(128, 32) TC_CASE(128, 64)
+#undef TC_CASE
+  if (!ok) {
+    if (err.empty()) err = "no tc instantiation";
+    return false;
+  }
+  static_assert(sizeof(TcParams) <= sizeof(d.params), "params block too small");
+  std::memcpy(d.params, &p, sizeof(p));
+  d.family = op.kind == BL_OP_GEMM ? "tc_gemm_bf16" : (p.mode == 0 ? "tc_conv1x1_bf16" : "tc_conv_bf16");
+  d.flops = 2.0 * p.M * p.N * p.K;
+  double a_bytes = (op.kind == BL_OP_CONV) ? 2.0 * op.dims[1] * op.dims[2] * op.dims[3] : 2.0 * p.M * p.K;
+  d.bytes = a_bytes + 2.0 * p.N * p.K + 2.0 * p.M * p.N * (p.R ? 2 : 1);
+  return true;
+}
+
 }  // namespace bless

@@ -248,6 +248,7 @@ bool DeviceRT::poll(uint64_t seq, LaunchStats* out) const {
     out->end_host = gt_to_host(s->end_gt);
     out->nsm = (int)s->nsm;
     out->fallback = (int)(s->flags & 1u);
+    for (int i = 0; i < 8; ++i) out->mask[i] = s->mask[i];
   }
   return true;
 }

@@ -16,6 +16,7 @@ struct LaunchStats {
   int64_t start_host, end_host;  // host clock (CLOCK_MONOTONIC ns)
   int nsm;
   int fallback;
+  uint32_t mask[8];
 };
 
 class DeviceRT {

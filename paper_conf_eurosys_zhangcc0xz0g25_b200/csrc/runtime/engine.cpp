@@ -493,6 +493,7 @@ void Engine::harvest() {
       r.end_ns = st.end_host;
       r.nsm = st.nsm;
       r.fallback = st.fallback;
+      for (int i = 0; i < 8; ++i) r.sm_mask[i] = st.mask[i];
     }
     if (p.req >= 0) {
       Req& q = reqs_[p.req];

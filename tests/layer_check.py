@@ -1,0 +1,39 @@
+"""Test helper: compare one kernel's GPU output with the float64 oracle on the
+kernel's own GPU input (per-layer comparison, errors do
+not compound).  Test infrastructure only."""
+import numpy as np
+
+from oracle import layers_ref as L
+
+
+def np64(t):
+    return None if t is None else t.detach().float().cpu().numpy().astype(np.float64)
+
+
+def reference(layer):
+    x = np64(layer.x)
+    if layer.kind == "gemm":
+        return L.gemm(x, np64(layer.w), np64(layer.shift), layer.act, np64(layer.res), np64(layer.scale))
+    if layer.kind == "conv":
+        g = layer.geom
+        return L.conv2d_nhwc(x, np64(layer.w), np64(layer.scale), np64(layer.shift), g["stride"], g["pad"],
+                             g.get("groups", 1), layer.act, np64(layer.res))
+    if layer.kind == "pool":
+        g = layer.geom
+        f = L.maxpool_nhwc if g["mode"] == "max" else L.avgpool_nhwc
+        return f(x, g["k"], g["stride"], g["pad"])
+    if layer.kind == "gap":
+        return L.global_avgpool_nhwc(x)
+    raise ValueError(layer.kind)
+
+
+def tolerance(dtype: str) -> float:
+    # north star: max relative error 1e-2 (bf16 in / fp32 accumulate), 1e-4 (fp32)
+    return 1e-2 if dtype == "bf16" else 1e-4
+
+
+def check_layer(layer, dtype):
+    ref = reference(layer)
+    got = np64(layer.y).reshape(ref.shape)
+    err = L.max_rel_err(got, ref)
+    return err, tolerance(dtype)
