@@ -28,6 +28,8 @@ template <>
 __device__ __forceinline__ float ldf<float>(const float* p) { return __ldg(p); }
 template <>
 __device__ __forceinline__ float ldf<__nv_bfloat16>(const __nv_bfloat16* p) { return __bfloat162float(*p); }
+__device__ __forceinline__ float to_f(float v) { return v; }
+__device__ __forceinline__ float to_f(__nv_bfloat16 v) { return __bfloat162float(v); }
 template <typename T>
 __device__ __forceinline__ void stf(T* p, float v);
 template <>
@@ -256,7 +258,7 @@ struct Gemv {
             const T* xr = X + (size_t)m * p.ldx + k;
             float s = 0.f;
 #pragma unroll
-            for (int v = 0; v < kVec; ++v) s = fmaf(ldf(we + v), ldf(xr + v), s);
+            for (int v = 0; v < kVec; ++v) s = fmaf(to_f(we[v]), ldf(xr + v), s);
             acc[m] += s;
           }
         }

@@ -1,0 +1,128 @@
+"""Per-kernel parity of the sm_100a tenant kernels with the float64 oracle
+(bf16: max relative error <= 1e-2, fp32: <= 1e-4; reading R24), on shapes of
+the configs' layers plus ragged and degenerate cases, run full-range and
+SM-restricted through the C ABI."""
+import numpy as np
+import pytest
+import torch
+
+from tests.layer_check import check_layer
+
+pytestmark = pytest.mark.gpu
+
+from paper_conf_eurosys_zhangcc0xz0g25_b200 import capi  # noqa: E402
+from paper_conf_eurosys_zhangcc0xz0g25_b200.models import Builder  # noqa: E402
+
+
+@pytest.fixture
+def ctx():
+    from paper_conf_eurosys_zhangcc0xz0g25_b200 import build
+    build.build(verbose=False)
+    c = capi.Ctx(0)
+    yield c
+    c.close()
+
+
+def one_layer(ctx, dtype, make):
+    t = ctx.register_tenant(1.0, "k")
+    b = Builder(ctx, t, "k", 1.0, dtype, seed=77)
+    make(b)
+    return b.m
+
+
+def run_and_check(ctx, m, dtype, ranges=((0, 148), (5, 9))):
+    errs = []
+    for lo, hi in ranges:
+        for k, layer in enumerate(m.layers):
+            layer.y.fill_(float("nan"))
+            ctx.run_kernel(m.tenant, k, lo, hi)
+            err, tol = check_layer(layer, dtype)
+            errs.append(err)
+            assert err <= tol, (k, lo, hi, err, tol)
+    return max(errs)
+
+
+GEMMS = [(256, 256, 256, "relu"), (128, 2304, 768, "none"), (384, 1024, 1024, "gelu"), (200, 48, 72, "relu"),
+         (17, 16, 16, "relu6"), (1000, 128, 64, "none"), (128, 768, 3072, "none")]
+
+
+@pytest.mark.parametrize("M,N,K,act", GEMMS)
+def test_tc_gemm(ctx, M, N, K, act):
+    def mk(b):
+        x = b.input((M, K))
+        r = b.param(np.random.default_rng(1).standard_normal((M, N)).astype(np.float32)) if act == "none" else None
+        b.gemm(x, N, act=act, bias=True, res=r)
+    m = one_layer(ctx, "bf16", mk)
+    run_and_check(ctx, m, "bf16")
+
+
+@pytest.mark.parametrize("M,N,K,dtype", [(1, 4096, 25088, "bf16"), (1, 1000, 2048, "bf16"), (3, 100, 50, "bf16"),
+                                         (1, 4096, 4096, "fp32"), (8, 64, 1000, "fp32")])
+def test_gemv(ctx, M, N, K, dtype):
+    def mk(b):
+        x = b.input((M, K))
+        b.gemm(x, N, act="relu", bias=True)
+    m = one_layer(ctx, dtype, mk)
+    run_and_check(ctx, m, dtype)
+
+
+CONVS = [  # H, W, C, K, k, stride, pad, act, residual
+    (56, 56, 64, 64, 3, 1, 1, "relu", False),
+    (56, 56, 64, 256, 1, 1, 0, "relu", True),
+    (56, 56, 128, 128, 3, 2, 1, "relu", False),
+    (56, 56, 256, 512, 1, 2, 0, "none", False),
+    (14, 14, 256, 256, 3, 1, 1, "relu", False),
+    (7, 7, 512, 2048, 1, 1, 0, "relu", True),
+    (7, 7, 512, 512, 3, 1, 1, "relu", False),
+    (32, 32, 16, 16, 3, 1, 1, "relu", False),
+    (112, 112, 64, 128, 3, 1, 1, "relu", False),
+    (10, 13, 32, 48, 3, 1, 1, "relu6", True),
+    (224, 224, 3, 64, 3, 1, 1, "relu", False),   # C = 3 -> generic path
+    (224, 224, 3, 64, 7, 2, 3, "relu", False),   # ResNet stem -> generic path
+]
+
+
+@pytest.mark.parametrize("H,W,C,K,k,s,p,act,res", CONVS)
+def test_conv_bf16(ctx, H, W, C, K, k, s, p, act, res):
+    def mk(b):
+        x = b.input((1, H, W, C))
+        OH, OW = (H + 2 * p - k) // s + 1, (W + 2 * p - k) // s + 1
+        r = b.param(np.random.default_rng(2).standard_normal((1, OH, OW, K)).astype(np.float32)) if res else None
+        b.conv(x, K, k, s, p, act=act, bn=True, res=r)
+    m = one_layer(ctx, "bf16", mk)
+    run_and_check(ctx, m, "bf16")
+
+
+@pytest.mark.parametrize("H,W,C,k,s,p,mode", [(112, 112, 64, 3, 2, 1, "max"), (224, 224, 64, 2, 2, 0, "max"),
+                                              (9, 8, 5, 3, 2, 1, "avg"), (7, 7, 2048, 0, 1, 0, "gap")])
+@pytest.mark.parametrize("dtype", ["bf16", "fp32"])
+def test_pool(ctx, H, W, C, k, s, p, mode, dtype):
+    def mk(b):
+        x = b.input((1, H, W, C))
+        b.pool(x, k, s, p, mode)
+    m = one_layer(ctx, dtype, mk)
+    run_and_check(ctx, m, dtype)
+
+
+def test_tc_kernel_uses_only_its_sms(ctx):
+    """A tensor-core conv launched on logical SMs [40, 44) processes tiles
+    only there (launch log mask), via the engine's STATIC policy."""
+    c = capi.Ctx(0, policy="STATIC")
+    t0 = c.register_tenant(0.03, "a")      # 148 * 0.03 = 4.44 -> 4 SMs
+    b = Builder(c, t0, "a", 0.03, "bf16", seed=5)
+    x = b.input((1, 56, 56, 64))
+    b.conv(x, 64, 3, 1, 1)
+    c.profile_tenant(t0, reps=2)
+    c.start()
+    base = capi.now_ns()
+    for i in range(3):
+        c.submit(t0, base + i)
+    c.drain(int(20e9))
+    c.stop()
+    q, _, _ = c.tenant_info(t0)
+    for r in c.launches():
+        bits = [w * 32 + i for w in range(8) for i in range(32) if r.sm_mask[w] >> i & 1]
+        assert bits and all(0 <= x < q for x in bits) and r.fallback == 0
+    err, tol = check_layer(b.m.layers[0], "bf16")
+    assert err <= tol
+    c.close()
