@@ -183,6 +183,15 @@ typedef struct {
   uint32_t sm_mask[8]; /* logical SMs that processed >= 1 tile (bit i = SM i) */
 } bl_launch_rec;
 
+/* Launch descriptor summary of one appended kernel (roofline accounting). */
+typedef struct {
+  char family[32];     /* e.g. "tc_conv_bf16", "gemv_bf16", "simt_mm_f32" */
+  int32_t tiles;       /* work tiles per launch (tile queue length) */
+  int32_t grid, block, smem;
+  double flops;        /* algorithmic FLOPs per launch */
+  double bytes;        /* algorithmic HBM bytes per launch (inputs + weights + outputs once) */
+} bl_kernel_info;
+
 /* Device facts from the probe kernel (A1). */
 typedef struct {
   int32_t device;
@@ -219,6 +228,17 @@ bl_status bl_append_kernel(bl_ctx* ctx, int tenant, const bl_op* op, int* kernel
 /* Run one kernel (not a request) once, unrestricted, on the tenant's stream and
  * wait: parity tests use it to compare a single layer with the oracle. */
 bl_status bl_run_kernel(bl_ctx* ctx, int tenant, int kernel_idx, int lo, int hi);
+/* Per-request host I/O (the paper's memory-management kernels, L87, L229):
+ * when set, every request of the tenant copies in_bytes from host_in to
+ * dev_in on the tenant's stream right before its first kernel, and out_bytes
+ * from dev_out to host_out right after its last kernel; the request finishes
+ * when that copy has landed.  host_in/host_out should be pinned
+ * (cudaHostAlloc / torch pin_memory) and stay valid until bl_destroy.
+ * Pass in_bytes = out_bytes = 0 to disable.  Before bl_start. */
+bl_status bl_set_tenant_io(bl_ctx* ctx, int tenant, const void* host_in, void* dev_in, size_t in_bytes,
+                           const void* dev_out, void* host_out, size_t out_bytes);
+/* Summary of kernel kernel_idx's launch descriptor.  BL_E_STATE without a device. */
+bl_status bl_kernel_info_get(bl_ctx* ctx, int tenant, int kernel_idx, bl_kernel_info* out);
 
 /* ---- offline profiler (L155-L161 §4.2.1; A2) ------------------------------------
  * bl_profile_kernel: time kernel on logical SMs [0, sm_count) with CUDA events:

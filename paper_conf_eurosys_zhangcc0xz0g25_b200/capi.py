@@ -69,6 +69,11 @@ class bl_launch_rec(C.Structure):
                 ("sm_mask", C.c_uint32 * 8)]
 
 
+class bl_kernel_info(C.Structure):
+    _fields_ = [("family", C.c_char * 32), ("tiles", C.c_int32), ("grid", C.c_int32), ("block", C.c_int32),
+                ("smem", C.c_int32), ("flops", C.c_double), ("bytes", C.c_double)]
+
+
 class bl_device_info(C.Structure):
     _fields_ = [("device", C.c_int32), ("sm_count", C.c_int32), ("max_smid", C.c_int32),
                 ("cc_major", C.c_int32), ("cc_minor", C.c_int32), ("tpc_pairs_found", C.c_int32),
@@ -93,6 +98,9 @@ _SIGS = {
     "bl_set_stream": (C.c_int, [C.c_void_p, C.c_int, C.c_void_p]),
     "bl_append_kernel": (C.c_int, [C.c_void_p, C.c_int, _P(bl_op), _P(C.c_int)]),
     "bl_run_kernel": (C.c_int, [C.c_void_p, C.c_int, C.c_int, C.c_int, C.c_int]),
+    "bl_set_tenant_io": (C.c_int, [C.c_void_p, C.c_int, C.c_void_p, C.c_void_p, C.c_size_t, C.c_void_p,
+                                   C.c_void_p, C.c_size_t]),
+    "bl_kernel_info_get": (C.c_int, [C.c_void_p, C.c_int, C.c_int, _P(bl_kernel_info)]),
     "bl_profile_kernel": (C.c_int, [C.c_void_p, C.c_int, C.c_int, C.c_int, C.c_int, _P(C.c_int64), _P(C.c_int)]),
     "bl_profile_tenant": (C.c_int, [C.c_void_p, C.c_int, C.c_int]),
     "bl_set_profile_row": (C.c_int, [C.c_void_p, C.c_int, C.c_int, _P(C.c_int64), C.c_int]),
@@ -195,6 +203,17 @@ class Ctx:
 
     def run_kernel(self, tenant: int, k: int, lo: int = 0, hi: int = 1 << 15):
         check("bl_run_kernel", lib().bl_run_kernel(self.h, tenant, k, lo, hi))
+
+    def set_tenant_io(self, tenant: int, host_in: int, dev_in: int, in_bytes: int, dev_out: int, host_out: int,
+                      out_bytes: int):
+        check("bl_set_tenant_io", lib().bl_set_tenant_io(self.h, tenant, C.c_void_p(host_in), C.c_void_p(dev_in),
+                                                         in_bytes, C.c_void_p(dev_out), C.c_void_p(host_out),
+                                                         out_bytes))
+
+    def kernel_info(self, tenant: int, k: int) -> bl_kernel_info:
+        out = bl_kernel_info()
+        check("bl_kernel_info_get", lib().bl_kernel_info_get(self.h, tenant, k, C.byref(out)))
+        return out
 
     def profile_kernel(self, tenant: int, k: int, sm_count: int, reps: int = 10):
         ns, d = C.c_int64(), C.c_int()

@@ -100,6 +100,15 @@ bl_status bl_run_kernel(bl_ctx* ctx, int tenant, int k, int lo, int hi) {
   GUARD(ctx);
   return wrap([&](std::string& e) { return ctx->eng->run_kernel(tenant, k, lo, hi, e); });
 }
+bl_status bl_set_tenant_io(bl_ctx* ctx, int tenant, const void* hin, void* din, size_t inb, const void* dout,
+                           void* hout, size_t outb) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->set_io(tenant, hin, din, inb, dout, hout, outb, e); });
+}
+bl_status bl_kernel_info_get(bl_ctx* ctx, int tenant, int k, bl_kernel_info* out) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->kernel_info(tenant, k, out, e); });
+}
 bl_status bl_profile_kernel(bl_ctx* ctx, int tenant, int k, int sm_count, int reps, int64_t* ns, int* d) {
   GUARD(ctx);
   return wrap([&](std::string& e) { return ctx->eng->profile_kernel(tenant, k, sm_count, reps, ns, d, e); });

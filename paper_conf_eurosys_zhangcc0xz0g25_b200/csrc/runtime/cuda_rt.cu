@@ -239,6 +239,37 @@ uint64_t DeviceRT::launch(int h, int lo, int hi, void* stream, std::string& err)
   return seq;
 }
 
+__global__ void k_marker(const GateArgs g) {
+  // zero tiles: the single CTA is the last one and publishes the stamps
+  int last = 0;
+  const bool fb = gate_leave(g, last);
+  if (last) gate_finalize(g, fb);
+}
+
+uint64_t DeviceRT::launch_marker(void* stream, std::string& err) {
+  const uint64_t seq = ++seq_;
+  const uint64_t slot = seq % kSlotRing;
+  GateArgs g;
+  g.slot = reinterpret_cast<DevSlot*>(slots_) + slot;
+  g.stats = reinterpret_cast<SlotStats*>(stats_dev_) + slot;
+  g.lid_map = nullptr;
+  g.seq = seq;
+  g.tiles = 0;
+  g.lo = 0;
+  g.hi = 0;
+  k_marker<<<1, 32, 0, (cudaStream_t)stream>>>(g);
+  const cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) {
+    err = std::string("marker: ") + cudaGetErrorString(e);
+    return 0;
+  }
+  return seq;
+}
+
+bool DeviceRT::memcpy_async(void* dst, const void* src, size_t n, void* stream) {
+  return cudaMemcpyAsync(dst, src, n, cudaMemcpyDefault, (cudaStream_t)stream) == cudaSuccess;
+}
+
 bool DeviceRT::poll(uint64_t seq, LaunchStats* out) const {
   const volatile SlotStats* s = reinterpret_cast<const volatile SlotStats*>(stats_host_) + (seq % kSlotRing);
   if (s->seq != seq) return false;

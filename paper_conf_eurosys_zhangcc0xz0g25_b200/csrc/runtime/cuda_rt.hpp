@@ -33,6 +33,9 @@ class DeviceRT {
 
   // Launch kernel h confined to logical SMs [lo, hi) on stream; returns seq (>0) or 0 on error.
   uint64_t launch(int h, int lo, int hi, void* stream, std::string& err);
+  // One-CTA completion marker (stats only, no work) on stream; returns seq or 0.
+  uint64_t launch_marker(void* stream, std::string& err);
+  bool memcpy_async(void* dst, const void* src, size_t n, void* stream);
   // Non-blocking: true if launch seq has published its stats.
   bool poll(uint64_t seq, LaunchStats* out) const;
 

@@ -133,6 +133,37 @@ bl_status Engine::run_kernel(int t, int k, int lo, int hi, std::string& err) {
   return BL_OK;
 }
 
+bl_status Engine::set_io(int t, const void* hin, void* din, size_t inb, const void* dout, void* hout, size_t outb,
+                         std::string& err) {
+  if (!rt_) { err = "no device"; return BL_E_STATE; }
+  if (t < 0 || t >= nten()) { err = "bad tenant"; return BL_E_INVALID; }
+  if (started_) { err = "set_io after bl_start"; return BL_E_STATE; }
+  if ((inb && (!hin || !din)) || (outb && (!dout || !hout))) { err = "null io buffer"; return BL_E_INVALID; }
+  TenantRT& tr = ten_[t];
+  tr.host_in = hin;
+  tr.dev_in = din;
+  tr.in_bytes = inb;
+  tr.dev_out = dout;
+  tr.host_out = hout;
+  tr.out_bytes = outb;
+  return BL_OK;
+}
+
+bl_status Engine::kernel_info(int t, int k, bl_kernel_info* out, std::string& err) {
+  if (!rt_) { err = "no device"; return BL_E_STATE; }
+  if (t < 0 || t >= nten() || k < 0 || k >= (int)ten_[t].handles.size() || !out) { err = "bad index"; return BL_E_INVALID; }
+  const KernelDesc& d = rt_->kernel(ten_[t].handles[k]);
+  std::memset(out, 0, sizeof(*out));
+  std::strncpy(out->family, d.family, sizeof(out->family) - 1);
+  out->tiles = (int32_t)d.tiles;
+  out->grid = d.grid;
+  out->block = d.block;
+  out->smem = d.smem;
+  out->flops = d.flops;
+  out->bytes = d.bytes;
+  return BL_OK;
+}
+
 bl_status Engine::profile_kernel(int t, int k, int sm_count, int reps, int64_t* ns, int* d, std::string& err) {
   if (!rt_) { err = "no device"; return BL_E_STATE; }
   if (started_) { err = "profile while running"; return BL_E_STATE; }
@@ -454,10 +485,42 @@ void Engine::scan_submissions() {
 
 uint64_t Engine::launch_one(int t, int k, int lo, int hi, void* stream, int64_t req, bool last) {
   std::string err;
-  const uint64_t seq = rt_->launch(ten_[t].handles[k], lo, hi, stream, err);
+  const TenantRT& tr = ten_[t];
+  if (k == 0 && tr.in_bytes && !rt_->memcpy_async(tr.dev_in, tr.host_in, tr.in_bytes, stream)) {
+    fail("H2D input copy failed");
+    return 0;
+  }
+  const uint64_t seq = rt_->launch(tr.handles[k], lo, hi, stream, err);
   if (!seq) {
     fail(err);
     return 0;
+  }
+  if (last && tr.out_bytes) {
+    // the request completes when its output has landed in host memory: a
+    // one-CTA marker after the D2H copy carries the completion stamp
+    if (!rt_->memcpy_async(tr.host_out, tr.dev_out, tr.out_bytes, stream)) {
+      fail("D2H output copy failed");
+      return 0;
+    }
+    const uint64_t mseq = rt_->launch_marker(stream, err);
+    if (!mseq) {
+      fail(err);
+      return 0;
+    }
+    {
+      bl_launch_rec rec{};
+      rec.seq = seq;
+      rec.tenant = t;
+      rec.kernel = k;
+      rec.lo = (int16_t)lo;
+      rec.hi = (int16_t)hi;
+      rec.req = req >= 0 ? (uint64_t)req : ~0ull;
+      std::lock_guard<std::mutex> lk(log_mu_);
+      pending_.push_back({seq, llog_.size(), req, k, 0});
+      llog_.push_back(rec);
+    }
+    pending_.push_back({mseq, (size_t)-1, req, -1, 1});
+    return seq;
   }
   bl_launch_rec rec{};
   rec.seq = seq;
@@ -486,7 +549,7 @@ void Engine::harvest() {
       pending_[w++] = p;
       continue;
     }
-    {
+    if (p.log_idx != (size_t)-1) {
       std::lock_guard<std::mutex> lk(log_mu_);
       bl_launch_rec& r = llog_[p.log_idx];
       r.start_ns = st.start_host;

@@ -36,6 +36,13 @@ struct TenantRT {
   int lo = 0, hi = 0;        // static (ISO/STATIC) range
   std::vector<void*> events; // ring for squad barriers
   size_t ev_next = 0;
+  // per-request host I/O (bl_set_tenant_io)
+  const void* host_in = nullptr;
+  void* dev_in = nullptr;
+  size_t in_bytes = 0;
+  const void* dev_out = nullptr;
+  void* host_out = nullptr;
+  size_t out_bytes = 0;
 };
 
 struct PendingLaunch {
@@ -56,6 +63,9 @@ class Engine {
   bl_status set_stream(int t, void* s, std::string& err);
   bl_status append_kernel(int t, const bl_op* op, int* out, std::string& err);
   bl_status run_kernel(int t, int k, int lo, int hi, std::string& err);
+  bl_status kernel_info(int t, int k, bl_kernel_info* out, std::string& err);
+  bl_status set_io(int t, const void* hin, void* din, size_t inb, const void* dout, void* hout, size_t outb,
+                   std::string& err);
   bl_status profile_kernel(int t, int k, int sm_count, int reps, int64_t* ns, int* d, std::string& err);
   bl_status profile_tenant(int t, int reps, std::string& err);
   bl_status set_profile_row(int t, int k, const int64_t* tns, int d, std::string& err);
