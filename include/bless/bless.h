@@ -280,6 +280,11 @@ bl_status bl_reset(bl_ctx* ctx, const bl_params* params);
 bl_status bl_decide(bl_ctx* ctx, int64_t now, int n_active, const int32_t* tenants,
                     const int64_t* arrivals, const int32_t* next_kernel, bl_decision* out);
 
+/* Diagnostics: mean per-launch device time of 'reps' back-to-back S-CTA
+ * launches of an executor skeleton (variant 0: empty kernel, 1: SM gate + tile
+ * queue + exit protocol, 2: 1 + host-mapped completion stamps). */
+bl_status bl_debug_overhead(bl_ctx* ctx, int variant, int reps, int64_t* ns_out);
+
 int64_t bl_now_ns(void);
 const char* bl_last_error(void);
 const char* bl_version(void);

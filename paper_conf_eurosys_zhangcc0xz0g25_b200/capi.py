@@ -118,6 +118,7 @@ _SIGS = {
     "bl_reset": (C.c_int, [C.c_void_p, _P(bl_params)]),
     "bl_decide": (C.c_int, [C.c_void_p, C.c_int64, C.c_int, _P(C.c_int32), _P(C.c_int64), _P(C.c_int32),
                             _P(bl_decision)]),
+    "bl_debug_overhead": (C.c_int, [C.c_void_p, C.c_int, C.c_int, _P(C.c_int64)]),
     "bl_now_ns": (C.c_int64, []),
     "bl_last_error": (C.c_char_p, []),
     "bl_version": (C.c_char_p, []),
@@ -209,6 +210,11 @@ class Ctx:
         check("bl_set_tenant_io", lib().bl_set_tenant_io(self.h, tenant, C.c_void_p(host_in), C.c_void_p(dev_in),
                                                          in_bytes, C.c_void_p(dev_out), C.c_void_p(host_out),
                                                          out_bytes))
+
+    def debug_overhead(self, variant: int, reps: int = 200) -> int:
+        ns = C.c_int64()
+        check("bl_debug_overhead", lib().bl_debug_overhead(self.h, variant, reps, C.byref(ns)))
+        return ns.value
 
     def kernel_info(self, tenant: int, k: int) -> bl_kernel_info:
         out = bl_kernel_info()

@@ -175,6 +175,11 @@ bl_status bl_decide(bl_ctx* ctx, int64_t now, int n, const int32_t* t, const int
   return wrap([&](std::string& e) { return ctx->eng->decide_pure(now, n, t, a, k, out, e); });
 }
 
+bl_status bl_debug_overhead(bl_ctx* ctx, int variant, int reps, int64_t* ns) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->debug_overhead(variant, reps, ns, e); });
+}
+
 int64_t bl_now_ns(void) {
   return std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now().time_since_epoch())
       .count();

@@ -9,44 +9,52 @@
 // boundary without MPS, MIG or any context switch (L253: BLESS needs a 50 us
 // context switch here; the gate costs one %smid read).
 //
-// Completion protocol (per launch "slot" of a ring in device memory):
-//   slot.next   tile counter (atomicAdd)
-//   slot.done   CTAs that have left (atomicAdd)
-//   slot.mask   logical SMs that processed >= 1 tile (R19, profiler's d)
-//   slot.start  %globaltimer when tile 0 was claimed
-// The CTA that brings 'done' to gridDim is the last one: it publishes
-// {start, end, nsm, flags, seq} to a host-mapped stats record (poll-able
-// by the host without any CUDA call) and zeroes the slot for reuse.
+// Per-launch state lives in a ring of "slots" (device memory):
+//   slot.ctr   64-bit word: low 32 bits = tile counter (claims), high 32 bits
+//              = CTAs that have left.  One atomic per CTA on exit returns both,
+//              so the last CTA learns "am I last" and "were all tiles claimed"
+//              in a single round trip.
+// and a ring of stats records (device memory, mirrored to the host by
+// copy-engine reads -- no SM ever waits on PCIe):
+//   stats.start  %globaltimer when tile 0 was claimed (written by that CTA)
+//   stats.mask   logical SMs that processed >= 1 tile (atomicOr per CTA; R19)
+//   stats.end / flags / seq   written by the last CTA (seq last, after a fence)
+// The last CTA also zeroes the mask of the stats record it will reuse
+// kMaskAhead launches later and resets its slot word.
 // Safety net: if the last CTA finds unclaimed tiles, no in-range CTA ran (the
 // hardware placed every CTA elsewhere); it then processes the tiles itself and
-// flags the launch (BL "fallback"), so correctness never depends on placement.
+// flags the launch ("fallback"), so correctness never depends on placement.
+//
+// Programmatic dependent launch: kernels are launched with programmatic stream
+// serialization; a CTA waits (griddepcontrol.wait) only right before touching
+// data produced by the previous kernel, and signals its dependents as soon as
+// the tile queue is exhausted, so a kernel's launch and prologue overlap the
+// tail of its predecessor on the tenant's stream.
 #pragma once
 #include <cstdint>
 
 namespace bless {
 
-struct __align__(64) SlotStats {  // host-mapped, written by the last CTA
+struct __align__(64) SlotStats {
   int64_t start_gt;
   int64_t end_gt;
-  uint32_t nsm;
-  uint32_t flags;                  // bit0: fallback executed
-  uint64_t seq;                    // written last (release)
-  uint32_t mask[8];                // logical SMs that processed >= 1 tile
+  uint32_t nsm;        // unused on device (host computes popcount of mask)
+  uint32_t flags;      // bit0: fallback executed
+  uint64_t seq;        // written last, after a device-scope fence
+  uint32_t mask[8];    // logical SMs that processed >= 1 tile
 };
 
-struct __align__(64) DevSlot {     // device memory, zero between launches
-  uint32_t next;
-  uint32_t done;
-  uint32_t flags;
-  uint32_t pad;
-  uint32_t mask[8];
-  unsigned long long start_gt;
-  uint32_t pad2[2];
+struct __align__(16) DevSlot {  // device memory, zero between launches
+  unsigned long long ctr;       // [31:0] claims, [63:32] CTAs done
+  unsigned long long pad;
 };
+
+constexpr uint64_t kMaskAhead = 32768;  // stats record zeroed this many launches ahead
 
 struct GateArgs {
   DevSlot* slot;
-  SlotStats* stats;
+  SlotStats* stats;        // this launch's record
+  SlotStats* stats_ahead;  // record of launch seq + kMaskAhead (mask zeroed here)
   const uint8_t* lid_map;  // logical SM index per %smid (255 = unusable); null = identity
   uint64_t seq;
   uint32_t tiles;
@@ -64,6 +72,9 @@ __device__ __forceinline__ uint64_t ptx_globaltimer() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 __device__ __forceinline__ int gate_lid(const GateArgs& g) {
   const uint32_t sm = ptx_smid() & 255u;
   return g.lid_map ? (int)__ldg(g.lid_map + sm) : (int)sm;
@@ -74,15 +85,15 @@ __device__ __forceinline__ bool gate_in_range(const GateArgs& g) {
 }
 
 // Claim the next tile (call from ONE thread).  Returns -1 when exhausted.
-// 'first' tracks whether this CTA already marked its SM in the mask.
+// 'marked' tracks whether this CTA already set its SM bit in the mask.
 __device__ __forceinline__ int gate_claim(const GateArgs& g, bool& marked) {
-  const uint32_t t = atomicAdd(&g.slot->next, 1u);
+  const uint32_t t = (uint32_t)atomicAdd(&g.slot->ctr, 1ull);
   if (t >= g.tiles) return -1;
-  if (t == 0) atomicExch(&g.slot->start_gt, (unsigned long long)ptx_globaltimer());
+  if (t == 0) g.stats->start_gt = (int64_t)ptx_globaltimer();
   if (!marked) {
     marked = true;
     const int lid = gate_lid(g);
-    atomicOr(&g.slot->mask[(lid >> 5) & 7], 1u << (lid & 31));
+    atomicOr(&g.stats->mask[(lid >> 5) & 7], 1u << (lid & 31));
   }
   return (int)t;
 }
@@ -109,14 +120,10 @@ __device__ __forceinline__ bool gate_leave(const GateArgs& g, int& is_last) {
   __shared__ int s_flag;
   __syncthreads();
   if (threadIdx.x == 0) {
-    __threadfence();
     const uint32_t nblk = gridDim.x * gridDim.y * gridDim.z;
-    const uint32_t prev = atomicAdd(&g.slot->done, 1u);
+    const unsigned long long prev = atomicAdd(&g.slot->ctr, 1ull << 32);
     int flag = 0;
-    if (prev == nblk - 1) {
-      const uint32_t nxt = atomicAdd(&g.slot->next, 0u);
-      flag = (nxt < g.tiles) ? 2 : 1;
-    }
+    if ((uint32_t)(prev >> 32) == nblk - 1) flag = ((uint32_t)prev < g.tiles) ? 2 : 1;
     s_flag = flag;
   }
   __syncthreads();
@@ -128,44 +135,54 @@ __device__ __forceinline__ bool gate_leave(const GateArgs& g, int& is_last) {
 __device__ __forceinline__ void gate_finalize(const GateArgs& g, bool fallback) {
   __syncthreads();
   if (threadIdx.x == 0) {
-    __threadfence();
-    DevSlot* s = g.slot;
-    uint32_t nsm = 0;
-    volatile SlotStats* out = g.stats;
-#pragma unroll
-    for (int i = 0; i < 8; ++i) {
-      const uint32_t w = ((volatile uint32_t*)s->mask)[i];
-      out->mask[i] = w;
-      nsm += __popc(w);
-    }
     const uint64_t end = ptx_globaltimer();
-    uint64_t st = *(volatile unsigned long long*)&s->start_gt;
-    if (st == 0) st = end;
-    out->start_gt = (int64_t)st;
+    SlotStats* out = g.stats;
     out->end_gt = (int64_t)end;
-    out->nsm = nsm;
+    if (g.tiles == 0) out->start_gt = (int64_t)end;
     out->flags = fallback ? 1u : 0u;
-    __threadfence_system();
-    out->seq = g.seq;
-    // reset the slot for its next use (ring reuse is >= 64K launches later)
-    s->next = 0;
-    s->done = 0;
-    s->flags = 0;
-#pragma unroll
-    for (int i = 0; i < 8; ++i) s->mask[i] = 0;
-    s->start_gt = 0;
+    // zero the mask of the record reused kMaskAhead launches from now
+    uint4* fm = reinterpret_cast<uint4*>(g.stats_ahead->mask);
+    fm[0] = make_uint4(0, 0, 0, 0);
+    fm[1] = make_uint4(0, 0, 0, 0);
+    g.slot->ctr = 0ull;
     __threadfence();
+    *reinterpret_cast<volatile uint64_t*>(&out->seq) = g.seq;
   }
 }
 
 // The canonical gated kernel body for tile-loop ops: Op::tile(params, t, smem).
 template <class Op>
 __device__ __forceinline__ void gated_run(const typename Op::Params& p, const GateArgs& g, unsigned char* smem) {
-  if (gate_in_range(g)) gate_tile_loop(g, [&](int t) { Op::tile(p, t, smem); });
+  if (gate_in_range(g)) {
+    pdl_wait();
+    gate_tile_loop(g, [&](int t) { Op::tile(p, t, smem); });
+  }
+  pdl_trigger();
   int last = 0;
   const bool fb = gate_leave(g, last);
-  if (fb) gate_tile_loop(g, [&](int t) { Op::tile(p, t, smem); });
+  if (fb) {
+    pdl_wait();
+    gate_tile_loop(g, [&](int t) { Op::tile(p, t, smem); });
+  }
   if (last) gate_finalize(g, fb);
+}
+#endif
+
+// Host: launch with programmatic stream serialization (PDL) unless disabled.
+extern int g_use_pdl;
+#ifdef __CUDACC__
+inline cudaError_t launch_kernel(const void* fn, dim3 grid, dim3 block, size_t smem, cudaStream_t st, void** args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = g_use_pdl ? 1 : 0;
+  return cudaLaunchKernelExC(&cfg, fn, args);
 }
 #endif
 

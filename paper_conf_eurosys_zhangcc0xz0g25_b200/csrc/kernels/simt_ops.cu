@@ -135,45 +135,126 @@ struct PoolParams {
   const void* X;
   void* Y;
   int Nb, H, W, C, OH, OW, k, stride, pad, mode;
-  int pix_per_tile, total_pix;
+  int vec;              // elements per vector access (C % vec == 0)
+  long long items;      // output pixels x C/vec (window pools) | Nb x C/vec (global)
+  int per_tile;         // items per tile (window pools) | vector groups per tile (global)
 };
 
 template <typename T>
+struct VecT;  // 16-byte vector of T
+template <>
+struct VecT<__nv_bfloat16> {
+  static constexpr int N = 8;
+};
+template <>
+struct VecT<float> {
+  static constexpr int N = 4;
+};
+
+template <typename T, int V>
+__device__ __forceinline__ void load_vec(const T* p, float (&f)[V]) {
+  if constexpr (V == 1) {
+    f[0] = to_f(*p);
+  } else {
+    const uint4 u = __ldg(reinterpret_cast<const uint4*>(p));
+    const T* e = reinterpret_cast<const T*>(&u);
+#pragma unroll
+    for (int i = 0; i < V; ++i) f[i] = to_f(e[i]);
+  }
+}
+template <typename T, int V>
+__device__ __forceinline__ void store_vec(T* p, const float (&f)[V]) {
+  if constexpr (V == 1) {
+    stf(p, f[0]);
+  } else {
+    uint4 u;
+    T* e = reinterpret_cast<T*>(&u);
+#pragma unroll
+    for (int i = 0; i < V; ++i) {
+      if constexpr (sizeof(T) == 2) e[i] = __float2bfloat16_rn(f[i]);
+      else e[i] = f[i];
+    }
+    *reinterpret_cast<uint4*>(p) = u;
+  }
+}
+
+// Window pools: one thread per (output pixel, vector of channels); the k*k
+// window loads are independent 16-byte loads.  Global average: a tile is a
+// block of channel vectors x all pixels, split over 8 pixel slices and
+// reduced in shared memory.
+template <typename T, int V>
 struct Pool {
   using Params = PoolParams;
-  __device__ static void tile(const Params& p, int t, unsigned char*) {
+  __device__ static void tile(const Params& p, int t, unsigned char* smem) {
     const T* X = (const T*)p.X;
     T* Y = (T*)p.Y;
+    const int CV = p.C / V;
     if (p.mode == BL_POOL_GLOBAL_AVG) {
-      // tile = (image, 256-channel chunk)
-      const int cchunks = (p.C + 255) / 256;
-      const int n = t / cchunks, c = (t - n * cchunks) * 256 + threadIdx.x;
-      if (c >= p.C || threadIdx.x >= 256) return;
-      float s = 0.f;
+      // per_tile vector groups; 256 threads = per_tile groups x (256/per_tile) slices
+      const int gpt = p.per_tile, slices = blockDim.x / gpt;
+      const int tiles_per_img = (CV + gpt - 1) / gpt;
+      const int n = t / tiles_per_img, g0 = (t - n * tiles_per_img) * gpt;
+      const int gl = threadIdx.x % gpt, sl = threadIdx.x / gpt;
+      const int g = g0 + gl;
       const int hw = p.H * p.W;
-      for (int i = 0; i < hw; ++i) s += ldf(X + ((size_t)n * hw + i) * p.C + c);
-      stf(Y + (size_t)n * p.C + c, s / (float)hw);
-      return;
-    }
-    const int p0 = t * p.pix_per_tile;
-    const int npix = min(p.pix_per_tile, p.total_pix - p0);
-    for (int idx = threadIdx.x; idx < npix * p.C; idx += blockDim.x) {
-      const int pl = idx / p.C, c = idx - pl * p.C;
-      const int pix = p0 + pl;
-      const int n = pix / (p.OH * p.OW), q = pix - n * p.OH * p.OW;
-      const int oh = q / p.OW, ow = q - oh * p.OW;
-      float acc = (p.mode == BL_POOL_MAX) ? -INFINITY : 0.f;
-      for (int r = 0; r < p.k; ++r) {
-        const int ih = oh * p.stride - p.pad + r;
-        for (int s = 0; s < p.k; ++s) {
-          const int iw = ow * p.stride - p.pad + s;
-          if (ih < 0 || ih >= p.H || iw < 0 || iw >= p.W) continue;  // max: -inf pad; avg: 0 pad
-          const float v = ldf(X + ((size_t)(n * p.H + ih) * p.W + iw) * p.C + c);
-          acc = (p.mode == BL_POOL_MAX) ? fmaxf(acc, v) : acc + v;
+      float acc[V];
+#pragma unroll
+      for (int i = 0; i < V; ++i) acc[i] = 0.f;
+      if (g < CV) {
+        const T* base = X + (size_t)n * hw * p.C + (size_t)g * V;
+#pragma unroll 4
+        for (int px = sl; px < hw; px += slices) {
+          float f[V];
+          load_vec<T, V>(base + (size_t)px * p.C, f);
+#pragma unroll
+          for (int i = 0; i < V; ++i) acc[i] += f[i];
         }
       }
-      if (p.mode == BL_POOL_AVG) acc /= (float)(p.k * p.k);  // count_include_pad
-      stf(Y + (size_t)pix * p.C + c, acc);
+      float* red = reinterpret_cast<float*>(smem);  // [slices][gpt][V]
+      __syncthreads();
+#pragma unroll
+      for (int i = 0; i < V; ++i) red[(sl * gpt + gl) * V + i] = acc[i];
+      __syncthreads();
+      if (sl == 0 && g < CV) {
+        for (int s2 = 1; s2 < slices; ++s2)
+#pragma unroll
+          for (int i = 0; i < V; ++i) acc[i] += red[(s2 * gpt + gl) * V + i];
+#pragma unroll
+        for (int i = 0; i < V; ++i) acc[i] /= (float)hw;
+        store_vec<T, V>(Y + (size_t)n * p.C + (size_t)g * V, acc);
+      }
+      return;
+    }
+    const long long it0 = (long long)t * p.per_tile;
+    const long long it1 = min(it0 + p.per_tile, p.items);
+    for (long long it = it0 + threadIdx.x; it < it1; it += blockDim.x) {
+      const int cv = (int)(it % CV);
+      const long long pix = it / CV;
+      const int n = (int)(pix / (p.OH * p.OW));
+      const int q = (int)(pix - (long long)n * p.OH * p.OW);
+      const int oh = q / p.OW, ow = q - oh * p.OW;
+      float acc[V];
+#pragma unroll
+      for (int i = 0; i < V; ++i) acc[i] = (p.mode == BL_POOL_MAX) ? -INFINITY : 0.f;
+      const int h0 = oh * p.stride - p.pad, w0 = ow * p.stride - p.pad;
+      for (int r = 0; r < p.k; ++r) {
+        const int ih = h0 + r;
+        if (ih < 0 || ih >= p.H) continue;   // max: -inf padding; avg: zero padding (count_include_pad)
+#pragma unroll 3
+        for (int s = 0; s < p.k; ++s) {
+          const int iw = w0 + s;
+          if (iw < 0 || iw >= p.W) continue;
+          float f[V];
+          load_vec<T, V>(X + ((size_t)(n * p.H + ih) * p.W + iw) * p.C + (size_t)cv * V, f);
+#pragma unroll
+          for (int i = 0; i < V; ++i) acc[i] = (p.mode == BL_POOL_MAX) ? fmaxf(acc[i], f[i]) : acc[i] + f[i];
+        }
+      }
+      if (p.mode == BL_POOL_AVG) {
+#pragma unroll
+        for (int i = 0; i < V; ++i) acc[i] /= (float)(p.k * p.k);
+      }
+      store_vec<T, V>(Y + (size_t)pix * p.C + (size_t)cv * V, acc);
     }
   }
 };
@@ -247,18 +328,41 @@ struct Gemv {
       float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
       const T* wrow = W + (size_t)n * p.K;
       int k = k0 + lane * kVec;
-      const bool vec_ok = ((p.K % kVec) == 0) && ((k0 % kVec) == 0);
+      const bool vec_ok = ((p.K % kVec) == 0) && ((k0 % kVec) == 0) && ((p.ldx % kVec) == 0);
       if (vec_ok) {
-        for (; k + kVec <= k1; k += 32 * kVec) {
+        // kU independent 16-byte weight loads per lane in flight (memory-level
+        // parallelism: a batch-1 FC layer is a pure weight stream from HBM)
+        constexpr int kU = 8;
+        constexpr int kStep = 32 * kVec;
+        for (; k + (kU - 1) * kStep + kVec <= k1; k += kU * kStep) {
+          uint4 wv[kU];
+#pragma unroll
+          for (int u = 0; u < kU; ++u)
+            asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                         : "=r"(wv[u].x), "=r"(wv[u].y), "=r"(wv[u].z), "=r"(wv[u].w)
+                         : "l"(wrow + k + u * kStep));
+#pragma unroll
+          for (int u = 0; u < kU; ++u) {
+            const T* we = reinterpret_cast<const T*>(&wv[u]);
+            _Pragma("unroll") for (int m = 0; m < 8; ++m) if (m < p.M) {
+              float xf[kVec];
+              load_vec<T, kVec>(X + (size_t)m * p.ldx + k + u * kStep, xf);
+              float s = 0.f;
+#pragma unroll
+              for (int v = 0; v < kVec; ++v) s = fmaf(to_f(we[v]), xf[v], s);
+              acc[m] += s;
+            }
+          }
+        }
+        for (; k + kVec <= k1; k += kStep) {
           const uint4 wv = __ldg(reinterpret_cast<const uint4*>(wrow + k));
           const T* we = reinterpret_cast<const T*>(&wv);
-#pragma unroll
-          for (int m = 0; m < 8; ++m) {
-            if (m >= p.M) break;
-            const T* xr = X + (size_t)m * p.ldx + k;
+          _Pragma("unroll") for (int m = 0; m < 8; ++m) if (m < p.M) {
+            float xf[kVec];
+            load_vec<T, kVec>(X + (size_t)m * p.ldx + k, xf);
             float s = 0.f;
 #pragma unroll
-            for (int v = 0; v < kVec; ++v) s = fmaf(to_f(we[v]), ldf(xr + v), s);
+            for (int v = 0; v < kVec; ++v) s = fmaf(to_f(we[v]), xf[v], s);
             acc[m] += s;
           }
         }
@@ -268,7 +372,7 @@ struct Gemv {
           for (int m = 0; m < p.M && m < 8; ++m) acc[m] = fmaf(w, ldf(X + (size_t)m * p.ldx + k), acc[m]);
         }
       }
-      for (int m = 0; m < p.M && m < 8; ++m) {
+      _Pragma("unroll") for (int m = 0; m < 8; ++m) if (m < p.M) {
         float v = acc[m];
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
@@ -329,7 +433,7 @@ __global__ void __launch_bounds__(256) k_gated(const typename Op::Params p, cons
 template <class Op>
 static cudaError_t launch_gated(const KernelDesc& d, const GateArgs& g, cudaStream_t st) {
   void* args[2] = {(void*)d.params, (void*)&g};
-  return cudaLaunchKernel((const void*)k_gated<Op>, dim3(d.grid), dim3(d.block), args, (size_t)d.smem, st);
+  return launch_kernel((const void*)k_gated<Op>, dim3(d.grid), dim3(d.block), (size_t)d.smem, st, args);
 }
 
 static inline size_t esize(int dt) { return dt == BL_BF16 ? 2 : 4; }
@@ -422,20 +526,31 @@ bool build_simt(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::str
     p.X = op.ptr[0]; p.Y = op.ptr[1];
     p.Nb = (int)op.dims[0]; p.H = (int)op.dims[1]; p.W = (int)op.dims[2]; p.C = (int)op.dims[3];
     p.k = (int)op.dims[4]; p.stride = (int)op.dims[5]; p.pad = (int)op.dims[6]; p.mode = (int)op.dims[7];
+    if (p.C < 1 || p.Nb < 1) { err = "pool dims"; return false; }
+    const int V = bf ? 8 : 4;
+    const bool vec = (p.C % V) == 0 && (((uintptr_t)p.X | (uintptr_t)p.Y) & 15) == 0;
+    p.vec = vec ? V : 1;
+    const int CV = p.C / p.vec;
     if (p.mode == BL_POOL_GLOBAL_AVG) {
       p.OH = p.OW = 1;
-      d.tiles = (uint32_t)(p.Nb * ((p.C + 255) / 256));
+      p.per_tile = 16;                       // vector groups per tile (x 16 pixel slices)
+      d.tiles = (uint32_t)(p.Nb * ((CV + p.per_tile - 1) / p.per_tile));
+      d.smem = 256 * 8 * sizeof(float);
     } else {
       if (p.k < 1 || p.stride < 1) { err = "pool dims"; return false; }
       p.OH = (p.H + 2 * p.pad - p.k) / p.stride + 1;
       p.OW = (p.W + 2 * p.pad - p.k) / p.stride + 1;
-      p.total_pix = p.Nb * p.OH * p.OW;
-      p.pix_per_tile = std::max(1, 4096 / std::max(1, p.C));
-      d.tiles = (uint32_t)((p.total_pix + p.pix_per_tile - 1) / p.pix_per_tile);
+      p.items = (long long)p.Nb * p.OH * p.OW * CV;
+      // ~2 tiles per SM, one item per thread per pass, at least 256 items
+      long long per = (p.items + 2LL * caps.S - 1) / (2LL * caps.S);
+      per = std::max<long long>(256, (per + 255) / 256 * 256);
+      p.per_tile = (int)std::min<long long>(per, 1 << 16);
+      d.tiles = (uint32_t)((p.items + p.per_tile - 1) / p.per_tile);
+      d.smem = 0;
     }
-    d.smem = 0;
     std::memcpy(d.params, &p, sizeof(p));
-    d.launch = bf ? launch_gated<Pool<__nv_bfloat16>> : launch_gated<Pool<float>>;
+    if (bf) d.launch = vec ? launch_gated<Pool<__nv_bfloat16, 8>> : launch_gated<Pool<__nv_bfloat16, 1>>;
+    else d.launch = vec ? launch_gated<Pool<float, 4>> : launch_gated<Pool<float, 1>>;
     d.family = bf ? "pool_bf16" : "pool_f32";
     d.bytes = esize(op.dtype) * ((double)p.Nb * p.H * p.W * p.C + (double)p.Nb * p.OH * p.OW * p.C);
     return true;

@@ -41,6 +41,10 @@ struct TcParams {
   int mode;          // 0 GEMM, 1 conv stride 1 (4-D map), 2 conv stride 2 (5-D parity map)
   int tiles_n, num_kb;
   int OH, OW, BH, BW, tiles_w, C, R_, S_, pad, kc_per_tap;
+  // split-K: work unit u -> (tile u / splits, K blocks [ks*kbs, min(num_kb, (ks+1)*kbs)))
+  int splits, kbs;
+  float* ws;        // [tiles][128][BN] fp32 partial sums (zero between launches)
+  unsigned* sem;    // [tiles] arrival counters (zero between launches)
 };
 
 #ifdef __CUDACC__
@@ -150,6 +154,51 @@ __device__ __forceinline__ float act_f(float y, int act) {
   }
 }
 
+// Fused epilogue for 16 consecutive columns of one output row:
+// y = act(acc * scale + shift + R), rounded to bf16 (RNE), vector stores.
+__device__ __forceinline__ void epi_store16(const TcParams& p, int m, int n0, float (&y)[16]) {
+  const bool full16 = n0 + 16 <= p.N;
+  if (p.scale) {
+#pragma unroll
+    for (int i = 0; i < 16; ++i)
+      if (full16 || n0 + i < p.N) y[i] *= __ldg(p.scale + n0 + i);
+  }
+  if (p.shift) {
+#pragma unroll
+    for (int i = 0; i < 16; ++i)
+      if (full16 || n0 + i < p.N) y[i] += __ldg(p.shift + n0 + i);
+  }
+  if (p.R) {
+    const __nv_bfloat16* rr = p.R + (size_t)m * p.ldr + n0;
+    if (full16 && ((p.ldr & 7) == 0)) {
+      uint4 r0 = *reinterpret_cast<const uint4*>(rr);
+      uint4 r1 = *reinterpret_cast<const uint4*>(rr + 8);
+      const __nv_bfloat16* e0 = reinterpret_cast<const __nv_bfloat16*>(&r0);
+      const __nv_bfloat16* e1 = reinterpret_cast<const __nv_bfloat16*>(&r1);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        y[i] += __bfloat162float(e0[i]);
+        y[8 + i] += __bfloat162float(e1[i]);
+      }
+    } else {
+      for (int i = 0; i < 16; ++i)
+        if (n0 + i < p.N) y[i] += __bfloat162float(rr[i]);
+    }
+  }
+  __nv_bfloat16* yy = p.Y + (size_t)m * p.ldy + n0;
+  if (full16 && ((p.ldy & 7) == 0)) {
+    uint4 o[2];
+    __nv_bfloat162* ob = reinterpret_cast<__nv_bfloat162*>(o);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) ob[i] = __floats2bfloat162_rn(act_f(y[2 * i], p.act), act_f(y[2 * i + 1], p.act));
+    *reinterpret_cast<uint4*>(yy) = o[0];
+    *reinterpret_cast<uint4*>(yy + 8) = o[1];
+  } else {
+    for (int i = 0; i < 16; ++i)
+      if (n0 + i < p.N) yy[i] = __float2bfloat16_rn(act_f(y[i], p.act));
+  }
+}
+
 template <int BN, int BK>
 struct TcCfg {
   static constexpr int kStageA = 128 * BK * 2;
@@ -177,6 +226,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   uint64_t* rempty = rfull + 2;     // [2]
   int* ring = (int*)(rempty + 2);   // [2]
   uint32_t* tmem_slot = (uint32_t*)(ring + 2);
+  volatile int* last_flag = (volatile int*)(tmem_slot + 1);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
@@ -202,6 +252,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  pdl_wait();  // setup above overlapped the previous kernel; data reads start below
 
   if (warp == 0) {
     // ---------------- tile scheduler + TMA producer
@@ -219,15 +270,20 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         ring[rs] = t;
         mbar_arrive(&rfull[rs]);
         if (++rs == 2) { rs = 0; rph ^= 1; }
-        if (t < 0) break;
-        const int tm = t / p.tiles_n, tn = t - tm * p.tiles_n;
+        if (t < 0) {
+          pdl_trigger();  // queue exhausted: let the next kernel on this stream launch
+          break;
+        }
+        const int tile = t / p.splits, ks = t - tile * p.splits;
+        const int kb0 = ks * p.kbs, kb1 = min(p.num_kb, kb0 + p.kbs);
+        const int tm = tile / p.tiles_n, tn = tile - tm * p.tiles_n;
         int oh0 = 0, ow0 = 0;
         if (p.mode != 0) {
           const int th = tm / p.tiles_w;
           oh0 = th * p.BH;
           ow0 = (tm - th * p.tiles_w) * p.BW;
         }
-        for (int kb = 0; kb < p.num_kb; ++kb) {
+        for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
           mbar_expect_tx(&full[stage], Cfg::kStageBytes);
           unsigned char* a = sA + stage * Cfg::kStageA;
@@ -268,10 +324,12 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       if (lane == 0) mbar_arrive(&rempty[rs]);
       if (++rs == 2) { rs = 0; rph ^= 1; }
       if (t < 0) break;
+      const int ks = t % p.splits;
+      const int kb0 = ks * p.kbs, kb1 = min(p.num_kb, kb0 + p.kbs);
       mbar_wait(&tempty[acc], aph ^ 1);
       tc_fence_after();
       const uint32_t d_tmem = tmem_base + acc * BN;
-      for (int kb = 0; kb < p.num_kb; ++kb) {
+      for (int kb = kb0; kb < kb1; ++kb) {
         mbar_wait(&full[stage], phase);
         tc_fence_after();
         if (lane == 0) {
@@ -279,7 +337,8 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           const uint32_t b0 = smem_u32(sB + stage * Cfg::kStageB);
 #pragma unroll
           for (int k = 0; k < BK / 16; ++k) {
-            tc_mma(d_tmem, smem_desc<BK>(a0 + k * 32), smem_desc<BK>(b0 + k * 32), idesc, (kb | k) ? 1u : 0u);
+            tc_mma(d_tmem, smem_desc<BK>(a0 + k * 32), smem_desc<BK>(b0 + k * 32), idesc,
+                   (kb != kb0 || k) ? 1u : 0u);
           }
           tc_commit(&empty[stage]);
         }
@@ -304,7 +363,8 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       if (lane == 0) mbar_arrive(&rempty[rs]);
       if (++rs == 2) { rs = 0; rph ^= 1; }
       if (t < 0) break;
-      const int tm = t / p.tiles_n, tn = t - tm * p.tiles_n;
+      const int tile = t / p.splits;
+      const int tm = tile / p.tiles_n, tn = tile - tm * p.tiles_n;
       const int row = q * 32 + lane;
       int m;
       bool valid;
@@ -320,60 +380,64 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       mbar_wait(&tfull[acc], aph);
       tc_fence_after();
       const uint32_t tbase = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN;
+      if (p.splits == 1) {
 #pragma unroll 1
-      for (int c = 0; c < BN; c += 16) {
-        uint32_t v[16];
-        tmem_ld16(tbase + c, v);
-        tmem_ld_wait();
-        const int n0 = tn * BN + c;
-        if (!valid || n0 >= p.N) continue;
-        float y[16];
+        for (int c = 0; c < BN; c += 16) {
+          uint32_t v[16];
+          tmem_ld16(tbase + c, v);
+          tmem_ld_wait();
+          const int n0 = tn * BN + c;
+          if (!valid || n0 >= p.N) continue;
+          float y[16];
 #pragma unroll
-        for (int i = 0; i < 16; ++i) y[i] = __uint_as_float(v[i]);
-        const bool full16 = n0 + 16 <= p.N;
-        if (p.scale) {
-#pragma unroll
-          for (int i = 0; i < 16; ++i)
-            if (full16 || n0 + i < p.N) y[i] *= __ldg(p.scale + n0 + i);
+          for (int i = 0; i < 16; ++i) y[i] = __uint_as_float(v[i]);
+          epi_store16(p, m, n0, y);
         }
-        if (p.shift) {
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&tempty[acc]);
+      } else {
+        // split-K: add this unit's partial tile into the fp32 workspace
+        float* wrow = p.ws + ((size_t)tile * 128 + row) * BN;
+#pragma unroll 1
+        for (int c = 0; c < BN; c += 16) {
+          uint32_t v[16];
+          tmem_ld16(tbase + c, v);
+          tmem_ld_wait();
+          if (!valid || tn * BN + c >= p.N) continue;
 #pragma unroll
-          for (int i = 0; i < 16; ++i)
-            if (full16 || n0 + i < p.N) y[i] += __ldg(p.shift + n0 + i);
+          for (int i = 0; i < 16; i += 4)
+            asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(wrow + c + i), "f"(__uint_as_float(v[i])),
+                         "f"(__uint_as_float(v[i + 1])), "f"(__uint_as_float(v[i + 2])), "f"(__uint_as_float(v[i + 3]))
+                         : "memory");
         }
-        if (p.R) {
-          const __nv_bfloat16* rr = p.R + (size_t)m * p.ldr + n0;
-          if (full16 && ((p.ldr & 7) == 0)) {
-            uint4 r0 = *reinterpret_cast<const uint4*>(rr);
-            uint4 r1 = *reinterpret_cast<const uint4*>(rr + 8);
-            const __nv_bfloat16* e0 = reinterpret_cast<const __nv_bfloat16*>(&r0);
-            const __nv_bfloat16* e1 = reinterpret_cast<const __nv_bfloat16*>(&r1);
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&tempty[acc]);  // TMEM no longer needed
+        __threadfence();
+        asm volatile("bar.sync 1, 128;" ::: "memory");   // the 4 epilogue warps
+        if (threadIdx.x == 64) *last_flag = (atomicAdd(p.sem + tile, 1u) == (unsigned)p.splits - 1) ? 1 : 0;
+        asm volatile("bar.sync 1, 128;" ::: "memory");
+        if (*last_flag) {
+          __threadfence();
+          if (valid) {
+#pragma unroll 1
+            for (int c = 0; c < BN; c += 16) {
+              const int n0 = tn * BN + c;
+              if (n0 >= p.N) break;
+              float y[16];
 #pragma unroll
-            for (int i = 0; i < 8; ++i) {
-              y[i] += __bfloat162float(e0[i]);
-              y[8 + i] += __bfloat162float(e1[i]);
+              for (int i = 0; i < 16; i += 4) {
+                float4 f = __ldcg(reinterpret_cast<const float4*>(wrow + c + i));
+                y[i] = f.x; y[i + 1] = f.y; y[i + 2] = f.z; y[i + 3] = f.w;
+                __stcg(reinterpret_cast<float4*>(wrow + c + i), make_float4(0.f, 0.f, 0.f, 0.f));
+              }
+              epi_store16(p, m, n0, y);
             }
-          } else {
-            for (int i = 0; i < 16; ++i)
-              if (n0 + i < p.N) y[i] += __bfloat162float(rr[i]);
           }
-        }
-        __nv_bfloat16* yy = p.Y + (size_t)m * p.ldy + n0;
-        if (full16 && ((p.ldy & 7) == 0)) {
-          uint4 o[2];
-          __nv_bfloat162* ob = reinterpret_cast<__nv_bfloat162*>(o);
-#pragma unroll
-          for (int i = 0; i < 8; ++i) ob[i] = __floats2bfloat162_rn(act_f(y[2 * i], p.act), act_f(y[2 * i + 1], p.act));
-          *reinterpret_cast<uint4*>(yy) = o[0];
-          *reinterpret_cast<uint4*>(yy + 8) = o[1];
-        } else {
-          for (int i = 0; i < 16; ++i)
-            if (n0 + i < p.N) yy[i] = __float2bfloat16_rn(act_f(y[i], p.act));
+          if (threadIdx.x == 64) p.sem[tile] = 0;
         }
       }
-      tc_fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&tempty[acc]);
       if (++acc == 2) { acc = 0; aph ^= 1; }
     }
   }
@@ -389,6 +453,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
 template <int BN, int BK>
 __global__ void __launch_bounds__(192, 1) k_tc_gemm(const __grid_constant__ TcParams p, const GateArgs g) {
   if (gate_in_range(g)) tc_work<BN, BK>(p, g);
+  pdl_trigger();
   int last = 0;
   const bool fb = gate_leave(g, last);
   if (fb) tc_work<BN, BK>(p, g);
@@ -400,7 +465,7 @@ __global__ void __launch_bounds__(192, 1) k_tc_gemm(const __grid_constant__ TcPa
 template <int BN, int BK>
 static cudaError_t launch_tc(const KernelDesc& d, const GateArgs& g, cudaStream_t st) {
   void* args[2] = {(void*)d.params, (void*)&g};
-  return cudaLaunchKernel((const void*)k_tc_gemm<BN, BK>, dim3(d.grid), dim3(d.block), args, (size_t)d.smem, st);
+  return launch_kernel((const void*)k_tc_gemm<BN, BK>, dim3(d.grid), dim3(d.block), (size_t)d.smem, st, args);
 }
 
 template <int BN, int BK>
@@ -541,19 +606,40 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   }
   // N tile: as wide as possible while keeping >= S tiles when the problem allows
   const int tiles_m = (p.mode == 0) ? (p.M + 127) / 128 : p.tiles_w * ((p.OH + p.BH - 1) / p.BH);
-  int BN = 128;
-  if (p.N <= 16) BN = 16;
-  else if (p.N <= 32) BN = 32;
-  else if (p.N <= 64) BN = 64;
-  while (BN > 32 && (long long)tiles_m * ((p.N + BN - 1) / BN) < caps.S) BN >>= 1;
+  // N tile: the widest that still yields >= S tiles; if even 32 does not,
+  // split K (>= 3 K blocks per work unit) until there are ~S work units, so a
+  // batch-1 layer with few output tiles can still spread over every SM of its
+  // range (SURVEY.md §8(d) "elastic" kernels).
+  auto ntiles = [&](int bn) { return (long long)tiles_m * ((p.N + bn - 1) / bn); };
+  int BN = p.N <= 16 ? 16 : (p.N <= 32 ? 32 : (p.N <= 64 ? 64 : 128));
+  while (BN > 32 && ntiles(BN) < caps.S) BN >>= 1;
   p.tiles_n = (p.N + BN - 1) / BN;
+  int splits = 1;
+  if (ntiles(BN) < caps.S) {
+    const int want = (int)((caps.S + ntiles(BN) - 1) / ntiles(BN));
+    splits = std::max(1, std::min(want, p.num_kb / 3));
+  }
+  p.kbs = (p.num_kb + splits - 1) / splits;
+  p.splits = (p.num_kb + p.kbs - 1) / p.kbs;
+  if (p.splits > 1) {
+    const size_t nt = (size_t)ntiles(BN);
+    const size_t wsb = nt * 128 * BN * sizeof(float);
+    void* buf = nullptr;
+    if (cudaMalloc(&buf, wsb + nt * sizeof(unsigned)) != cudaSuccess ||
+        cudaMemset(buf, 0, wsb + nt * sizeof(unsigned)) != cudaSuccess) {
+      err = "split-K workspace alloc";
+      return false;
+    }
+    p.ws = (float*)buf;
+    p.sem = (unsigned*)((char*)buf + wsb);
+  }
   {
     cuuint64_t db[2] = {(cuuint64_t)p.K, (cuuint64_t)p.N}, sb[1] = {(cuuint64_t)p.K * 2};
     cuuint32_t bb[2] = {(cuuint32_t)BK, (cuuint32_t)BN};
     if (!encode(&p.tmB, 2, W, db, sb, bb, BK, err)) return false;
   }
   d.op = op;
-  d.tiles = (uint32_t)(tiles_m * p.tiles_n);
+  d.tiles = (uint32_t)(tiles_m * p.tiles_n * p.splits);
   d.block = 192;
   d.grid = caps.S;
   bool ok = false;

@@ -7,11 +7,14 @@
 #include <atomic>
 #include <chrono>
 #include <cstring>
+#include <cstdlib>
 #include <thread>
 
 #include "../kernels/executor.cuh"
 
 namespace bless {
+
+int g_use_pdl = 1;
 
 static int64_t host_now_ns() {
   return std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now().time_since_epoch())
@@ -106,15 +109,23 @@ std::unique_ptr<DeviceRT> DeviceRT::create(int device, void* ws, size_t ws_bytes
     rt->own_slots_ = true;
   }
   if (cudaMemset(rt->slots_, 0, slot_bytes) != cudaSuccess) { err = "memset slots"; return nullptr; }
-  if (cudaHostAlloc(&rt->stats_host_, kSlotRing * sizeof(SlotStats), cudaHostAllocMapped) != cudaSuccess) {
-    err = "cudaHostAlloc stats";
+  // stats ring in device memory + pinned host mirror refreshed by async copies
+  if (cudaMalloc(&rt->stats_dev_, kSlotRing * sizeof(SlotStats)) != cudaSuccess ||
+      cudaMemset(rt->stats_dev_, 0, kSlotRing * sizeof(SlotStats)) != cudaSuccess) {
+    err = "cudaMalloc stats";
+    return nullptr;
+  }
+  if (cudaHostAlloc(&rt->stats_host_, kSlotRing * sizeof(SlotStats), cudaHostAllocDefault) != cudaSuccess) {
+    err = "cudaHostAlloc stats mirror";
     return nullptr;
   }
   std::memset(rt->stats_host_, 0, kSlotRing * sizeof(SlotStats));
-  if (cudaHostGetDevicePointer(&rt->stats_dev_, rt->stats_host_, 0) != cudaSuccess) {
-    err = "cudaHostGetDevicePointer";
+  if (cudaStreamCreateWithPriority((cudaStream_t*)&rt->reader_, cudaStreamNonBlocking, 0) != cudaSuccess ||
+      cudaEventCreateWithFlags((cudaEvent_t*)&rt->reader_ev_, cudaEventDisableTiming) != cudaSuccess) {
+    err = "reader stream";
     return nullptr;
   }
+  if (const char* e = std::getenv("BLESS_PDL")) g_use_pdl = std::atoi(e) != 0;
   if (!rt->probe(err)) return nullptr;
   if (!rt->calibrate_clock(err)) return nullptr;
   return rt;
@@ -124,7 +135,10 @@ DeviceRT::~DeviceRT() {
   cudaSetDevice(device_);
   cudaDeviceSynchronize();
   if (own_slots_ && slots_) cudaFree(slots_);
+  if (stats_dev_) cudaFree(stats_dev_);
   if (stats_host_) cudaFreeHost(stats_host_);
+  if (reader_ev_) cudaEventDestroy((cudaEvent_t)reader_ev_);
+  if (reader_) cudaStreamDestroy((cudaStream_t)reader_);
   if (lid_map_dev_) cudaFree(lid_map_dev_);
 }
 
@@ -219,18 +233,23 @@ int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
   return (int)kernels_.size() - 1;
 }
 
+GateArgs DeviceRT::make_gate(uint64_t seq, uint32_t tiles, int lo, int hi) const {
+  GateArgs g;
+  g.slot = reinterpret_cast<DevSlot*>(slots_) + seq % kSlotRing;
+  g.stats = reinterpret_cast<SlotStats*>(stats_dev_) + seq % kSlotRing;
+  g.stats_ahead = reinterpret_cast<SlotStats*>(stats_dev_) + (seq + kMaskAhead) % kSlotRing;
+  g.lid_map = identity_map_ ? nullptr : lid_map_dev_;
+  g.seq = seq;
+  g.tiles = tiles;
+  g.lo = lo;
+  g.hi = hi;
+  return g;
+}
+
 uint64_t DeviceRT::launch(int h, int lo, int hi, void* stream, std::string& err) {
   const KernelDesc& kd = *kernels_[h];
   const uint64_t seq = ++seq_;
-  const uint64_t slot = seq % kSlotRing;
-  GateArgs g;
-  g.slot = reinterpret_cast<DevSlot*>(slots_) + slot;
-  g.stats = reinterpret_cast<SlotStats*>(stats_dev_) + slot;
-  g.lid_map = identity_map_ ? nullptr : lid_map_dev_;
-  g.seq = seq;
-  g.tiles = kd.tiles;
-  g.lo = lo;
-  g.hi = hi;
+  const GateArgs g = make_gate(seq, kd.tiles, lo, hi);
   const cudaError_t e = kd.launch(kd, g, (cudaStream_t)stream);
   if (e != cudaSuccess) {
     err = std::string("launch ") + kd.family + ": " + cudaGetErrorString(e);
@@ -248,15 +267,8 @@ __global__ void k_marker(const GateArgs g) {
 
 uint64_t DeviceRT::launch_marker(void* stream, std::string& err) {
   const uint64_t seq = ++seq_;
-  const uint64_t slot = seq % kSlotRing;
-  GateArgs g;
-  g.slot = reinterpret_cast<DevSlot*>(slots_) + slot;
-  g.stats = reinterpret_cast<SlotStats*>(stats_dev_) + slot;
+  GateArgs g = make_gate(seq, 0, 0, 0);
   g.lid_map = nullptr;
-  g.seq = seq;
-  g.tiles = 0;
-  g.lo = 0;
-  g.hi = 0;
   k_marker<<<1, 32, 0, (cudaStream_t)stream>>>(g);
   const cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) {
@@ -266,18 +278,116 @@ uint64_t DeviceRT::launch_marker(void* stream, std::string& err) {
   return seq;
 }
 
+// ---------------------------------------------------------------- diagnostics
+__global__ void k_empty() {}
+__global__ void k_gate_only(const GateArgs g, int publish) {
+  __shared__ int s_t;
+  bool marked = false;
+  if (gate_in_range(g)) {
+    pdl_wait();
+    for (;;) {
+      if (threadIdx.x == 0) s_t = gate_claim(g, marked);
+      __syncthreads();
+      const int t = s_t;
+      __syncthreads();
+      if (t < 0) break;
+    }
+  }
+  pdl_trigger();
+  int last = 0;
+  const bool fb = gate_leave(g, last);
+  if (last) {
+    if (publish) {
+      gate_finalize(g, fb);
+    } else if (threadIdx.x == 0) {
+      g.slot->ctr = 0ull;
+    }
+  }
+}
+
+bool DeviceRT::overhead(int variant, int reps, int64_t* ns_out, std::string& err) {
+  cudaStream_t s = nullptr;
+  RT_CHECK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  cudaEvent_t e0, e1;
+  RT_CHECK(cudaEventCreate(&e0));
+  RT_CHECK(cudaEventCreate(&e1));
+  const int S = info_.sm_count;
+  const int saved_pdl = g_use_pdl;
+  g_use_pdl = variant == 3 ? 1 : 0;
+  auto one = [&]() {
+    const uint64_t seq = ++seq_;
+    const GateArgs g = make_gate(seq, 1, 0, S);
+    if (variant == 0) {
+      k_empty<<<S, 192, 0, s>>>();
+    } else {
+      int publish = variant >= 2 ? 1 : 0;
+      void* args[2] = {(void*)&g, (void*)&publish};
+      launch_kernel((const void*)k_gate_only, dim3(S), dim3(192), 0, s, args);
+    }
+  };
+  for (int i = 0; i < 10; ++i) one();
+  RT_CHECK(cudaEventRecord(e0, s));
+  for (int i = 0; i < reps; ++i) one();
+  RT_CHECK(cudaEventRecord(e1, s));
+  RT_CHECK(cudaEventSynchronize(e1));
+  float ms = 0;
+  RT_CHECK(cudaEventElapsedTime(&ms, e0, e1));
+  *ns_out = (int64_t)(ms * 1e6 / reps);
+  g_use_pdl = saved_pdl;
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaStreamDestroy(s);
+  return true;
+}
+
 bool DeviceRT::memcpy_async(void* dst, const void* src, size_t n, void* stream) {
   return cudaMemcpyAsync(dst, src, n, cudaMemcpyDefault, (cudaStream_t)stream) == cudaSuccess;
 }
 
-bool DeviceRT::poll(uint64_t seq, LaunchStats* out) const {
+void DeviceRT::copy_range(uint64_t lo, uint64_t hi) {
+  if (hi < lo) return;
+  uint64_t n = std::min<uint64_t>(hi - lo + 1, kSlotRing);
+  const uint64_t s0 = lo % kSlotRing;
+  const uint64_t n1 = std::min<uint64_t>(n, kSlotRing - s0);
+  char* h = reinterpret_cast<char*>(stats_host_);
+  const char* d = reinterpret_cast<const char*>(stats_dev_);
+  cudaMemcpyAsync(h + s0 * sizeof(SlotStats), d + s0 * sizeof(SlotStats), n1 * sizeof(SlotStats),
+                  cudaMemcpyDeviceToHost, (cudaStream_t)reader_);
+  if (n > n1)
+    cudaMemcpyAsync(h, d, (n - n1) * sizeof(SlotStats), cudaMemcpyDeviceToHost, (cudaStream_t)reader_);
+}
+
+bool DeviceRT::reader_idle() {
+  if (!reader_busy_) return true;
+  if (cudaEventQuery((cudaEvent_t)reader_ev_) != cudaSuccess) return false;
+  reader_busy_ = false;
+  return true;
+}
+
+void DeviceRT::refresh_async(uint64_t lo, uint64_t hi) {
+  if (!reader_idle()) return;
+  copy_range(lo, hi);
+  cudaEventRecord((cudaEvent_t)reader_ev_, (cudaStream_t)reader_);
+  reader_busy_ = true;
+}
+
+void DeviceRT::refresh_sync(uint64_t lo, uint64_t hi) {
+  copy_range(lo, hi);
+  cudaStreamSynchronize((cudaStream_t)reader_);
+  reader_busy_ = false;
+}
+
+bool DeviceRT::poll(uint64_t seq, LaunchStats* out) {
+  if (!reader_idle()) return false;  // never read the mirror while a copy is landing
   const volatile SlotStats* s = reinterpret_cast<const volatile SlotStats*>(stats_host_) + (seq % kSlotRing);
   if (s->seq != seq) return false;
   std::atomic_thread_fence(std::memory_order_acquire);
   if (out) {
     out->start_host = gt_to_host(s->start_gt);
     out->end_host = gt_to_host(s->end_gt);
-    out->nsm = (int)s->nsm;
+    int nsm = 0;
+    for (int i = 0; i < 8; ++i) nsm += __builtin_popcount(s->mask[i]);
+    out->nsm = nsm;
     out->fallback = (int)(s->flags & 1u);
     for (int i = 0; i < 8; ++i) out->mask[i] = s->mask[i];
   }
@@ -321,9 +431,11 @@ bool DeviceRT::profile(int h, int sm_count, int reps, void* stream, int64_t* ns_
     const uint64_t q = launch(h, 0, S, s, err);
     if (!q) return false;
     RT_CHECK(cudaStreamSynchronize(s));
+    refresh_sync(q, q);
     LaunchStats st{};
-    int spins = 0;
-    while (!poll(q, &st) && spins++ < 1000000) {
+    if (!poll(q, &st)) {
+      err = "profile: launch stats missing";
+      return false;
     }
     *d_out = std::max(1, st.nsm);
   }

@@ -36,8 +36,17 @@ class DeviceRT {
   // One-CTA completion marker (stats only, no work) on stream; returns seq or 0.
   uint64_t launch_marker(void* stream, std::string& err);
   bool memcpy_async(void* dst, const void* src, size_t n, void* stream);
-  // Non-blocking: true if launch seq has published its stats.
-  bool poll(uint64_t seq, LaunchStats* out) const;
+  // Diagnostics: per-launch time of back-to-back S-CTA launches.  variant 0:
+  // empty kernel; 1: gate + tile queue + exit protocol; 2: 1 + host-mapped stamps.
+  bool overhead(int variant, int reps, int64_t* ns_out, std::string& err);
+  // Non-blocking: true if launch seq's stats are in the host mirror.
+  bool poll(uint64_t seq, LaunchStats* out);
+  // Mirror the device stats of launches [lo, hi] (seq numbers) into host
+  // memory: asynchronously (skipped while a previous copy is in flight) or
+  // synchronously (after the launches are known complete).
+  void refresh_async(uint64_t lo, uint64_t hi);
+  void refresh_sync(uint64_t lo, uint64_t hi);
+  uint64_t last_seq() const { return seq_; }
 
   // Streams / events (thin wrappers so the engine does not include CUDA headers).
   void* stream_create();
@@ -58,6 +67,7 @@ class DeviceRT {
 
   int64_t gt_to_host(int64_t gt) const { return gt - info_.clock_offset_ns; }
   bool calibrate_clock(std::string& err);
+  GateArgs make_gate(uint64_t seq, uint32_t tiles, int lo, int hi) const;
 
  private:
   DeviceRT() = default;
@@ -68,8 +78,13 @@ class DeviceRT {
   DeviceCaps caps_{};
   void* slots_ = nullptr;        // DevSlot ring (device)
   bool own_slots_ = false;
-  void* stats_host_ = nullptr;   // SlotStats ring (host-mapped)
-  void* stats_dev_ = nullptr;
+  void copy_range(uint64_t lo, uint64_t hi);
+  bool reader_idle();
+  void* stats_host_ = nullptr;   // pinned host mirror of the SlotStats ring
+  void* stats_dev_ = nullptr;    // SlotStats ring (device memory)
+  void* reader_ = nullptr;       // stream for mirror copies (copy engine)
+  void* reader_ev_ = nullptr;
+  bool reader_busy_ = false;
   uint8_t* lid_map_dev_ = nullptr;
   bool identity_map_ = true;
   uint64_t seq_ = 0;

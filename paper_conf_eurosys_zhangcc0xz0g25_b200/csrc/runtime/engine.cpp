@@ -149,6 +149,14 @@ bl_status Engine::set_io(int t, const void* hin, void* din, size_t inb, const vo
   return BL_OK;
 }
 
+bl_status Engine::debug_overhead(int variant, int reps, int64_t* ns, std::string& err) {
+  if (!rt_) { err = "no device"; return BL_E_STATE; }
+  if (started_) { err = "diagnostics while running"; return BL_E_STATE; }
+  if (!ns || variant < 0 || variant > 3 || reps < 1) { err = "bad args"; return BL_E_INVALID; }
+  rt_->set_device();
+  return rt_->overhead(variant, reps, ns, err) ? BL_OK : BL_E_CUDA;
+}
+
 bl_status Engine::kernel_info(int t, int k, bl_kernel_info* out, std::string& err) {
   if (!rt_) { err = "no device"; return BL_E_STATE; }
   if (t < 0 || t >= nten() || k < 0 || k >= (int)ten_[t].handles.size() || !out) { err = "bad index"; return BL_E_INVALID; }
@@ -300,6 +308,7 @@ bl_status Engine::start(std::string& err) {
   fifo_.assign(nten(), {});
   scan_ = 0;
   pending_.clear();
+  if (rt_) run_first_seq_ = rt_->last_seq() + 1;
   inflight_.clear();
   prev_events_.clear();
   stop_ = false;
@@ -370,7 +379,25 @@ bl_status Engine::stop(std::string& err) {
   if (rt_ && started_) {
     rt_->set_device();
     if (!rt_->device_sync()) { err = "device error at stop"; started_ = false; return BL_E_CUDA; }
+    // every launch of the run has finished: mirror the whole stats range once
+    // (includes the SM masks) and complete the logs
+    const uint64_t hi = rt_->last_seq();
+    const uint64_t lo = hi >= run_first_seq_ ? std::max<uint64_t>(run_first_seq_, hi > kSlotRing ? hi - kSlotRing + 1 : 1) : hi + 1;
+    rt_->refresh_sync(lo, hi);
+    harvest_all_ = true;
     harvest();
+    harvest_all_ = false;
+    std::lock_guard<std::mutex> lk(log_mu_);
+    for (bl_launch_rec& r : llog_) {
+      LaunchStats st;
+      if (r.seq >= lo && rt_->poll(r.seq, &st)) {
+        r.start_ns = st.start_host;
+        r.end_ns = st.end_host;
+        r.nsm = st.nsm;
+        r.fallback = st.fallback;
+        for (int i = 0; i < 8; ++i) r.sm_mask[i] = st.mask[i];
+      }
+    }
   }
   started_ = false;
   if (failed_) { err = fail_msg_; return BL_E_CUDA; }
@@ -541,6 +568,14 @@ uint64_t Engine::launch_one(int t, int k, int lo, int hi, void* stream, int64_t 
 
 void Engine::harvest() {
   if (!rt_ || pending_.empty()) return;
+  if (!harvest_all_) {
+    // mirror the pending launches' stats (copy engine), at most every 25 us
+    const int64_t t = now_ns();
+    if (t - last_refresh_ns_ >= 25000) {
+      rt_->refresh_async(pending_.front().seq, pending_.back().seq);
+      last_refresh_ns_ = t;
+    }
+  }
   size_t w = 0;
   for (size_t i = 0; i < pending_.size(); ++i) {
     PendingLaunch& p = pending_[i];

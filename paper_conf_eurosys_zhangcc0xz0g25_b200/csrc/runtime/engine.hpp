@@ -64,6 +64,7 @@ class Engine {
   bl_status append_kernel(int t, const bl_op* op, int* out, std::string& err);
   bl_status run_kernel(int t, int k, int lo, int hi, std::string& err);
   bl_status kernel_info(int t, int k, bl_kernel_info* out, std::string& err);
+  bl_status debug_overhead(int variant, int reps, int64_t* ns, std::string& err);
   bl_status set_io(int t, const void* hin, void* din, size_t inb, const void* dout, void* hout, size_t outb,
                    std::string& err);
   bl_status profile_kernel(int t, int k, int sm_count, int reps, int64_t* ns, int* d, std::string& err);
@@ -129,6 +130,9 @@ class Engine {
   DecideScratch scratch_;
   Decision dec_;
   std::vector<PendingLaunch> pending_;
+  uint64_t run_first_seq_ = 1;
+  int64_t last_refresh_ns_ = 0;
+  bool harvest_all_ = false;
   struct Inflight {
     std::vector<void*> events;
   };
