@@ -41,5 +41,6 @@ bool build_kernel(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std:
 // Per-family builders (return true if they took the op).
 bool build_simt(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
 bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
+bool build_gemv_tma(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
 
 }  // namespace bless
