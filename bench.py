@@ -51,6 +51,8 @@ def parse():
     ap.add_argument("--profile-reps", type=int, default=5)
     ap.add_argument("--no-baselines", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--load-profile", default="", help="reuse a saved profile table instead of profiling")
+    ap.add_argument("--light", action="store_true", help="timed steps only (for ncu launch lists)")
     ap.add_argument("--out-dir", default=os.path.join(ROOT, "gpurun_out"))
     return ap.parse_args()
 
@@ -113,6 +115,35 @@ def stats(xs):
         return {}
     rank = lambda p: xs[max(0, int(np.ceil(p / 100 * len(xs))) - 1)]  # noqa: E731
     return {"mean_ms": float(np.mean(xs)) / 1e6, "p50_ms": rank(50) / 1e6, "p99_ms": rank(99) / 1e6, "n": len(xs)}
+
+
+def squad_timeline(decisions, launches):
+    """Map each BLESS decision to its launches (logged in pick order) and
+    measure: squad makespan vs the predicted t_hat (Eq. 1 for SP, Eq. 2 for
+    NSP; PAPER.md L214/L227 report 6.7%/7.1% error on A100) and the GPU idle
+    gap between consecutive squads (L432: 20 us squad switch on A100)."""
+    i = 0
+    spans = []
+    for d in decisions:
+        ls = launches[i:i + d.n_picks]
+        i += d.n_picks
+        if len(ls) != d.n_picks or any(r.end_ns <= 0 for r in ls):
+            continue
+        spans.append((min(r.start_ns for r in ls), max(r.end_ns for r in ls), d.t_hat, bool(d.config_sp)))
+    if not spans:
+        return {}
+    err = {True: [], False: []}
+    gaps = []
+    for a, b in zip(spans, spans[1:]):
+        gaps.append(max(0, b[0] - a[1]))
+    for s, e, th, sp in spans:
+        err[sp].append(abs((e - s) - th) / max(1, e - s))
+    return {"squads": len(spans),
+            "pred_err_sp_pct": 100 * float(np.mean(err[True])) if err[True] else None,
+            "pred_err_nsp_pct": 100 * float(np.mean(err[False])) if err[False] else None,
+            "gap_us_median": float(np.median(gaps)) / 1e3 if gaps else None,
+            "gap_us_mean": float(np.mean(gaps)) / 1e3 if gaps else None,
+            "makespan_us_median": float(np.median([e - s for s, e, _, _ in spans])) / 1e3}
 
 
 def make_trace(T_iso, rho, n, seed):
@@ -201,8 +232,11 @@ def native(args):
     tms = models.build_config(ctx, args.config, dtype)
     names = [m.name for m in tms]
     t_prof = time.perf_counter()
-    for m in tms:
-        ctx.profile_tenant(m.tenant, reps=args.profile_reps)
+    if args.load_profile:
+        ctx.load_profile(args.load_profile)
+    else:
+        for m in tms:
+            ctx.profile_tenant(m.tenant, reps=args.profile_reps)
     t_prof = time.perf_counter() - t_prof
     os.makedirs(args.out_dir, exist_ok=True)
     prof_path = os.path.join(args.out_dir, f"profile_{args.config}_rank{rank}.txt")
@@ -223,6 +257,7 @@ def native(args):
     # ---------------- timed region: K BLESS steps
     lat_all = {j: [] for j in range(len(tms))}
     launches_all, decisions_all = [], []
+    timelines = []
     if dist:
         dist.barrier()
     torch.cuda.synchronize()
@@ -235,6 +270,7 @@ def native(args):
                 lat_all[j].extend(v)
             launches_all.extend(launches)
             decisions_all.extend(decisions)
+            timelines.append((decisions, launches))
         torch.cuda.synchronize()
         t1 = time.perf_counter()
     step_ms = (t1 - t0) * 1e3 / args.steps
@@ -245,6 +281,12 @@ def native(args):
         dist.barrier()
     n_req = sum(len(v) for v in lat_all.values())
     mean_ms = float(np.mean([x for v in lat_all.values() for x in v])) / 1e6
+    if args.light:
+        if rank == 0:
+            print(json.dumps({"metric": METRIC, "value": mean_ms, "unit": "ms", "light": True,
+                              "gpu_launches": len(launches_all), "ms_per_step": step_ms}))
+        ctx.close()
+        return
 
     # ---------------- in-run baselines on the seed-1 trace
     per_tenant = {}
@@ -374,7 +416,8 @@ def native(args):
         "e2e": e2e, "gpu_launches": gpu_launches, "roofline": roofline, "cpu_baseline": cpu,
         "clocks": clk.summary(),
         "scheduler": {"decisions": len(decisions_all), "sp_squads": sp_squads, "fallback_launches": fallbacks,
-                      "oracle_replay_bit_exact": replay_ok, "profile_s": t_prof},
+                      "oracle_replay_bit_exact": replay_ok, "profile_s": t_prof,
+                      "timeline": squad_timeline(*timelines[0]) if timelines else {}},
         "device": {"sm_count": S, "globaltimer_res_ns": info.globaltimer_res_ns, "host_cores": os.cpu_count()},
     }
     if rank == 0:

@@ -114,6 +114,23 @@ __device__ __forceinline__ void gate_tile_loop(const GateArgs& g, Body&& body) {
   }
 }
 
+// Out-of-range CTAs linger until some in-range CTA has claimed a tile (or a
+// bounded timeout): otherwise, when the kernel's own SMs are still busy (e.g.
+// its predecessor under programmatic dependent launch, or another tenant's
+// CTAs), every CTA of the grid could be placed out of range and leave, and
+// the work would fall back to a single CTA.  The timeout breaks mutual waits
+// between tenants.
+constexpr uint64_t kLingerNs = 30000;
+__device__ __forceinline__ void gate_linger(const GateArgs& g) {
+  if (threadIdx.x == 0 && g.tiles > 0 && g.lo < g.hi) {
+    const uint64_t t0 = ptx_globaltimer();
+    while ((uint32_t)(*reinterpret_cast<volatile unsigned long long*>(&g.slot->ctr)) == 0u) {
+      if (ptx_globaltimer() - t0 > kLingerNs) break;
+      __nanosleep(256);
+    }
+  }
+}
+
 // Exit protocol.  Returns true if THIS CTA must run the work loop as the
 // fallback (see header).  All threads of the CTA must call it.
 __device__ __forceinline__ bool gate_leave(const GateArgs& g, int& is_last) {
@@ -156,6 +173,8 @@ __device__ __forceinline__ void gated_run(const typename Op::Params& p, const Ga
   if (gate_in_range(g)) {
     pdl_wait();
     gate_tile_loop(g, [&](int t) { Op::tile(p, t, smem); });
+  } else {
+    gate_linger(g);
   }
   pdl_trigger();
   int last = 0;

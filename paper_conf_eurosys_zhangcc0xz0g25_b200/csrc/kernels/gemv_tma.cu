@@ -231,6 +231,7 @@ __device__ void gemv_work(const GemvTmaParams& p, const GateArgs& g) {
 template <int MAXM>
 __global__ void __launch_bounds__(kGvThreads, 2) k_gemv_tma(const GemvTmaParams p, const GateArgs g) {
   if (gate_in_range(g)) gemv_work<MAXM>(p, g);
+  else gate_linger(g);
   pdl_trigger();
   int last = 0;
   const bool fb = gate_leave(g, last);
