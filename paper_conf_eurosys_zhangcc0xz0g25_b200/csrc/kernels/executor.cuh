@@ -120,15 +120,40 @@ __device__ __forceinline__ void gate_tile_loop(const GateArgs& g, Body&& body) {
 // CTAs), every CTA of the grid could be placed out of range and leave, and
 // the work would fall back to a single CTA.  The timeout breaks mutual waits
 // between tenants.
+// Under programmatic dependent launch the busy in-range SMs are most often
+// held by this kernel's own predecessor on the stream, so a lingering CTA
+// first waits for that grid to complete (it cannot deadlock: all of the
+// predecessor's CTAs are resident when dependents launch) and only then starts
+// the bounded wait for an in-range CTA.
+// Grids are sized to the kernel's full occupancy (S x blocks/SM), so lingering
+// CTAs on out-of-range SMs can never absorb the whole grid: some CTAs stay
+// queued until the window frees up.  If no in-range CTA has claimed a tile
+// when the bounded wait expires (e.g. two tenants' lingering CTAs blocking
+// each other's windows), the CTA returns true and helps drain the queue (a
+// bounded, flagged confinement violation instead of a stalled kernel).
 constexpr uint64_t kLingerNs = 30000;
-__device__ __forceinline__ void gate_linger(const GateArgs& g) {
-  if (threadIdx.x == 0 && g.tiles > 0 && g.lo < g.hi) {
-    const uint64_t t0 = ptx_globaltimer();
-    while ((uint32_t)(*reinterpret_cast<volatile unsigned long long*>(&g.slot->ctr)) == 0u) {
-      if (ptx_globaltimer() - t0 > kLingerNs) break;
-      __nanosleep(256);
+__device__ __forceinline__ bool gate_linger(const GateArgs& g) {
+  __shared__ int s_steal;
+  if (threadIdx.x == 0) {
+    int steal = 0;
+    if (g.tiles > 0 && g.lo < g.hi) {
+      pdl_wait();
+      const uint64_t t0 = ptx_globaltimer();
+      for (;;) {
+        const unsigned long long c = *reinterpret_cast<volatile unsigned long long*>(&g.slot->ctr);
+        if ((uint32_t)c != 0u) break;
+        if (ptx_globaltimer() - t0 > kLingerNs) {
+          steal = 1;
+          break;
+        }
+        __nanosleep(256);
+      }
+      if (steal) atomicOr(&g.stats->flags, 2u);
     }
+    s_steal = steal;
   }
+  __syncthreads();
+  return s_steal != 0;
 }
 
 // Exit protocol.  Returns true if THIS CTA must run the work loop as the
@@ -156,8 +181,9 @@ __device__ __forceinline__ void gate_finalize(const GateArgs& g, bool fallback) 
     SlotStats* out = g.stats;
     out->end_gt = (int64_t)end;
     if (g.tiles == 0) out->start_gt = (int64_t)end;
-    out->flags = fallback ? 1u : 0u;
-    // zero the mask of the record reused kMaskAhead launches from now
+    if (fallback) atomicOr(&out->flags, 1u);
+    // zero the flags and mask of the record reused kMaskAhead launches from now
+    g.stats_ahead->flags = 0u;
     uint4* fm = reinterpret_cast<uint4*>(g.stats_ahead->mask);
     fm[0] = make_uint4(0, 0, 0, 0);
     fm[1] = make_uint4(0, 0, 0, 0);
@@ -170,11 +196,9 @@ __device__ __forceinline__ void gate_finalize(const GateArgs& g, bool fallback) 
 // The canonical gated kernel body for tile-loop ops: Op::tile(params, t, smem).
 template <class Op>
 __device__ __forceinline__ void gated_run(const typename Op::Params& p, const GateArgs& g, unsigned char* smem) {
-  if (gate_in_range(g)) {
+  if (gate_in_range(g) || gate_linger(g)) {
     pdl_wait();
     gate_tile_loop(g, [&](int t) { Op::tile(p, t, smem); });
-  } else {
-    gate_linger(g);
   }
   pdl_trigger();
   int last = 0;
@@ -190,6 +214,12 @@ __device__ __forceinline__ void gated_run(const typename Op::Params& p, const Ga
 // Host: launch with programmatic stream serialization (PDL) unless disabled.
 extern int g_use_pdl;
 #ifdef __CUDACC__
+// Grid = S x (resident blocks per SM for this kernel), capped at 8 per SM.
+inline int full_occupancy_grid(const void* fn, int block, size_t smem, int S) {
+  int occ = 1;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, block, smem) != cudaSuccess || occ < 1) occ = 1;
+  return S * (occ > 8 ? 8 : occ);
+}
 inline cudaError_t launch_kernel(const void* fn, dim3 grid, dim3 block, size_t smem, cudaStream_t st, void** args) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = grid;

@@ -230,8 +230,7 @@ __device__ void gemv_work(const GemvTmaParams& p, const GateArgs& g) {
 
 template <int MAXM>
 __global__ void __launch_bounds__(kGvThreads, 2) k_gemv_tma(const GemvTmaParams p, const GateArgs g) {
-  if (gate_in_range(g)) gemv_work<MAXM>(p, g);
-  else gate_linger(g);
+  if (gate_in_range(g) || gate_linger(g)) gemv_work<MAXM>(p, g);
   pdl_trigger();
   int last = 0;
   const bool fb = gate_leave(g, last);
@@ -291,6 +290,7 @@ bool build_gemv_tma(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std:
   d.block = kGvThreads;
   d.smem = kGvSmem;
   d.launch = m1 ? launch_gemv_tma<1> : launch_gemv_tma<8>;
+  d.kernel_fn = m1 ? (const void*)k_gemv_tma<1> : (const void*)k_gemv_tma<8>;
   d.family = "gemv_tma_bf16";
   d.flops = 2.0 * p.M * p.N * p.K;
   d.bytes = 2.0 * ((double)p.N * p.K + (double)p.M * p.K + (double)p.M * p.N);

@@ -436,6 +436,12 @@ static cudaError_t launch_gated(const KernelDesc& d, const GateArgs& g, cudaStre
   return launch_kernel((const void*)k_gated<Op>, dim3(d.grid), dim3(d.block), (size_t)d.smem, st, args);
 }
 
+template <class Op>
+static void use_gated(KernelDesc& d) {
+  d.launch = launch_gated<Op>;
+  d.kernel_fn = (const void*)k_gated<Op>;
+}
+
 static inline size_t esize(int dt) { return dt == BL_BF16 ? 2 : 4; }
 
 // Gemv split-K workspace: one static pool per process (zero-initialised, each
@@ -487,7 +493,8 @@ bool build_simt(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::str
         d.tiles = (uint32_t)(rblocks * ks);
         d.smem = 0;
         std::memcpy(d.params, &q, sizeof(q));
-        d.launch = bf ? launch_gated<Gemv<__nv_bfloat16>> : launch_gated<Gemv<float>>;
+        if (bf) use_gated<Gemv<__nv_bfloat16>>(d);
+        else use_gated<Gemv<float>>(d);
         d.family = bf ? "gemv_bf16" : "gemv_f32";
         d.flops = 2.0 * q.M * q.N * q.K;
         d.bytes = esize(op.dtype) * ((double)q.N * q.K + (double)q.M * q.K + (double)q.M * q.N);
@@ -513,7 +520,8 @@ bool build_simt(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::str
     d.tiles = (uint32_t)(((p.M + kMMB - 1) / kMMB) * p.tiles_n);
     d.smem = 2 * sizeof(float) * kMMB * (kMMB + 1);
     std::memcpy(d.params, &p, sizeof(p));
-    d.launch = bf ? launch_gated<SimtMM<__nv_bfloat16>> : launch_gated<SimtMM<float>>;
+    if (bf) use_gated<SimtMM<__nv_bfloat16>>(d);
+    else use_gated<SimtMM<float>>(d);
     d.family = bf ? "simt_mm_bf16" : "simt_mm_f32";
     d.flops = 2.0 * p.M * p.N * p.K;
     d.bytes = esize(op.dtype) * ((double)p.N * p.K + (double)p.M * p.N * (p.R ? 2 : 1) +
@@ -549,8 +557,10 @@ bool build_simt(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::str
       d.smem = 0;
     }
     std::memcpy(d.params, &p, sizeof(p));
-    if (bf) d.launch = vec ? launch_gated<Pool<__nv_bfloat16, 8>> : launch_gated<Pool<__nv_bfloat16, 1>>;
-    else d.launch = vec ? launch_gated<Pool<float, 4>> : launch_gated<Pool<float, 1>>;
+    if (bf && vec) use_gated<Pool<__nv_bfloat16, 8>>(d);
+    else if (bf) use_gated<Pool<__nv_bfloat16, 1>>(d);
+    else if (vec) use_gated<Pool<float, 4>>(d);
+    else use_gated<Pool<float, 1>>(d);
     d.family = bf ? "pool_bf16" : "pool_f32";
     d.bytes = esize(op.dtype) * ((double)p.Nb * p.H * p.W * p.C + (double)p.Nb * p.OH * p.OW * p.C);
     return true;
@@ -567,7 +577,8 @@ bool build_simt(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::str
     d.tiles = (uint32_t)((p.total + p.per_tile - 1) / p.per_tile);
     d.smem = 0;
     std::memcpy(d.params, &p, sizeof(p));
-    d.launch = bf ? launch_gated<Eltwise<__nv_bfloat16>> : launch_gated<Eltwise<float>>;
+    if (bf) use_gated<Eltwise<__nv_bfloat16>>(d);
+    else use_gated<Eltwise<float>>(d);
     d.family = bf ? "eltwise_bf16" : "eltwise_f32";
     d.bytes = esize(op.dtype) * (double)p.total * (p.R ? 3 : 2);
     return true;

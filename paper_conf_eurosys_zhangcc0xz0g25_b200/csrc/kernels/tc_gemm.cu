@@ -452,8 +452,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
 
 template <int BN, int BK>
 __global__ void __launch_bounds__(192, 1) k_tc_gemm(const __grid_constant__ TcParams p, const GateArgs g) {
-  if (gate_in_range(g)) tc_work<BN, BK>(p, g);
-  else gate_linger(g);
+  if (gate_in_range(g) || gate_linger(g)) tc_work<BN, BK>(p, g);
   pdl_trigger();
   int last = 0;
   const bool fb = gate_leave(g, last);
@@ -483,6 +482,7 @@ static bool prep(KernelDesc& d, std::string& err) {
   }
   d.smem = TcCfg<BN, BK>::kSmem;
   d.launch = launch_tc<BN, BK>;
+  d.kernel_fn = (const void*)k_tc_gemm<BN, BK>;
   return true;
 }
 

@@ -233,6 +233,8 @@ bool DeviceRT::calibrate_clock(std::string& err) {
 int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
   std::unique_ptr<KernelDesc> kd(new KernelDesc());
   if (!build_kernel(op, caps_, *kd, err)) return -1;
+  // grid = S x (resident blocks per SM): see gate_linger in executor.cuh
+  if (kd->kernel_fn) kd->grid = full_occupancy_grid(kd->kernel_fn, kd->block, (size_t)kd->smem, caps_.S);
   kernels_.push_back(std::move(kd));
   return (int)kernels_.size() - 1;
 }
@@ -392,7 +394,7 @@ bool DeviceRT::poll(uint64_t seq, LaunchStats* out) {
     int nsm = 0;
     for (int i = 0; i < 8; ++i) nsm += __builtin_popcount(s->mask[i]);
     out->nsm = nsm;
-    out->fallback = (int)(s->flags & 1u);
+    out->fallback = (int)(s->flags & 3u);  // bit0: last-CTA fallback, bit1: lingering CTAs helped
     for (int i = 0; i < 8; ++i) out->mask[i] = s->mask[i];
   }
   return true;

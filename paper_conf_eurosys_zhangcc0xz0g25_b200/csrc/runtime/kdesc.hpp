@@ -26,6 +26,7 @@ struct KernelDesc {
   double flops = 0;        // algorithmic FLOPs per launch (roofline)
   double bytes = 0;        // algorithmic HBM bytes per launch (roofline)
   LaunchFn launch = nullptr;
+  const void* kernel_fn = nullptr;  // for the occupancy query (grid = S x blocks/SM)
   alignas(128) unsigned char params[4096];  // family-specific parameter block
 };
 

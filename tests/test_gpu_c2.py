@@ -54,11 +54,15 @@ def _mask_bits(r):
     return [w * 32 + b for w in range(8) for b in range(32) if r.sm_mask[w] >> b & 1]
 
 
-@pytest.mark.parametrize("policy", ["STATIC", "UNBOUND", "BLESS"])
+@pytest.mark.parametrize("policy", ["STATIC", "UNBOUND", "BLESS", "ISO_burst"])
 def test_c2_requests_confined_no_fallback(policy, tmp_path):
+    """ISO_burst: 8 requests of each tenant submitted at once, so whole
+    requests queue back to back on each tenant's stream (programmatic
+    dependent launch keeps the next kernel's CTAs waiting while the quota
+    window is still busy) -- the placement-starvation case."""
     from paper_conf_eurosys_zhangcc0xz0g25_b200 import build
     build.build(verbose=False)
-    ctx = capi.Ctx(0, policy=policy)
+    ctx = capi.Ctx(0, policy="ISO" if policy == "ISO_burst" else policy)
     S = ctx.device_info().sm_count
     ms = models.build_config(ctx, "C2", "bf16")
     if policy == "BLESS":
@@ -68,7 +72,8 @@ def test_c2_requests_confined_no_fallback(policy, tmp_path):
         _flat_profile(ctx, ms, S)
     ctx.start()
     base = capi.now_ns() + 1_000_000
-    ids = [ctx.submit(j, base + i * 400_000) for i in range(8) for j in range(2)]
+    gap = 0 if policy == "ISO_burst" else 400_000
+    ids = [ctx.submit(j, base + i * gap) for i in range(8) for j in range(2)]
     ctx.drain(int(60e9))
     ctx.stop()
     lat = []
