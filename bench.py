@@ -213,7 +213,7 @@ def native(args):
 
     from paper_conf_eurosys_zhangcc0xz0g25_b200 import build as bld
     bld.build(verbose=False)
-    from paper_conf_eurosys_zhangcc0xz0g25_b200 import capi, models
+    from paper_conf_eurosys_zhangcc0xz0g25_b200 import capi, models, replicas
 
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
@@ -223,6 +223,8 @@ def native(args):
     if world > 1:
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    plan = replicas.plan(rank, world, local, args.config, sorted(models.CONFIGS))
+    args.config = plan.config
 
     dtype = "fp32" if args.config == "C1" else "bf16"
     params = capi.default_params(squad_max=args.squad_max)
@@ -248,7 +250,8 @@ def native(args):
 
     def step(seed, pol="BLESS", filt=None, extra=None):
         p = capi.default_params(squad_max=args.squad_max, policy=pol, **(extra or {}))
-        return run_policy(ctx, capi, p, make_trace(T_iso, args.rho, args.requests, seed), filt)
+        return run_policy(ctx, capi, p, make_trace(T_iso, args.rho, args.requests, seed + plan.trace_seed_offset),
+                          filt)
 
     for w in range(args.warmup):
         flush.zero_()
@@ -273,14 +276,14 @@ def native(args):
             timelines.append((decisions, launches))
         torch.cuda.synchronize()
         t1 = time.perf_counter()
-    step_ms = (t1 - t0) * 1e3 / args.steps
+    step_ms = replicas.max_over_ranks((t1 - t0) * 1e3 / args.steps, dist, device="cuda")
     if dist:
-        tt = torch.tensor([step_ms], device="cuda")
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        step_ms = float(tt.item())
         dist.barrier()
-    n_req = sum(len(v) for v in lat_all.values())
-    mean_ms = float(np.mean([x for v in lat_all.values() for x in v])) / 1e6
+    n_local = sum(len(v) for v in lat_all.values())
+    agg = replicas.sum_over_ranks({"n": n_local, "lat_sum": float(sum(x for v in lat_all.values() for x in v))},
+                                  dist, device="cuda")
+    n_req = int(agg["n"])                          # whole job (all ranks)
+    mean_ms = agg["lat_sum"] / max(1.0, agg["n"]) / 1e6
     if args.light:
         if rank == 0:
             print(json.dumps({"metric": METRIC, "value": mean_ms, "unit": "ms", "light": True,
@@ -385,7 +388,7 @@ def native(args):
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         from oracle.sched_ref import Prof
         prof = Prof(synprof.load(prof_path))
-        sq = len(decisions_all) / max(1, n_req)
+        sq = len(decisions_all) / max(1, n_local)
         cpu = oracle_timing(names, decisions_all, prof, [len(lat_all[j]) for j in range(len(tms))], sq * 2)
 
     # decisions replayed bit-exactly through the oracle (sample)
