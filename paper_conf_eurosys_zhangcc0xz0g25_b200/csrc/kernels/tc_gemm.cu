@@ -156,18 +156,13 @@ __device__ __forceinline__ float act_f(float y, int act) {
 
 // Fused epilogue for 16 consecutive columns of one output row:
 // y = act(acc * scale + shift + R), rounded to bf16 (RNE), vector stores.
-__device__ __forceinline__ void epi_store16(const TcParams& p, int m, int n0, float (&y)[16]) {
+// sc/sh: the tile's per-column scale/shift staged in shared memory (1 / 0
+// where absent), indexed from this 16-column chunk.
+__device__ __forceinline__ void epi_store16(const TcParams& p, int m, int n0, float (&y)[16], const float* sc,
+                                            const float* sh) {
   const bool full16 = n0 + 16 <= p.N;
-  if (p.scale) {
 #pragma unroll
-    for (int i = 0; i < 16; ++i)
-      if (full16 || n0 + i < p.N) y[i] *= __ldg(p.scale + n0 + i);
-  }
-  if (p.shift) {
-#pragma unroll
-    for (int i = 0; i < 16; ++i)
-      if (full16 || n0 + i < p.N) y[i] += __ldg(p.shift + n0 + i);
-  }
+  for (int i = 0; i < 16; ++i) y[i] = fmaf(y[i], sc[i], sh[i]);
   if (p.R) {
     const __nv_bfloat16* rr = p.R + (size_t)m * p.ldr + n0;
     if (full16 && ((p.ldr & 7) == 0)) {
@@ -206,7 +201,7 @@ struct TcCfg {
   static constexpr int kStageBytes = kStageA + kStageB;
   static constexpr int kStages = std::min(6, (96 * 1024) / kStageBytes);
   static constexpr int kTmemCols = (2 * BN) < 32 ? 32 : 2 * BN;
-  static constexpr int kSmem = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/;
+  static constexpr int kSmem = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/ + 2 * BN * 4 /*sc, sh*/;
 };
 
 template <int BN, int BK>
@@ -227,6 +222,8 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   int* ring = (int*)(rempty + 2);   // [2]
   uint32_t* tmem_slot = (uint32_t*)(ring + 2);
   volatile int* last_flag = (volatile int*)(tmem_slot + 1);
+  float* epi_sc = (float*)(smem + ST * Cfg::kStageBytes + 256);  // [BN] tile scale
+  float* epi_sh = epi_sc + BN;                                    // [BN] tile shift
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
@@ -252,7 +249,10 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
-  pdl_wait();  // setup above overlapped the previous kernel; data reads start below
+  // No grid-wide griddepcontrol.wait here: under programmatic dependent launch
+  // the setup above, the first tile claim, the weight (B) loads and the
+  // epilogue constants overlap the previous kernel; only reads of activations
+  // (A operand, residual) and writes of the output wait for it.
 
   if (warp == 0) {
     // ---------------- tile scheduler + TMA producer
@@ -260,6 +260,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       asm volatile("prefetch.tensormap [%0];" ::"l"(&p.tmA) : "memory");
       asm volatile("prefetch.tensormap [%0];" ::"l"(&p.tmB) : "memory");
       bool marked = false;
+      bool dep_waited = false;
       int stage = 0;
       uint32_t phase = 0;
       int rs = 0;
@@ -283,27 +284,55 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           oh0 = th * p.BH;
           ow0 = (tm - th * p.tiles_w) * p.BW;
         }
-        for (int kb = kb0; kb < kb1; ++kb) {
-          mbar_wait(&empty[stage], phase ^ 1);
-          mbar_expect_tx(&full[stage], Cfg::kStageBytes);
-          unsigned char* a = sA + stage * Cfg::kStageA;
-          unsigned char* b = sB + stage * Cfg::kStageB;
+        auto load_B = [&](int kb, int st) {
+          unsigned char* b = sB + st * Cfg::kStageB;
           if (p.mode == 0) {
-            tma_load_2d(a, &p.tmA, &full[stage], kb * BK, tm * 128);
-            tma_load_2d(b, &p.tmB, &full[stage], kb * BK, tn * BN);
+            tma_load_2d(b, &p.tmB, &full[st], kb * BK, tn * BN);
+          } else {
+            const int tap = kb / p.kc_per_tap, c0 = (kb - tap * p.kc_per_tap) * BK;
+            tma_load_2d(b, &p.tmB, &full[st], tap * p.C + c0, tn * BN);
+          }
+        };
+        auto load_A = [&](int kb, int st) {
+          unsigned char* a = sA + st * Cfg::kStageA;
+          if (p.mode == 0) {
+            tma_load_2d(a, &p.tmA, &full[st], kb * BK, tm * 128);
           } else {
             const int tap = kb / p.kc_per_tap, c0 = (kb - tap * p.kc_per_tap) * BK;
             const int r = tap / p.S_, s = tap - r * p.S_;
             if (p.mode == 1) {
-              tma_load_4d(a, &p.tmA, &full[stage], c0, ow0 - p.pad + s, oh0 - p.pad + r, 0);
+              tma_load_4d(a, &p.tmA, &full[st], c0, ow0 - p.pad + s, oh0 - p.pad + r, 0);
             } else {
               const int dr = r - p.pad, ds = s - p.pad;
               const int ph = dr & 1, pw = ds & 1;        // parity of the input row/col
               const int qh = (dr - ph) / 2, qw = (ds - pw) / 2;
-              tma_load_5d(a, &p.tmA, &full[stage], c0, pw, ow0 + qw, ph, oh0 + qh);
+              tma_load_5d(a, &p.tmA, &full[st], c0, pw, ow0 + qw, ph, oh0 + qh);
             }
-            tma_load_2d(b, &p.tmB, &full[stage], tap * p.C + c0, tn * BN);
           }
+        };
+        int kb = kb0;
+        if (!dep_waited) {
+          // first tile: weights for up to ST stages before the grid dependency
+          // resolves, activations after it
+          const int npre = min(kb1 - kb0, ST);
+          for (int i = 0; i < npre; ++i) {
+            const int st = (stage + i) % ST;
+            mbar_wait(&empty[st], (phase ^ (stage + i >= ST ? 1 : 0)) ^ 1);
+            mbar_expect_tx(&full[st], Cfg::kStageBytes);
+            load_B(kb0 + i, st);
+          }
+          pdl_wait();
+          dep_waited = true;
+          for (int i = 0; i < npre; ++i) load_A(kb0 + i, (stage + i) % ST);
+          for (int i = 0; i < npre; ++i)
+            if (++stage == ST) { stage = 0; phase ^= 1; }
+          kb = kb0 + npre;
+        }
+        for (; kb < kb1; ++kb) {
+          mbar_wait(&empty[stage], phase ^ 1);
+          mbar_expect_tx(&full[stage], Cfg::kStageBytes);
+          load_B(kb, stage);
+          load_A(kb, stage);
           if (++stage == ST) { stage = 0; phase ^= 1; }
         }
       }
@@ -352,6 +381,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   } else {
     // ---------------- epilogue warps 2..5 (TMEM lane quarter = warp % 4)
     const int q = warp & 3;
+    bool dep_waited = false;
     int rs = 0;
     uint32_t rph = 0;
     int acc = 0;
@@ -377,6 +407,22 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         valid = oh < p.OH && ow < p.OW;
         m = oh * p.OW + ow;
       }
+      // stage this tile's scale/shift (independent of the previous kernel)
+      asm volatile("bar.sync 2, 128;" ::: "memory");   // previous tile's readers are done
+      for (int i = threadIdx.x - 64; i < BN; i += 128) {
+        const int n = tn * BN + i;
+        epi_sc[i] = (p.scale && n < p.N) ? __ldg(p.scale + n) : 1.f;
+        epi_sh[i] = (p.shift && n < p.N) ? __ldg(p.shift + n) : 0.f;
+      }
+      asm volatile("bar.sync 2, 128;" ::: "memory");
+      if (!dep_waited) {   // residual reads / output writes depend on earlier kernels
+        pdl_wait();
+        dep_waited = true;
+      }
+      if (p.R && valid) {  // pull this row's residual segment into L2 while the MMAs run
+        const char* rr = reinterpret_cast<const char*>(p.R + (size_t)m * p.ldr + tn * BN);
+        for (int b = 0; b < BN * 2; b += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(rr + b));
+      }
       mbar_wait(&tfull[acc], aph);
       tc_fence_after();
       const uint32_t tbase = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN;
@@ -391,7 +437,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           float y[16];
 #pragma unroll
           for (int i = 0; i < 16; ++i) y[i] = __uint_as_float(v[i]);
-          epi_store16(p, m, n0, y);
+          epi_store16(p, m, n0, y, epi_sc + c, epi_sh + c);
         }
         tc_fence_before();
         __syncwarp();
@@ -432,7 +478,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
                 y[i] = f.x; y[i + 1] = f.y; y[i + 2] = f.z; y[i + 3] = f.w;
                 __stcg(reinterpret_cast<float4*>(wrow + c + i), make_float4(0.f, 0.f, 0.f, 0.f));
               }
-              epi_store16(p, m, n0, y);
+              epi_store16(p, m, n0, y, epi_sc + c, epi_sh + c);
             }
           }
           if (threadIdx.x == 64) p.sem[tile] = 0;
