@@ -108,6 +108,7 @@ typedef enum {
   BL_OP_CONV = 1,    /* NHWC conv, KRSC weights, same epilogue                        */
   BL_OP_POOL = 2,    /* max / avg / global-avg pooling, NHWC                          */
   BL_OP_ELTWISE = 3, /* Y = act(X * scale + shift (+ R)), per-channel, any layout      */
+  BL_OP_IM2COL = 4,  /* Y[m, k] = im2col of an NHWC input, zero-padded to Kpad columns */
   BL_OP_VIRTUAL = 15 /* no device work (BL_DEVICE_NONE contexts / profile-only)       */
 } bl_op_kind;
 
@@ -127,6 +128,10 @@ typedef enum { BL_POOL_MAX = 0, BL_POOL_AVG = 1, BL_POOL_GLOBAL_AVG = 2 } bl_poo
  *  POOL  dims = {Nb, H, W, C, k, stride, pad, mode(bl_pool_mode)}
  *        ptr  = {X, Y}
  *  ELTWISE dims = {rows, C}  ptr = {X, scale, shift, R, Y}
+ *  IM2COL dims = {Nb, H, W, C, R, S, stride, pad, Kpad}  ptr = {X, Y}
+ *        Y[(n*OH + oh)*OW + ow, (r*S + s)*C + c] = X[n, oh*stride - pad + r,
+ *        ow*stride - pad + s, c] (0 outside the image and for k >= R*S*C);
+ *        used for first layers with C < 16 so the conv runs as a tensor-core GEMM
  */
 typedef struct {
   int32_t kind;     /* bl_op_kind */

@@ -260,6 +260,60 @@ struct Pool {
 };
 
 // ---------------------------------------------------------------------------
+// Im2col: Y[m, k] (row-major, Kpad columns) for a conv with few input channels,
+// so that the conv itself runs as a tensor-core GEMM (first layers, C = 3).
+// One thread per output element; consecutive threads write consecutive k.
+// ---------------------------------------------------------------------------
+struct Im2colParams {
+  const void* X;
+  void* Y;
+  int H, W, C, R, S, stride, pad, Kpad, OH, OW;
+  long long total;
+  int per_tile;
+};
+
+template <typename T>
+struct Im2col {
+  using Params = Im2colParams;
+  static constexpr int V = 16 / sizeof(T);   // one 16-byte output vector per thread
+  __device__ static void tile(const Params& p, int t, unsigned char*) {
+    const T* X = (const T*)p.X;
+    T* Y = (T*)p.Y;
+    const int K = p.R * p.S * p.C;
+    const int KV = p.Kpad / V;                 // vectors per output row
+    const int nvec = (int)(p.total / V);
+    const int v0 = t * p.per_tile, v1 = min(v0 + p.per_tile, nvec);
+    const int hw = p.OH * p.OW;
+    for (int vi = v0 + (int)threadIdx.x; vi < v1; vi += blockDim.x) {
+      const int m = vi / KV;
+      const int k0 = (vi - m * KV) * V;
+      const int n = m / hw, q = m - n * hw;
+      const int oh = q / p.OW, ow = q - oh * p.OW;
+      const int h0 = oh * p.stride - p.pad, w0 = ow * p.stride - p.pad;
+      // (r, s, c) of k0, then stepped incrementally
+      int r = k0 / (p.S * p.C);
+      int rem = k0 - r * p.S * p.C;
+      int s = rem / p.C, c = rem - s * p.C;
+      float f[V];
+#pragma unroll
+      for (int j = 0; j < V; ++j) {
+        float v = 0.f;
+        if (k0 + j < K) {
+          const int ih = h0 + r, iw = w0 + s;
+          if (ih >= 0 && ih < p.H && iw >= 0 && iw < p.W) v = ldf(X + ((size_t)(n * p.H + ih) * p.W + iw) * p.C + c);
+        }
+        f[j] = v;
+        if (++c == p.C) {
+          c = 0;
+          if (++s == p.S) { s = 0; ++r; }
+        }
+      }
+      store_vec<T, V>(Y + (size_t)vi * V, f);
+    }
+  }
+};
+
+// ---------------------------------------------------------------------------
 // Eltwise: Y[r, c] = act(X*scale[c] + shift[c] + R)
 // ---------------------------------------------------------------------------
 struct EltParams {
@@ -563,6 +617,35 @@ bool build_simt(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::str
     else use_gated<Pool<float, 1>>(d);
     d.family = bf ? "pool_bf16" : "pool_f32";
     d.bytes = esize(op.dtype) * ((double)p.Nb * p.H * p.W * p.C + (double)p.Nb * p.OH * p.OW * p.C);
+    return true;
+  }
+  if (op.kind == BL_OP_IM2COL) {
+    Im2colParams p{};
+    p.X = op.ptr[0];
+    p.Y = op.ptr[1];
+    const int Nb = (int)op.dims[0];
+    p.H = (int)op.dims[1]; p.W = (int)op.dims[2]; p.C = (int)op.dims[3];
+    p.R = (int)op.dims[4]; p.S = (int)op.dims[5]; p.stride = (int)op.dims[6]; p.pad = (int)op.dims[7];
+    p.Kpad = (int)op.dims[8];
+    if (Nb < 1 || p.C < 1 || p.R < 1 || p.S < 1 || p.stride < 1 || p.Kpad < p.R * p.S * p.C) {
+      err = "im2col dims";
+      return false;
+    }
+    p.OH = (p.H + 2 * p.pad - p.R) / p.stride + 1;
+    p.OW = (p.W + 2 * p.pad - p.S) / p.stride + 1;
+    p.total = (long long)Nb * p.OH * p.OW * p.Kpad;
+    const int V = bf ? 8 : 4;
+    if (p.Kpad % V || (((uintptr_t)p.Y) & 15) || p.total / V >= (1LL << 31)) { err = "im2col: Kpad/alignment"; return false; }
+    const long long nvec = p.total / V;
+    long long per = (nvec + 4LL * caps.S - 1) / (4LL * caps.S);   // ~4 tiles per SM
+    p.per_tile = (int)std::max<long long>(256, (per + 255) / 256 * 256);
+    d.tiles = (uint32_t)((nvec + p.per_tile - 1) / p.per_tile);
+    d.smem = 0;
+    std::memcpy(d.params, &p, sizeof(p));
+    if (bf) use_gated<Im2col<__nv_bfloat16>>(d);
+    else use_gated<Im2col<float>>(d);
+    d.family = bf ? "im2col_bf16" : "im2col_f32";
+    d.bytes = esize(op.dtype) * ((double)Nb * p.H * p.W * p.C + (double)p.total);
     return true;
   }
   if (op.kind == BL_OP_ELTWISE) {

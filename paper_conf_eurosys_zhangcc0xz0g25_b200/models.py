@@ -102,11 +102,32 @@ class Builder:
              res=None, name=""):
         N, H, W, C = x.shape
         pad = k // 2 if pad is None else pad
-        w = self.param(syn.weight(self.g, (k_out, k, k, C), k * k * C))
+        w_np = syn.weight(self.g, (k_out, k, k, C), k * k * C)
         scale = self.param(syn.bn_scale(self.g, k_out), fp32=True) if bn else None
         shift = self.param(syn.bn_shift(self.g, k_out) if bn else syn.bias(self.g, k_out), fp32=True) \
             if (bn or bias) else None
         OH, OW = (H + 2 * pad - k) // stride + 1, (W + 2 * pad - k) // stride + 1
+        if C < 16 and self.bl_dtype == capi.BL_BF16:
+            # first layers (C = 3): explicit im2col into a zero-padded [M, Kpad]
+            # matrix, then the conv is a tensor-core GEMM
+            K = k * k * C
+            Kpad = (K + 63) // 64 * 64
+            cols = self.act_buf((N * OH * OW, Kpad))
+            op = self._op(capi.BL_OP_IM2COL, "none", [N, H, W, C, k, k, stride, pad, Kpad], [x, cols])
+            self.ctx.append_kernel(self.m.tenant, op)
+            self.m.layers.append(Layer("im2col", x, cols, act="none",
+                                       geom=dict(k=k, stride=stride, pad=pad, Kpad=Kpad), name=name + ".im2col"))
+            wp = np.zeros((k_out, Kpad), np.float32)
+            wp[:, :K] = w_np.reshape(k_out, K)
+            w = self.param(wp)
+            y = self.act_buf((N, OH, OW, k_out))
+            y2 = y.view(N * OH * OW, k_out)
+            r2 = res.view(N * OH * OW, k_out) if res is not None else None
+            op = self._op(capi.BL_OP_GEMM, act, [N * OH * OW, k_out, Kpad, 0, 0, 0, 0], [cols, w, scale, shift, r2, y2])
+            self.ctx.append_kernel(self.m.tenant, op)
+            self.m.layers.append(Layer("gemm", cols, y2, w, scale, shift, r2, act, {}, name))
+            return y
+        w = self.param(w_np)
         y = self.act_buf((N, OH, OW, k_out))
         op = self._op(capi.BL_OP_CONV, act, [N, H, W, C, k_out, k, k, stride, pad, 1, 0, 0],
                       [x, w, scale, shift, res, y])

@@ -24,7 +24,26 @@ def reference(layer):
         return f(x, g["k"], g["stride"], g["pad"])
     if layer.kind == "gap":
         return L.global_avgpool_nhwc(x)
+    if layer.kind == "im2col":
+        g = layer.geom
+        return im2col_ref(x, g["k"], g["stride"], g["pad"], g["Kpad"])
     raise ValueError(layer.kind)
+
+
+def im2col_ref(x, k, stride, pad, kpad):
+    """Plain im2col: row = output pixel (raster order), column = (r*k + s)*C + c,
+    zero padding outside the image and beyond k*k*C."""
+    N, H, W, C = x.shape
+    OH, OW = (H + 2 * pad - k) // stride + 1, (W + 2 * pad - k) // stride + 1
+    xp = np.zeros((N, H + 2 * pad, W + 2 * pad, C))
+    xp[:, pad:pad + H, pad:pad + W, :] = x
+    out = np.zeros((N * OH * OW, kpad))
+    cols = []
+    for r in range(k):
+        for s in range(k):
+            cols.append(xp[:, r:r + stride * (OH - 1) + 1:stride, s:s + stride * (OW - 1) + 1:stride, :])
+    out[:, :k * k * C] = np.concatenate(cols, axis=-1).reshape(N * OH * OW, k * k * C)
+    return out
 
 
 def tolerance(dtype: str) -> float:

@@ -65,6 +65,20 @@ def test_conv_vs_torch(k, stride, pad, groups):
     assert np.allclose(got, np.maximum(ref + res, 0), rtol=1e-12, atol=1e-12)
 
 
+@pytest.mark.parametrize("k,stride,pad", [(3, 1, 1), (7, 2, 3)])
+def test_im2col_ref_times_weights_is_conv(k, stride, pad):
+    """The test-side im2col (tests/layer_check.py) pinned to the conv
+    definition: im2col(x) @ w.reshape(K, -1)^T == conv2d(x, w)."""
+    from tests.layer_check import im2col_ref
+    x = R.standard_normal((1, 11, 9, 3))
+    w = R.standard_normal((5, k, k, 3))
+    cols = im2col_ref(x, k, stride, pad, 3 * k * k + 5)
+    assert np.all(cols[:, 3 * k * k:] == 0)
+    got = cols[:, :3 * k * k] @ w.reshape(5, -1).T
+    ref = L.conv2d_nhwc(x, w, stride=stride, pad=pad).reshape(-1, 5)
+    assert np.allclose(got, ref, rtol=1e-12, atol=1e-12)
+
+
 def test_conv_delta_kernel_is_identity():
     x = R.standard_normal((1, 5, 5, 3))
     w = np.zeros((3, 3, 3, 3))
