@@ -109,6 +109,10 @@ typedef enum {
   BL_OP_POOL = 2,    /* max / avg / global-avg pooling, NHWC                          */
   BL_OP_ELTWISE = 3, /* Y = act(X * scale + shift (+ R)), per-channel, any layout      */
   BL_OP_IM2COL = 4,  /* Y[m, k] = im2col of an NHWC input, zero-padded to Kpad columns */
+  BL_OP_LAYERNORM = 5, /* Y = LN(X (+ R)) * gamma + beta over the last dim (eps = fparam[0]) */
+  BL_OP_ATTENTION = 6, /* per head: O = softmax(Q K^T * scale) V (all-ones mask)          */
+  BL_OP_EMBED = 7,     /* Y = LN(word[ids] + pos[0:L] + type[0]) * gamma + beta            */
+  BL_OP_DWCONV = 8,    /* depthwise NHWC conv (groups = C), weights [C, R, S, 1] + epilogue */
   BL_OP_VIRTUAL = 15 /* no device work (BL_DEVICE_NONE contexts / profile-only)       */
 } bl_op_kind;
 
@@ -125,9 +129,19 @@ typedef enum { BL_POOL_MAX = 0, BL_POOL_AVG = 1, BL_POOL_GLOBAL_AVG = 2 } bl_poo
  *  CONV  dims = {Nb, H, W, C, K, R, S, stride, pad, groups, ldx(0=C), ldy(0=K)}
  *        ptr  = {X, W(KRSC), scale, shift, R(ld = ldy), Y}
  *        (channel slices: offset the pointers, give ld*)
- *  POOL  dims = {Nb, H, W, C, k, stride, pad, mode(bl_pool_mode)}
- *        ptr  = {X, Y}
- *  ELTWISE dims = {rows, C}  ptr = {X, scale, shift, R, Y}
+ *  POOL  dims = {Nb, H, W, C, k, stride, pad, mode(bl_pool_mode), ldy(0=C)}
+ *        ptr  = {X, Y}   (ldy: output channel stride of window pools)
+ *  ELTWISE dims = {rows, C, ldx(0=C), ldy(0=C)}  ptr = {X, scale, shift, R(ld = ldy), Y}
+ *  LAYERNORM dims = {rows, C, ldx(0=C), ldy(0=C)}  ptr = {X, gamma, beta, R(ld = ldx), Y}
+ *        fparam[0] = eps (0 -> 1e-12)
+ *  ATTENTION dims = {L, heads, dh, ld_qkv, ld_o}  ptr = {QKV, O}
+ *        QKV row t = [Q (heads*dh) | K (heads*dh) | V (heads*dh)], head h at
+ *        column h*dh of each block; O[t, h*dh + i]; fparam[0] = scale
+ *        (0 -> 1/sqrt(dh)); L <= 512, dh = 64
+ *  EMBED dims = {L, C, vocab}  ptr = {ids (int32), word [vocab, C], pos [>=L, C],
+ *        type [>=1, C], gamma, beta, Y}  fparam[0] = eps (0 -> 1e-12)
+ *  DWCONV dims = {Nb, H, W, C, R, S, stride, pad}  ptr = {X, W [C,R,S,1], scale,
+ *        shift, R, Y}  (epilogue as CONV)
  *  IM2COL dims = {Nb, H, W, C, R, S, stride, pad, Kpad}  ptr = {X, Y}
  *        Y[(n*OH + oh)*OW + ow, (r*S + s)*C + c] = X[n, oh*stride - pad + r,
  *        ow*stride - pad + s, c] (0 outside the image and for k >= R*S*C);

@@ -28,6 +28,7 @@ POLICIES = {"BLESS": 0, "ISO": 1, "STATIC": 2, "TEMPORAL": 3, "UNBOUND": 4}
 BL_CLOCK_WALL, BL_CLOCK_VIRTUAL = 0, 1
 # ops
 BL_OP_GEMM, BL_OP_CONV, BL_OP_POOL, BL_OP_ELTWISE, BL_OP_IM2COL, BL_OP_VIRTUAL = 0, 1, 2, 3, 4, 15
+BL_OP_LAYERNORM, BL_OP_ATTENTION, BL_OP_EMBED, BL_OP_DWCONV = 5, 6, 7, 8
 BL_F32, BL_BF16 = 0, 1
 BL_ACT_NONE, BL_ACT_RELU, BL_ACT_RELU6, BL_ACT_GELU = 0, 1, 2, 3
 ACTS = {"none": 0, "relu": 1, "relu6": 2, "gelu": 3}

@@ -136,6 +136,7 @@ struct PoolParams {
   void* Y;
   int Nb, H, W, C, OH, OW, k, stride, pad, mode;
   int vec;              // elements per vector access (C % vec == 0)
+  int ldy;              // output channel stride (window pools; DenseNet concat slices)
   long long items;      // output pixels x C/vec (window pools) | Nb x C/vec (global)
   int per_tile;         // items per tile (window pools) | vector groups per tile (global)
 };
@@ -254,7 +255,7 @@ struct Pool {
 #pragma unroll
         for (int i = 0; i < V; ++i) acc[i] /= (float)(p.k * p.k);
       }
-      store_vec<T, V>(Y + (size_t)pix * p.C + (size_t)cv * V, acc);
+      store_vec<T, V>(Y + (size_t)pix * p.ldy + (size_t)cv * V, acc);
     }
   }
 };
@@ -588,9 +589,10 @@ bool build_simt(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::str
     p.X = op.ptr[0]; p.Y = op.ptr[1];
     p.Nb = (int)op.dims[0]; p.H = (int)op.dims[1]; p.W = (int)op.dims[2]; p.C = (int)op.dims[3];
     p.k = (int)op.dims[4]; p.stride = (int)op.dims[5]; p.pad = (int)op.dims[6]; p.mode = (int)op.dims[7];
+    p.ldy = op.dims[8] ? (int)op.dims[8] : p.C;
     if (p.C < 1 || p.Nb < 1) { err = "pool dims"; return false; }
     const int V = bf ? 8 : 4;
-    const bool vec = (p.C % V) == 0 && (((uintptr_t)p.X | (uintptr_t)p.Y) & 15) == 0;
+    const bool vec = (p.C % V) == 0 && (p.ldy % V) == 0 && (((uintptr_t)p.X | (uintptr_t)p.Y) & 15) == 0;
     p.vec = vec ? V : 1;
     const int CV = p.C / p.vec;
     if (p.mode == BL_POOL_GLOBAL_AVG) {

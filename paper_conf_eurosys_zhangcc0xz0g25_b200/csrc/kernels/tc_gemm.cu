@@ -602,11 +602,14 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     const int ldx = op.dims[10] ? (int)op.dims[10] : C;
     p.ldy = op.dims[11] ? (int)op.dims[11] : K;
     p.ldr = p.ldy;
-    if (Nb != 1 || groups != 1 || C % 16 || ldx % 8 || K % 16 || p.ldy % 8) return false;
+    const bool one_by_one = R == 1 && S == 1 && stride == 1 && pad == 0;
+    if (Nb != 1 || groups != 1 || C % 8 || ldx % 8 || K % 8 || p.ldy % 8) return false;
+    if (!one_by_one && C % 16) return false;
     if (stride != 1 && stride != 2) return false;
     if (stride == 2 && ((H | Wd) & 1)) return false;
     if (((uintptr_t)X | (uintptr_t)W) & 15) return false;
-    BK = (C % 64 == 0) ? 64 : (C % 32 == 0 ? 32 : 16);
+    // 1x1 stride-1 convs are plain GEMMs over pixels: any C % 8, K tail zero-filled by TMA
+    BK = one_by_one ? 64 : ((C % 64 == 0) ? 64 : (C % 32 == 0 ? 32 : 16));
     p.OH = (H + 2 * pad - R) / stride + 1;
     p.OW = (Wd + 2 * pad - S) / stride + 1;
     p.M = p.OH * p.OW;
@@ -616,7 +619,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     p.R_ = R;
     p.S_ = S;
     p.pad = pad;
-    p.kc_per_tap = C / BK;
+    p.kc_per_tap = one_by_one ? (C + BK - 1) / BK : C / BK;
     p.num_kb = R * S * p.kc_per_tap;
     // M tile = BH x BW output pixels (BH*BW = 128), BW the smallest power of two >= OW (<= 128)
     int BW = 1;
@@ -626,7 +629,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     p.BH = 128 / BW;
     p.tiles_w = (p.OW + BW - 1) / BW;
     const int tiles_h = (p.OH + p.BH - 1) / p.BH;
-    if (R == 1 && S == 1 && stride == 1 && pad == 0 && ldx == C) {
+    if (one_by_one) {
       // 1x1 stride-1: plain GEMM over pixels
       p.mode = 0;
       cuuint64_t da[2] = {(cuuint64_t)C, (cuuint64_t)(H * Wd)}, sa[1] = {(cuuint64_t)ldx * 2};

@@ -43,5 +43,6 @@ bool build_kernel(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std:
 bool build_simt(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
 bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
 bool build_gemv_tma(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
+bool build_nn(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
 
 }  // namespace bless

@@ -99,7 +99,8 @@ class Builder:
         return y
 
     def conv(self, x: torch.Tensor, k_out: int, k: int, stride=1, pad=None, act="relu", bn=True, bias=False,
-             res=None, name=""):
+             res=None, name="", out=None):
+        """out: optional NHWC view of a wider buffer (DenseNet concat slice) to write into."""
         N, H, W, C = x.shape
         pad = k // 2 if pad is None else pad
         w_np = syn.weight(self.g, (k_out, k, k, C), k * k * C)
@@ -128,27 +129,99 @@ class Builder:
             self.m.layers.append(Layer("gemm", cols, y2, w, scale, shift, r2, act, {}, name))
             return y
         w = self.param(w_np)
-        y = self.act_buf((N, OH, OW, k_out))
-        op = self._op(capi.BL_OP_CONV, act, [N, H, W, C, k_out, k, k, stride, pad, 1, 0, 0],
+        ldy = 0
+        if out is not None:
+            y, ldy = out, out.stride(2)
+        else:
+            y = self.act_buf((N, OH, OW, k_out))
+        ldx = x.stride(2) if x.stride(2) != C else 0
+        op = self._op(capi.BL_OP_CONV, act, [N, H, W, C, k_out, k, k, stride, pad, 1, ldx, ldy],
                       [x, w, scale, shift, res, y])
         self.ctx.append_kernel(self.m.tenant, op)
         self.m.layers.append(Layer("conv", x, y, w, scale, shift, res, act,
                                    dict(stride=stride, pad=pad, groups=1), name))
         return y
 
-    def pool(self, x, k, stride, pad=0, mode="max", name=""):
+    def pool(self, x, k, stride, pad=0, mode="max", name="", out=None):
+        """out: optional NHWC view of a wider buffer (channel slice) to write into."""
         N, H, W, C = x.shape
+        ldy = 0
         if mode == "gap":
             y = self.act_buf((N, C))
             md = capi.BL_POOL_GLOBAL_AVG
         else:
             OH, OW = (H + 2 * pad - k) // stride + 1, (W + 2 * pad - k) // stride + 1
-            y = self.act_buf((N, OH, OW, C))
+            if out is not None:
+                y, ldy = out, out.stride(2)
+            else:
+                y = self.act_buf((N, OH, OW, C))
             md = capi.BL_POOL_MAX if mode == "max" else capi.BL_POOL_AVG
-        op = self._op(capi.BL_OP_POOL, "none", [N, H, W, C, k, stride, pad, md], [x, y])
+        op = self._op(capi.BL_OP_POOL, "none", [N, H, W, C, k, stride, pad, md, ldy], [x, y])
         self.ctx.append_kernel(self.m.tenant, op)
         self.m.layers.append(Layer("gap" if mode == "gap" else "pool", x, y, act="none",
                                    geom=dict(k=k, stride=stride, pad=pad, mode=mode), name=name))
+        return y
+
+    def dwconv(self, x, k, stride, act="relu6", name=""):
+        """Depthwise k x k conv + folded BN + act (MobileNetV2), weights [C, k, k, 1]."""
+        N, H, W, C = x.shape
+        pad = k // 2
+        w = self.param(syn.weight(self.g, (C, k, k, 1), k * k))
+        scale = self.param(syn.bn_scale(self.g, C), fp32=True)
+        shift = self.param(syn.bn_shift(self.g, C), fp32=True)
+        OH, OW = (H + 2 * pad - k) // stride + 1, (W + 2 * pad - k) // stride + 1
+        y = self.act_buf((N, OH, OW, C))
+        op = self._op(capi.BL_OP_DWCONV, act, [N, H, W, C, k, k, stride, pad], [x, w, scale, shift, None, y])
+        self.ctx.append_kernel(self.m.tenant, op)
+        self.m.layers.append(Layer("conv", x, y, w, scale, shift, None, act,
+                                   dict(stride=stride, pad=pad, groups=C), name))
+        return y
+
+    def bn_act(self, x2d, act="relu", out=None, name=""):
+        """Per-channel folded BN + act on a [rows, C] (possibly strided) view."""
+        rows, C = x2d.shape
+        scale = self.param(syn.bn_scale(self.g, C), fp32=True)
+        shift = self.param(syn.bn_shift(self.g, C), fp32=True)
+        y = out if out is not None else self.act_buf((rows, C))
+        op = self._op(capi.BL_OP_ELTWISE, act, [rows, C, x2d.stride(0), y.stride(0)], [x2d, scale, shift, None, y])
+        self.ctx.append_kernel(self.m.tenant, op)
+        self.m.layers.append(Layer("eltwise", x2d, y, None, scale, shift, None, act, {}, name))
+        return y
+
+    def layernorm(self, x, res=None, name=""):
+        rows, C = x.shape
+        gamma = self.param(syn.bn_scale(self.g, C), fp32=True)
+        beta = self.param(syn.bn_shift(self.g, C), fp32=True)
+        y = self.act_buf((rows, C))
+        op = self._op(capi.BL_OP_LAYERNORM, "none", [rows, C, 0, 0], [x, gamma, beta, res, y])
+        op.fparam[0] = 1e-12
+        self.ctx.append_kernel(self.m.tenant, op)
+        self.m.layers.append(Layer("layernorm", x, y, None, gamma, beta, res, "none", dict(eps=1e-12), name))
+        return y
+
+    def attention(self, qkv, heads, dh, name=""):
+        L = qkv.shape[0]
+        o = self.act_buf((L, heads * dh))
+        op = self._op(capi.BL_OP_ATTENTION, "none", [L, heads, dh, 0, 0], [qkv, o])
+        self.ctx.append_kernel(self.m.tenant, op)
+        self.m.layers.append(Layer("attention", qkv, o, act="none", geom=dict(heads=heads, dh=dh), name=name))
+        return o
+
+    def embedding(self, L, C, vocab=30522, max_pos=512, name="embed"):
+        ids = torch.from_numpy(syn.token_ids(self.g, L)).to(self.dev)
+        self.m.keep.append(ids)
+        self.m.input = ids
+        word = self.param(0.02 * syn.activation(self.g, (vocab, C)))
+        pos = self.param(0.02 * syn.activation(self.g, (max_pos, C)))
+        typ = self.param(0.02 * syn.activation(self.g, (2, C)))
+        gamma = self.param(syn.bn_scale(self.g, C), fp32=True)
+        beta = self.param(syn.bn_shift(self.g, C), fp32=True)
+        y = self.act_buf((L, C))
+        op = self._op(capi.BL_OP_EMBED, "none", [L, C, vocab], [ids, word, pos, typ, gamma, beta, y])
+        op.fparam[0] = 1e-12
+        self.ctx.append_kernel(self.m.tenant, op)
+        self.m.layers.append(Layer("embed", ids, y, word, gamma, beta, None, "none",
+                                   dict(pos=pos, typ=typ, eps=1e-12), name))
         return y
 
     def done(self, y) -> TenantModel:
@@ -225,17 +298,132 @@ def resnet(ctx, tenant, quota, depth=50, dtype="bf16", seed=1000) -> TenantModel
     return b.done(x)
 
 
+VGG_CFG = {
+    "vgg11": [64, "M", 128, "M", 256, 256, "M", 512, 512, "M", 512, 512, "M"],
+    "vgg16": [64, 64, "M", 128, 128, "M", 256, 256, 256, "M", 512, 512, 512, "M", 512, 512, 512, "M"],
+}
+
+
+def vgg(ctx, tenant, quota, name="vgg16", dtype="bf16", seed=1000) -> TenantModel:
+    """torchvision VGG (cfg A = vgg11, D = vgg16), as vgg11() above."""
+    b = Builder(ctx, tenant, name, quota, dtype, seed)
+    x = b.input((1, 224, 224, 3))
+    i = 0
+    for v in VGG_CFG[name]:
+        if v == "M":
+            x = b.pool(x, 2, 2, 0, "max", name=f"pool{i}")
+        else:
+            x = b.conv(x, v, 3, 1, 1, act="relu", bn=False, bias=True, name=f"conv{i}")
+            i += 1
+    x = x.view(1, -1)
+    x = b.gemm(x, 4096, act="relu", name="fc1")
+    x = b.gemm(x, 4096, act="relu", name="fc2")
+    x = b.gemm(x, 1000, act="none", name="fc3")
+    return b.done(x)
+
+
+def mobilenet_v2(ctx, tenant, quota, dtype="bf16", seed=1000) -> TenantModel:
+    """torchvision MobileNetV2 (width 1.0), batch 1, 224x224: ReLU6 everywhere
+    except the linear bottleneck projections; residual when stride 1 and
+    in == out channels."""
+    b = Builder(ctx, tenant, "mobilenet_v2", quota, dtype, seed)
+    x = b.input((1, 224, 224, 3))
+    x = b.conv(x, 32, 3, 2, 1, act="relu6", name="stem")
+    cin = 32
+    settings = [(1, 16, 1, 1), (6, 24, 2, 2), (6, 32, 3, 2), (6, 64, 4, 2), (6, 96, 3, 1), (6, 160, 3, 2),
+                (6, 320, 1, 1)]
+    bi = 0
+    for t, c, n, s in settings:
+        for i in range(n):
+            stride = s if i == 0 else 1
+            h = x
+            if t != 1:
+                h = b.conv(h, cin * t, 1, 1, 0, act="relu6", name=f"b{bi}.expand")
+            h = b.dwconv(h, 3, stride, act="relu6", name=f"b{bi}.dw")
+            res = x if (stride == 1 and cin == c) else None
+            x = b.conv(h, c, 1, 1, 0, act="none", res=res, name=f"b{bi}.project")
+            cin = c
+            bi += 1
+    x = b.conv(x, 1280, 1, 1, 0, act="relu6", name="head")
+    x = b.pool(x, 0, 1, 0, "gap", name="avgpool")
+    x = b.gemm(x, 1000, act="none", name="classifier")
+    return b.done(x)
+
+
+def bert(ctx, tenant, quota, size="base", seq=128, dtype="bf16", seed=1000) -> TenantModel:
+    """HF BertModel encoder (post-LN), batch 1, all-ones mask, erf-GELU,
+    LayerNorm eps 1e-12; 7 kernels per layer:
+    QKV GEMM, attention, output GEMM (+ residual), LN, FFN1 (GELU), FFN2
+    (+ residual), LN; plus the embedding (gather + add + LN)."""
+    layers, C, H = {"base": (12, 768, 12), "large": (24, 1024, 16)}[size]
+    b = Builder(ctx, tenant, f"bert_{size}", quota, dtype, seed)
+    x = b.embedding(seq, C)
+    for li in range(layers):
+        qkv = b.gemm(x, 3 * C, act="none", bias=True, name=f"l{li}.qkv")
+        ctx_ = b.attention(qkv, H, C // H, name=f"l{li}.attn")
+        a = b.gemm(ctx_, C, act="none", bias=True, res=x, name=f"l{li}.out")
+        h1 = b.layernorm(a, name=f"l{li}.ln1")
+        f = b.gemm(h1, 4 * C, act="gelu", bias=True, name=f"l{li}.ffn1")
+        o = b.gemm(f, C, act="none", bias=True, res=h1, name=f"l{li}.ffn2")
+        x = b.layernorm(o, name=f"l{li}.ln2")
+    return b.done(x)
+
+
+def densenet121(ctx, tenant, quota, dtype="bf16", seed=1000) -> TenantModel:
+    """torchvision DenseNet-121 (growth 32, bn_size 4, blocks 6/12/24/16),
+    batch 1, 224x224.  Each block owns one NHWC concat buffer; a dense layer is
+    BN-ReLU on the first C_i channels (strided eltwise) -> 1x1 conv with BN-ReLU
+    epilogue -> 3x3 conv writing its 32 channels into the buffer slice
+    (SURVEY.md §8(c) C-4)."""
+    b = Builder(ctx, tenant, "densenet121", quota, dtype, seed)
+    x = b.input((1, 224, 224, 3))
+    x = b.conv(x, 64, 7, 2, 3, act="relu", name="conv0")
+    c = 64
+    hw = 56
+    blocks = [6, 12, 24, 16]
+    buf = b.act_buf((1, hw, hw, c + blocks[0] * 32))
+    b.pool(x, 3, 2, 1, "max", name="pool0", out=buf[..., :c])
+    for bi, nl in enumerate(blocks):
+        for li in range(nl):
+            xin = buf.view(hw * hw, -1)[:, :c]          # first c channels of the concat buffer
+            t = b.bn_act(xin, "relu", name=f"b{bi}l{li}.norm1")
+            t = t.view(1, hw, hw, c)
+            h = b.conv(t, 128, 1, 1, 0, act="relu", bn=True, name=f"b{bi}l{li}.conv1")   # + norm2 + relu2
+            b.conv(h, 32, 3, 1, 1, act="none", bn=False, bias=False, name=f"b{bi}l{li}.conv2",
+                   out=buf[..., c:c + 32])
+            c += 32
+        if bi < len(blocks) - 1:
+            t = b.bn_act(buf.view(hw * hw, -1), "relu", name=f"trans{bi}.norm")
+            t = b.conv(t.view(1, hw, hw, c), c // 2, 1, 1, 0, act="none", bn=False, bias=False,
+                       name=f"trans{bi}.conv")
+            c = c // 2
+            hw //= 2
+            buf = b.act_buf((1, hw, hw, c + blocks[bi + 1] * 32))
+            b.pool(t, 2, 2, 0, "avg", name=f"trans{bi}.pool", out=buf[..., :c])
+    t = b.bn_act(buf.view(hw * hw, -1), "relu", name="norm5")
+    x = b.pool(t.view(1, hw, hw, c), 0, 1, 0, "gap", name="avgpool")
+    x = b.gemm(x, 1000, act="none", name="classifier")
+    return b.done(x)
+
+
 BUILDERS = {
     "mlp": tiny_mlp,
     "cnn": tiny_cnn,
     "vgg11": vgg11,
+    "vgg16": lambda ctx, t, q, dtype="bf16", seed=1000: vgg(ctx, t, q, "vgg16", dtype, seed),
     "resnet50": lambda ctx, t, q, dtype="bf16", seed=1000: resnet(ctx, t, q, 50, dtype, seed),
     "resnet152": lambda ctx, t, q, dtype="bf16", seed=1000: resnet(ctx, t, q, 152, dtype, seed),
+    "mobilenet_v2": mobilenet_v2,
+    "bert_base": lambda ctx, t, q, dtype="bf16", seed=1000: bert(ctx, t, q, "base", 128, dtype, seed),
+    "bert_large": lambda ctx, t, q, dtype="bf16", seed=1000: bert(ctx, t, q, "large", 384, dtype, seed),
+    "densenet121": densenet121,
 }
 
 CONFIGS = {
     "C1": [("mlp", 1 / 3), ("cnn", 2 / 3)],
     "C2": [("vgg11", 1 / 3), ("resnet50", 2 / 3)],
+    "C3": [("resnet50", 0.4), ("vgg16", 0.3), ("bert_base", 0.2), ("mobilenet_v2", 0.1)],
+    "C4": [("bert_large", 0.5), ("resnet152", 0.25), ("densenet121", 0.25)],
 }
 
 

@@ -27,6 +27,22 @@ def reference(layer):
     if layer.kind == "im2col":
         g = layer.geom
         return im2col_ref(x, g["k"], g["stride"], g["pad"], g["Kpad"])
+    if layer.kind == "eltwise":
+        return L.bn_act_nhwc(x, np64(layer.scale), np64(layer.shift), layer.act)
+    if layer.kind == "layernorm":
+        return L.layernorm(x, np64(layer.scale), np64(layer.shift), layer.geom["eps"], np64(layer.res))
+    if layer.kind == "attention":
+        H, dh = layer.geom["heads"], layer.geom["dh"]
+        Lq = x.shape[0]
+        q = x[:, :H * dh].reshape(Lq, H, dh).transpose(1, 0, 2)
+        k = x[:, H * dh:2 * H * dh].reshape(Lq, H, dh).transpose(1, 0, 2)
+        v = x[:, 2 * H * dh:].reshape(Lq, H, dh).transpose(1, 0, 2)
+        return L.sdpa(q, k, v).transpose(1, 0, 2).reshape(Lq, H * dh)
+    if layer.kind == "embed":
+        g = layer.geom
+        ids = layer.x.detach().cpu().numpy()
+        return L.embedding(ids, np64(layer.w), np64(g["pos"]), np64(g["typ"]), np64(layer.scale),
+                           np64(layer.shift), g["eps"])
     raise ValueError(layer.kind)
 
 

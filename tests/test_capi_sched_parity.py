@@ -37,6 +37,13 @@ def test_library_exports_every_declared_symbol():
     assert b"sm_100a" in L.bl_version()
 
 
+def test_enum_mirror_matches_header():
+    """Every enumerator of bless.h has the same value in the Python binding."""
+    src = open(HEADER).read()
+    for name, val in re.findall(r"\b(BL_[A-Z0-9_]+)\s*=\s*(-?\d+)", src):
+        assert getattr(capi, name) == int(val), name
+
+
 def _ctx_from(pf, tmp_path, **kw):
     path = str(tmp_path / "profile.txt")
     sp.save(path, pf)
