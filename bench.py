@@ -35,7 +35,21 @@ from synth import profile as synprof  # noqa: E402
 from synth import trace as syntrace  # noqa: E402
 
 METRIC = "avg/p99 request latency per tenant at fixed quotas vs time-slice/static-split; quota attainment %"
-CONFIG_NAMES = {"C1": "tiny MLP (1/3) + tiny CNN (2/3), fp32", "C2": "VGG11 (1/3) + ResNet50 (2/3), bf16 batch 1"}
+CONFIG_NAMES = {"C1": "tiny MLP (1/3) + tiny CNN (2/3), fp32",
+                "C2": "VGG11 (1/3) + ResNet50 (2/3), bf16 batch 1",
+                "C3": "ResNet50 (0.4) + VGG16 (0.3) + BERT-base s128 (0.2) + MobileNetV2 (0.1), bf16 batch 1",
+                "C4": "BERT-large s384 (1/2) + ResNet152 (1/4) + DenseNet121 (1/4), bf16 batch 1, bursty",
+                "C5": "per-GPU mix of C2/C3/C4 (GPU g hosts C[2 + g mod 3])"}
+
+
+# tenant (name, quota) per config -- data only, so the reference arm imports
+# nothing from the product package
+REF_CONFIGS = {
+    "C1": [("mlp", 1 / 3), ("cnn", 2 / 3)],
+    "C2": [("vgg11", 1 / 3), ("resnet50", 2 / 3)],
+    "C3": [("resnet50", 0.4), ("vgg16", 0.3), ("bert_base", 0.2), ("mobilenet_v2", 0.1)],
+    "C4": [("bert_large", 0.5), ("resnet152", 0.25), ("densenet121", 0.25)],
+}
 
 
 def parse():
@@ -44,7 +58,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="native", choices=["native", "reference"])
-    ap.add_argument("--config", default="C2", choices=["C1", "C2"])
+    ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4", "C5"])
     ap.add_argument("--rho", type=float, default=0.5, help="per-tenant load relative to its ISO latency")
     ap.add_argument("--requests", type=int, default=60, help="requests per tenant per step")
     ap.add_argument("--squad-max", type=int, default=50)
@@ -146,8 +160,13 @@ def squad_timeline(decisions, launches):
             "makespan_us_median": float(np.median([e - s for s, e, _, _ in spans])) / 1e3}
 
 
-def make_trace(T_iso, rho, n, seed):
-    return syntrace.poisson([T / rho for T in T_iso], n, seed)
+def make_trace(T_iso, rho, n, seed, bursty=False):
+    """Poisson (C1-C3, C5) or bursty MMPP-2 (C4: ON 20% at 4x, OFF at 0.25x the
+    mean rate, exponential dwell 20 / 80 ms) per tenant."""
+    gaps = [T / rho for T in T_iso]
+    if bursty:
+        return syntrace.mmpp2(gaps, n, seed)
+    return syntrace.poisson(gaps, n, seed)
 
 
 def run_policy(ctx, capi, params, trace, tenants_filter=None):
@@ -250,8 +269,8 @@ def native(args):
 
     def step(seed, pol="BLESS", filt=None, extra=None):
         p = capi.default_params(squad_max=args.squad_max, policy=pol, **(extra or {}))
-        return run_policy(ctx, capi, p, make_trace(T_iso, args.rho, args.requests, seed + plan.trace_seed_offset),
-                          filt)
+        return run_policy(ctx, capi, p, make_trace(T_iso, args.rho, args.requests, seed + plan.trace_seed_offset,
+                                                   args.config == "C4"), filt)
 
     for w in range(args.warmup):
         flush.zero_()
@@ -411,7 +430,8 @@ def native(args):
         "metric": METRIC, "value": mean_ms, "unit": "ms", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": step_ms, "higher_is_better": False, "scaling": "weak",
         "vs_baseline": None, "dtype": "bf16" if dtype == "bf16" else "f32", "data": "synthetic",
-        "config": {"workload": f"{args.config}: {CONFIG_NAMES[args.config]}", "trace": f"Poisson rho={args.rho} "
+        "config": {"workload": f"{args.config}: {CONFIG_NAMES[args.config]}",
+                   "trace": f"{'MMPP-2 bursty' if args.config == 'C4' else 'Poisson'} rho={args.rho} "
                    f"per tenant, {args.requests} requests/tenant/step, seeds 1-3", "squad_max": args.squad_max,
                    "parallelism": f"replicas x{world} (no collective)",
                    "l2": "256 MiB buffer written between timed steps (> 126 MB L2); VGG11 weights 266 MB > L2"},
@@ -439,22 +459,23 @@ def reference(args):
     from oracle.sched_ref import Params, Prof
     from threadpoolctl import threadpool_info
 
-    names = {"C1": ["mlp", "cnn"], "C2": ["vgg11", "resnet50"]}[args.config]
+    cfg = "C2" if args.config == "C5" else args.config
+    tenants = REF_CONFIGS[cfg]
+    names = [n for n, _ in tenants]
     # profile table: the last B200 profile committed under profiles/, else a synthetic stand-in
-    cand = os.path.join(ROOT, "profiles", f"profile_{args.config}_b200.txt")
+    cand = os.path.join(ROOT, "profiles", f"profile_{cfg}_b200.txt")
     if os.path.exists(cand):
         prof = Prof(synprof.load(cand))
         src = cand
     else:
         g = np.random.Generator(np.random.PCG64(7))
-        tn = [synprof.random_tenant(n, q, m, 148, g, s, 0.6, 0.2, 1500)
-              for n, q, m, s in zip(names, [333333, 666667], [16, 56], [1.5e6, 0.6e6])]
+        tn = [synprof.random_tenant(n, int(round(q * 1e6)), 40, 148, g, 1e6, 0.6, 0.2, 1500) for n, q in tenants]
         prof = Prof(synprof.ProfileFile(148, 4, tn))
         src = "synthetic"
     vals = []
     for it in range(args.warmup + args.steps):
         t0 = time.perf_counter()
-        trace = make_trace(prof.T, args.rho, max(4, args.requests // 10), 1 + it % 3)
+        trace = make_trace(prof.T, args.rho, max(4, args.requests // 10), 1 + it % 3, cfg == "C4")
         res = des.run_bless(trace, prof, Params(squad_max=args.squad_max))
         t_dec = time.perf_counter() - t0
         fw = {}
