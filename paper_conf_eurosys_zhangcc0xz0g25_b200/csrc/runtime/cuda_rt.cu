@@ -70,6 +70,8 @@ __global__ void k_gt_res(long long* out) {
 bool build_kernel(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err) {
   if (op.kind == BL_OP_VIRTUAL) { err = "virtual op on a device ctx"; return false; }
   std::string e2;
+  if (build_attn_tc(op, caps, out, e2)) return true;
+  if (!e2.empty()) { err = e2; return false; }
   if (build_nn(op, caps, out, e2)) return true;
   if (!e2.empty()) { err = e2; return false; }
   if (op.dtype == BL_BF16 && op.kind == BL_OP_GEMM && op.dims[0] <= 8) {

@@ -44,5 +44,6 @@ bool build_simt(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::s
 bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
 bool build_gemv_tma(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
 bool build_nn(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
+bool build_attn_tc(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
 
 }  // namespace bless

@@ -105,6 +105,44 @@ def test_pool(ctx, H, W, C, k, s, p, mode, dtype):
     run_and_check(ctx, m, dtype)
 
 
+@pytest.mark.parametrize("L,H", [(128, 12), (384, 16), (256, 4), (96, 2)])
+@pytest.mark.parametrize("path", ["tc", "simt"])
+def test_attention(ctx, L, H, path, monkeypatch):
+    """SDPA per head (all-ones mask): tcgen05 path for L % 128 == 0, L <= 384;
+    CUDA-core path otherwise or when forced."""
+    if path == "simt":
+        monkeypatch.setenv("BLESS_ATTN_SIMT", "1")
+    else:
+        monkeypatch.delenv("BLESS_ATTN_SIMT", raising=False)
+
+    def mk(b):
+        qkv = b.input((L, 3 * H * 64))
+        b.attention(qkv, H, 64)
+    m = one_layer(ctx, "bf16", mk)
+    fam = ctx.kernel_info(m.tenant, 0).family.decode()
+    assert fam == ("attention_tc_bf16" if path == "tc" and L % 128 == 0 else "attention_bf16"), fam
+    run_and_check(ctx, m, "bf16")
+
+
+@pytest.mark.parametrize("rows,C,res", [(128, 768, False), (384, 1024, True), (7, 256, True)])
+def test_layernorm(ctx, rows, C, res):
+    def mk(b):
+        x = b.input((rows, C))
+        r = b.param(np.random.default_rng(3).standard_normal((rows, C)).astype(np.float32)) if res else None
+        b.layernorm(x, res=r)
+    m = one_layer(ctx, "bf16", mk)
+    run_and_check(ctx, m, "bf16")
+
+
+@pytest.mark.parametrize("H,C,stride", [(112, 32, 1), (56, 144, 2), (7, 960, 1)])
+def test_dwconv(ctx, H, C, stride):
+    def mk(b):
+        x = b.input((1, H, H, C))
+        b.dwconv(x, 3, stride)
+    m = one_layer(ctx, "bf16", mk)
+    run_and_check(ctx, m, "bf16")
+
+
 def test_tc_kernel_uses_only_its_sms(ctx):
     """A tensor-core conv launched on logical SMs [40, 44) processes tiles
     only there (launch log mask), via the engine's STATIC policy."""
