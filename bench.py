@@ -61,7 +61,12 @@ def parse():
     ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4", "C5"])
     ap.add_argument("--rho", type=float, default=0.5, help="per-tenant load relative to its ISO latency")
     ap.add_argument("--requests", type=int, default=60, help="requests per tenant per step")
-    ap.add_argument("--squad-max", type=int, default=50)
+    # B200 operating point chosen by the c% x S_max sweep, the
+    # way the paper picks its own empirically (§6.7).
+    ap.add_argument("--squad-max", type=int, default=20)
+    ap.add_argument("--split-pct", type=int, default=25)
+    ap.add_argument("--lookahead-us", type=float, default=20.0)
+    ap.add_argument("--max-inflight", type=int, default=2)
     ap.add_argument("--profile-reps", type=int, default=5)
     ap.add_argument("--no-baselines", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -194,7 +199,7 @@ def run_policy(ctx, capi, params, trace, tenants_filter=None):
 
 
 # ---------------------------------------------------------------------------- cpu baseline (oracle)
-def oracle_timing(cfg_models, decisions, prof, requests_per_tenant_seen, squads_per_req):
+def oracle_timing(cfg_models, decisions, prof, requests_per_tenant_seen, squads_per_req, params):
     """Time the oracle as it stands: one fp64 forward per tenant (all host
     cores, numpy BLAS) plus decide_ref on a sample of decision records."""
     from threadpoolctl import threadpool_info
@@ -212,7 +217,7 @@ def oracle_timing(cfg_models, decisions, prof, requests_per_tenant_seen, squads_
     for rec in decisions[:40]:
         got = _c.decision_to_tuple(rec)
         t0 = time.perf_counter()
-        decide_ref(got["now"], [Active(*a) for a in got["active"]], prof, Params(squad_max=50))
+        decide_ref(got["now"], [Active(*a) for a in got["active"]], prof, params)
         dec_t.append(time.perf_counter() - t0)
     mean_dec = float(np.mean(dec_t)) if dec_t else 0.0
     per_req = [fwd[n] + mean_dec * squads_per_req for n in cfg_models]
@@ -268,7 +273,9 @@ def native(args):
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 
     def step(seed, pol="BLESS", filt=None, extra=None):
-        p = capi.default_params(squad_max=args.squad_max, policy=pol, **(extra or {}))
+        p = capi.default_params(squad_max=args.squad_max, policy=pol, split_pct=args.split_pct,
+                                lookahead_ns=int(args.lookahead_us * 1000), max_inflight_squads=args.max_inflight,
+                                **(extra or {}))
         return run_policy(ctx, capi, p, make_trace(T_iso, args.rho, args.requests, seed + plan.trace_seed_offset,
                                                    args.config == "C4"), filt)
 
@@ -405,10 +412,11 @@ def native(args):
     # ---------------- cpu baseline (oracle), rank 0 at N=1 only
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        from oracle.sched_ref import Prof
+        from oracle.sched_ref import Params, Prof
         prof = Prof(synprof.load(prof_path))
         sq = len(decisions_all) / max(1, n_local)
-        cpu = oracle_timing(names, decisions_all, prof, [len(lat_all[j]) for j in range(len(tms))], sq * 2)
+        cpu = oracle_timing(names, decisions_all, prof, [len(lat_all[j]) for j in range(len(tms))], sq * 2,
+                            Params(squad_max=args.squad_max, split_pct=args.split_pct))
 
     # decisions replayed bit-exactly through the oracle (sample)
     replay_ok = None
@@ -418,7 +426,7 @@ def native(args):
         replay_ok = 0
         for rec in decisions_all[:200]:
             got = capi.decision_to_tuple(rec)
-            ref = decide_ref(got["now"], [Active(*a) for a in got["active"]], prof, Params(squad_max=args.squad_max))
+            ref = decide_ref(got["now"], [Active(*a) for a in got["active"]], prof, Params(squad_max=args.squad_max, split_pct=args.split_pct))
             replay_ok += int(got["picks"] == [tuple(p) for p in ref.picks] and got["config"] == ref.config
                              and got["t_hat"] == ref.t_hat)
         replay_ok = f"{replay_ok}/{min(200, len(decisions_all))}"
@@ -476,7 +484,7 @@ def reference(args):
     for it in range(args.warmup + args.steps):
         t0 = time.perf_counter()
         trace = make_trace(prof.T, args.rho, max(4, args.requests // 10), 1 + it % 3, cfg == "C4")
-        res = des.run_bless(trace, prof, Params(squad_max=args.squad_max))
+        res = des.run_bless(trace, prof, Params(squad_max=args.squad_max, split_pct=args.split_pct))
         t_dec = time.perf_counter() - t0
         fw = {}
         for i, n in enumerate(names):
