@@ -21,6 +21,8 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 
@@ -200,7 +202,11 @@ struct TcCfg {
   static constexpr int kStageB = BN * BK * 2;
   static constexpr int kStageBytes = kStageA + kStageB;
   static constexpr int kStages = std::min(6, (96 * 1024) / kStageBytes);
-  static constexpr int kTmemCols = (2 * BN) < 32 ? 32 : 2 * BN;
+  // TMEM accumulators: double buffered (epilogue of tile i overlaps the MMAs of
+  // tile i+1) up to BN = 128; BN = 256 keeps one so a second co-resident CTA
+  // (another tenant's kernel on the same SM) can still allocate.
+  static constexpr int kAcc = BN >= 256 ? 1 : 2;
+  static constexpr int kTmemCols = (kAcc * BN) < 32 ? 32 : kAcc * BN;
   static constexpr int kSmem = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/ + 2 * BN * 4 /*sc, sh*/;
 };
 
@@ -376,7 +382,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       }
       if (lane == 0) tc_commit(&tfull[acc]);
       __syncwarp();
-      if (++acc == 2) { acc = 0; aph ^= 1; }
+      if (++acc == Cfg::kAcc) { acc = 0; aph ^= 1; }
     }
   } else {
     // ---------------- epilogue warps 2..5 (TMEM lane quarter = warp % 4)
@@ -484,7 +490,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           if (threadIdx.x == 64) p.sem[tile] = 0;
         }
       }
-      if (++acc == 2) { acc = 0; aph ^= 1; }
+      if (++acc == Cfg::kAcc) { acc = 0; aph ^= 1; }
     }
   }
   tc_fence_before();
@@ -567,7 +573,7 @@ static bool encode(CUtensorMap* map, int rank, const void* base, const cuuint64_
   return true;
 }
 
-bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::string& err) {
+bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::string& err, const TcChoice* force) {
   err.clear();
   if (op.dtype != BL_BF16 || caps.cc_major != 10) return false;
   TcParams p;
@@ -580,6 +586,10 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   const void* X = op.ptr[0];
   const void* W = op.ptr[1];
   int BK = 64;
+  // BLESS_TC_CFG="BN,BK,splits" forces a tile configuration (sweeps only, tools/tcsweep.py)
+  int fbn = 0, fbk = 0, fs = 0;
+  if (const char* f = std::getenv("BLESS_TC_CFG")) std::sscanf(f, "%d,%d,%d", &fbn, &fbk, &fs);
+  const bool fbk_ok = fbk == 16 || fbk == 32 || fbk == 64;
   if (op.kind == BL_OP_GEMM) {
     p.M = (int)op.dims[0];
     p.N = (int)op.dims[1];
@@ -590,7 +600,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     if (p.M <= 8 || p.N % 16 || p.K % 8 || ldx % 8 || p.ldy % 8 || p.ldr % 8) return false;  // GEMV / SIMT
     if (((uintptr_t)X | (uintptr_t)W) & 15) return false;
     p.mode = 0;
-    BK = 64;
+    BK = fbk_ok ? fbk : 64;
     p.num_kb = (p.K + BK - 1) / BK;
     cuuint64_t da[2] = {(cuuint64_t)p.K, (cuuint64_t)p.M}, sa[1] = {(cuuint64_t)ldx * 2};
     cuuint32_t ba[2] = {(cuuint32_t)BK, 128};
@@ -610,6 +620,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     if (((uintptr_t)X | (uintptr_t)W) & 15) return false;
     // 1x1 stride-1 convs are plain GEMMs over pixels: any C % 8, K tail zero-filled by TMA
     BK = one_by_one ? 64 : ((C % 64 == 0) ? 64 : (C % 32 == 0 ? 32 : 16));
+    if (fbk_ok && fbk < BK) BK = fbk;
     p.OH = (H + 2 * pad - R) / stride + 1;
     p.OW = (Wd + 2 * pad - S) / stride + 1;
     p.M = p.OH * p.OW;
@@ -669,6 +680,15 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     const int want = (int)((caps.S + ntiles(BN) - 1) / ntiles(BN));
     splits = std::max(1, std::min(want, p.num_kb / 3));
   }
+  if (force && force->bn) {
+    fbn = force->bn;
+    fs = force->splits;
+  }
+  if (fbn >= 16 && fbn <= 256 && (fbn & (fbn - 1)) == 0) {
+    BN = fbn;
+    p.tiles_n = (p.N + BN - 1) / BN;
+  }
+  if (fs >= 1) splits = std::min(fs, p.num_kb);
   p.kbs = (p.num_kb + splits - 1) / splits;
   p.splits = (p.num_kb + p.kbs - 1) / p.kbs;
   if (p.splits > 1) {
@@ -682,6 +702,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     }
     p.ws = (float*)buf;
     p.sem = (unsigned*)((char*)buf + wsb);
+    d.owned = buf;
   }
   {
     cuuint64_t db[2] = {(cuuint64_t)p.K, (cuuint64_t)p.N}, sb[1] = {(cuuint64_t)p.K * 2};
@@ -699,6 +720,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   TC_CASE(32, 16) TC_CASE(32, 32) TC_CASE(32, 64)
   TC_CASE(64, 16) TC_CASE(64, 32) TC_CASE(64, 64)
   TC_CASE(128, 16) TC_CASE(128, 32) TC_CASE(128, 64)
+  TC_CASE(256, 16) TC_CASE(256, 32) TC_CASE(256, 64)
 #undef TC_CASE
   if (!ok) {
     if (err.empty()) err = "no tc instantiation";
@@ -706,11 +728,51 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   }
   static_assert(sizeof(TcParams) <= sizeof(d.params), "params block too small");
   std::memcpy(d.params, &p, sizeof(p));
+  d.choice_bn = BN;
+  d.choice_splits = p.splits;
   d.family = op.kind == BL_OP_GEMM ? "tc_gemm_bf16" : (p.mode == 0 ? "tc_conv1x1_bf16" : "tc_conv_bf16");
   d.flops = 2.0 * p.M * p.N * p.K;
   double a_bytes = (op.kind == BL_OP_CONV) ? 2.0 * op.dims[1] * op.dims[2] * op.dims[3] : 2.0 * p.M * p.K;
   d.bytes = a_bytes + 2.0 * p.N * p.K + 2.0 * p.M * p.N * (p.R ? 2 : 1);
   return true;
+}
+
+// Candidate tile configurations for the registration-time autotuner
+// (DeviceRT::add_kernel): BN in {32, 64, 128} (narrower when N is small), each
+// unsplit and split-K to about S work units.  Measured on B200 (tools/tcsweep.py,
+// profiles/round1/tcsweep.txt) no single rule picks the fastest: unsplit tiles
+// below S often win (split-K's fp32 reduction costs several us), wide tiles win
+// on large convs; BN = 256 never won with 96 KB of pipeline stages.
+int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int max) {
+  long long M, N, num_kb, tiles_m;
+  if (op.kind == BL_OP_GEMM) {
+    M = op.dims[0], N = op.dims[1];
+    num_kb = (op.dims[2] + 63) / 64;
+    tiles_m = (M + 127) / 128;
+  } else if (op.kind == BL_OP_CONV) {
+    const long long H = op.dims[1], W = op.dims[2], C = op.dims[3], R = op.dims[5], S = op.dims[6];
+    const long long st = op.dims[7] ? op.dims[7] : 1, pad = op.dims[8];
+    const long long OH = (H + 2 * pad - R) / st + 1, OW = (W + 2 * pad - S) / st + 1;
+    N = op.dims[4];
+    num_kb = R * S * std::max(1LL, C / 64);
+    long long BW = 8;
+    while (BW < OW && BW < 128) BW <<= 1;
+    tiles_m = ((OW + BW - 1) / BW) * ((OH + (128 / BW) - 1) / (128 / BW));
+  } else {
+    return 0;
+  }
+  int n = 0;
+  const int nmax = N <= 16 ? 16 : (N <= 32 ? 32 : (N <= 64 ? 64 : 128));
+  for (int bn = std::min(32, nmax); bn <= nmax && n < max; bn <<= 1) {
+    const long long tiles = tiles_m * ((N + bn - 1) / bn);
+    out[n++] = TcChoice{bn, 1};
+    if (tiles < caps.S && num_kb >= 6 && n < max) {
+      const long long want = std::min<long long>((caps.S + tiles - 1) / tiles, num_kb / 3);
+      if (want >= 2) out[n++] = TcChoice{bn, (int)want};
+      if (want >= 6 && n < max) out[n++] = TcChoice{bn, (int)(want / 2)};
+    }
+  }
+  return n;
 }
 
 }  // namespace bless

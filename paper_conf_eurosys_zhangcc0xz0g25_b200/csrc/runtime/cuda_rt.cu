@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdio>
 #include <atomic>
 #include <chrono>
 #include <cstring>
@@ -134,6 +135,16 @@ std::unique_ptr<DeviceRT> DeviceRT::create(int device, void* ws, size_t ws_bytes
     return nullptr;
   }
   if (const char* e = std::getenv("BLESS_PDL")) g_use_pdl = std::atoi(e) != 0;
+  if (const char* e = std::getenv("BLESS_TC_AUTOTUNE")) rt->autotune_ = std::atoi(e) != 0;
+  if (const char* e = std::getenv("BLESS_TC_TUNE_FILE")) {   // "sig bn splits" lines, appended as tuned
+    rt->tune_file_ = e;
+    if (FILE* f = std::fopen(e, "r")) {
+      char sig[512];
+      int bn = 0, sp = 0;
+      while (std::fscanf(f, "%511s %d %d", sig, &bn, &sp) == 3) rt->tune_cache_[sig] = TcChoice{bn, sp};
+      std::fclose(f);
+    }
+  }
   if (!rt->probe(err)) return nullptr;
   if (!rt->calibrate_clock(err)) return nullptr;
   return rt;
@@ -148,6 +159,9 @@ DeviceRT::~DeviceRT() {
   if (reader_ev_) cudaEventDestroy((cudaEvent_t)reader_ev_);
   if (reader_) cudaStreamDestroy((cudaStream_t)reader_);
   if (lid_map_dev_) cudaFree(lid_map_dev_);
+  for (auto& k : kernels_)
+    if (k && k->owned) cudaFree(k->owned);
+  if (tune_stream_) cudaStreamDestroy((cudaStream_t)tune_stream_);
 }
 
 bool DeviceRT::set_device() { return cudaSetDevice(device_) == cudaSuccess; }
@@ -239,8 +253,95 @@ int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
   if (!build_kernel(op, caps_, *kd, err)) return -1;
   // grid = S x (resident blocks per SM): see gate_linger in executor.cuh
   if (kd->kernel_fn) kd->grid = full_occupancy_grid(kd->kernel_fn, kd->block, (size_t)kd->smem, caps_.S);
+  if (kd->choice_bn && autotune_ && !std::getenv("BLESS_TC_CFG")) {
+    const std::string sig = tc_signature(op);
+    auto it = tune_cache_.find(sig);
+    if (it != tune_cache_.end()) {
+      if (it->second.bn != kd->choice_bn || it->second.splits != kd->choice_splits) {
+        std::unique_ptr<KernelDesc> k2(new KernelDesc());
+        std::string e2;
+        if (build_tc_gemm(op, caps_, *k2, e2, &it->second)) {
+          k2->grid = full_occupancy_grid(k2->kernel_fn, k2->block, (size_t)k2->smem, caps_.S);
+          if (kd->owned) cudaFree(kd->owned);
+          kd = std::move(k2);
+        }
+      }
+    } else {
+      if (!autotune_tc(op, kd, err)) return -1;
+      tune_cache_[sig] = TcChoice{kd->choice_bn, kd->choice_splits};
+      if (!tune_file_.empty()) {
+        if (FILE* f = std::fopen(tune_file_.c_str(), "a")) {
+          std::fprintf(f, "%s %d %d\n", sig.c_str(), kd->choice_bn, kd->choice_splits);
+          std::fclose(f);
+        }
+      }
+    }
+  }
   kernels_.push_back(std::move(kd));
   return (int)kernels_.size() - 1;
+}
+
+// Shape signature of a tc op for the tuning cache (pointers excluded).
+std::string DeviceRT::tc_signature(const bl_op& op) const {
+  std::string s = "k" + std::to_string(op.kind) + "_t" + std::to_string(op.dtype) + "_r" + (op.ptr[4] ? "1" : "0");
+  for (int i = 0; i < 12; ++i) s += "_" + std::to_string(op.dims[i]);
+  return s;
+}
+
+// Registration-time choice of the tcgen05 tile configuration (part of the
+// offline profiling stage): every candidate is timed like
+// the profiler times a kernel (back-to-back launches on one stream, CUDA
+// events, all S SMs) on the layer's own buffers; the fastest wins, and within
+// 3 % of it the one with fewer tiles (smaller d leaves more SMs to co-runners).
+bool DeviceRT::autotune_tc(const bl_op& op, std::unique_ptr<KernelDesc>& best, std::string& err) {
+  TcChoice cand[8];
+  const int nc = tc_candidates(op, caps_, cand, 8);
+  if (nc <= 1) return true;
+  if (!tune_stream_ && cudaStreamCreateWithFlags((cudaStream_t*)&tune_stream_, cudaStreamNonBlocking) != cudaSuccess) {
+    err = "autotune stream";
+    return false;
+  }
+  int64_t best_ns = 0;
+  {
+    kernels_.push_back(std::move(best));
+    const int h = (int)kernels_.size() - 1;
+    const bool ok = profile(h, caps_.S, 4, tune_stream_, &best_ns, nullptr, err);
+    best = std::move(kernels_.back());
+    kernels_.pop_back();
+    if (!ok) return false;
+  }
+  for (int i = 0; i < nc; ++i) {
+    if (cand[i].bn == best->choice_bn && cand[i].splits == best->choice_splits) continue;
+    std::unique_ptr<KernelDesc> kd(new KernelDesc());
+    std::string e2;
+    if (!build_tc_gemm(op, caps_, *kd, e2, &cand[i])) continue;
+    if (kd->choice_bn == best->choice_bn && kd->choice_splits == best->choice_splits) {
+      if (kd->owned) cudaFree(kd->owned);
+      continue;
+    }
+    kd->grid = full_occupancy_grid(kd->kernel_fn, kd->block, (size_t)kd->smem, caps_.S);
+    kernels_.push_back(std::move(kd));
+    const int h = (int)kernels_.size() - 1;
+    int64_t ns = 0;
+    const bool ok = profile(h, caps_.S, 4, tune_stream_, &ns, nullptr, err);
+    kd = std::move(kernels_.back());
+    kernels_.pop_back();
+    if (!ok) {
+      if (kd->owned) cudaFree(kd->owned);
+      return false;
+    }
+    const bool better = (double)ns < 0.97 * (double)best_ns ||
+                        ((double)ns <= 1.03 * (double)best_ns && kd->tiles < best->tiles);
+    std::unique_ptr<KernelDesc>& loser = better ? best : kd;
+    if (better) best_ns = ns;
+    if (loser->owned) {
+      cudaStreamSynchronize((cudaStream_t)tune_stream_);
+      cudaFree(loser->owned);
+      loser->owned = nullptr;
+    }
+    if (better) best = std::move(kd);
+  }
+  return true;
 }
 
 GateArgs DeviceRT::make_gate(uint64_t seq, uint32_t tiles, int lo, int hi) const {

@@ -3,6 +3,7 @@
 // (A2).  Host-only declarations; implemented in cuda_rt.cu.
 #pragma once
 #include <cstdint>
+#include <map>
 #include <memory>
 #include <string>
 #include <vector>
@@ -89,6 +90,12 @@ class DeviceRT {
   bool identity_map_ = true;
   uint64_t seq_ = 0;
   std::vector<std::unique_ptr<KernelDesc>> kernels_;
+  bool autotune_ = true;          // BLESS_TC_AUTOTUNE=0 keeps the builder's heuristic
+  void* tune_stream_ = nullptr;
+  bool autotune_tc(const bl_op& op, std::unique_ptr<KernelDesc>& best, std::string& err);
+  std::string tc_signature(const bl_op& op) const;
+  std::map<std::string, TcChoice> tune_cache_;   // BLESS_TC_TUNE_FILE
+  std::string tune_file_;
 };
 
 constexpr uint64_t kSlotRing = 65536;

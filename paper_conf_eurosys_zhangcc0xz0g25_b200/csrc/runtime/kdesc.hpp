@@ -27,6 +27,8 @@ struct KernelDesc {
   double bytes = 0;        // algorithmic HBM bytes per launch (roofline)
   LaunchFn launch = nullptr;
   const void* kernel_fn = nullptr;  // for the occupancy query (grid = S x blocks/SM)
+  void* owned = nullptr;   // device scratch owned by this kernel (split-K workspace), cudaFree'd with it
+  int choice_bn = 0, choice_splits = 0;  // tcgen05 tile configuration (0 = not a tc kernel)
   alignas(128) unsigned char params[4096];  // family-specific parameter block
 };
 
@@ -41,7 +43,15 @@ bool build_kernel(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std:
 
 // Per-family builders (return true if they took the op).
 bool build_simt(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
-bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
+// tcgen05 GEMM/conv: tile configuration (BN, split-K factor); zero = the
+// builder's default heuristic.  tc_candidates lists the configurations the
+// registration-time autotuner times for one op (returns how many).
+struct TcChoice {
+  int bn = 0, splits = 0;
+};
+bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err,
+                   const TcChoice* force = nullptr);
+int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int max);
 bool build_gemv_tma(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
 bool build_nn(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);
 bool build_attn_tc(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err);

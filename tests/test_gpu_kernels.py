@@ -94,6 +94,31 @@ def test_conv_bf16(ctx, H, W, C, K, k, s, p, act, res):
     run_and_check(ctx, m, "bf16")
 
 
+@pytest.mark.parametrize("cfg", ["256,64,1", "256,32,3", "128,64,5", "64,32,2", "32,64,1"])
+@pytest.mark.parametrize("shape", [("conv", (56, 56, 64, 256, 3, 1, 1)), ("conv", (28, 28, 128, 256, 3, 2, 1)),
+                                   ("conv", (14, 14, 256, 512, 1, 1, 0)), ("gemm", (384, 1024, 320)),
+                                   ("gemm", (200, 272, 136))])
+def test_tc_forced_configs(ctx, cfg, shape, monkeypatch):
+    """Every tile configuration the selector may pick (BN 32..256, BK 32/64,
+    split-K) is exact on convs (stride 1/2, 1x1) and ragged GEMMs."""
+    monkeypatch.setenv("BLESS_TC_CFG", cfg)
+    kind, dims = shape
+
+    def mk(b):
+        if kind == "conv":
+            H, W, C, K, k, s, p = dims
+            x = b.input((1, H, W, C))
+            OH, OW = (H + 2 * p - k) // s + 1, (W + 2 * p - k) // s + 1
+            r = b.param(np.random.default_rng(2).standard_normal((1, OH, OW, K)).astype(np.float32))
+            b.conv(x, K, k, s, p, act="relu", bn=True, res=r)
+        else:
+            M, N, K = dims
+            b.gemm(b.input((M, K)), N, act="gelu", bias=True)
+    m = one_layer(ctx, "bf16", mk)
+    assert ctx.kernel_info(m.tenant, 0).family.decode().startswith("tc_")
+    run_and_check(ctx, m, "bf16")
+
+
 @pytest.mark.parametrize("H,W,C,k,s,p,mode", [(112, 112, 64, 3, 2, 1, "max"), (224, 224, 64, 2, 2, 0, "max"),
                                               (9, 8, 5, 3, 2, 1, "avg"), (7, 7, 2048, 0, 1, 0, "gap")])
 @pytest.mark.parametrize("dtype", ["bf16", "fp32"])

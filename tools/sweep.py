@@ -25,6 +25,16 @@ def main():
         k, vs = g.split("=")
         axes.append([(k, v) for v in vs.split(",")])
     prof = os.path.join(ROOT, "profiles", f"profile_{a.config}_b200.txt")
+    if not os.path.exists(prof):   # profile once (kernel configs are autotuned at registration), reuse for all points
+        os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
+        subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--config", a.config, "--no-cpu-baseline",
+                        "--no-baselines", "--steps", "1", "--warmup", "1", "--requests", "10"], capture_output=True)
+        for kind in ("profile", "tctune"):
+            gen = os.path.join(ROOT, "gpurun_out", f"{kind}_{a.config}_rank0.txt")
+            if os.path.exists(gen):
+                os.makedirs(os.path.dirname(prof), exist_ok=True)
+                with open(gen) as f, open(prof.replace("profile_", kind + "_"), "w") as g:
+                    g.write(f.read())
     for point in itertools.product(*axes):
         args = [sys.executable, os.path.join(ROOT, "bench.py"), "--config", a.config, "--no-cpu-baseline",
                 "--steps", str(a.steps), "--warmup", "1", "--requests", str(a.requests)]
