@@ -238,6 +238,16 @@ bl_status bl_device_info_get(bl_ctx* ctx, bl_device_info* out);
 /* Register an application with a GPU quota in (0, 1] (L143, L157).  Before
  * bl_start only.  Sum of quotas must be <= 1 + 1e-9 (BL_E_QUOTA). */
 bl_status bl_register_tenant(bl_ctx* ctx, double quota, const char* name, int* tenant_out);
+/* SLO mode (§6.5: "replacing the isolated latency T[n%] in §4.3.1 with
+ * the required QoS target").  slo_ns > 0 is the tenant's latency target: the
+ * progress order then paces the tenant against tau_prog[k] =
+ * floor(tau[k] * slo_ns / T) instead of tau[k] (reading R30), so a tenant
+ * with a tight target is scheduled as if it were further behind.  slo_ns = 0
+ * restores the default (pace = isolated latency T).  Nothing else changes
+ * (quota SMs, predictors, ranges).  Before bl_start; BL_E_INVALID for a bad
+ * tenant or slo_ns < 0, BL_E_STATE after bl_start.  A profile file may also
+ * carry it ("slo <ns>" after the tenant line; bl_load_profile adopts it). */
+bl_status bl_set_tenant_slo(bl_ctx* ctx, int tenant, int64_t slo_ns);
 /* Optional: run tenant's kernels on a caller-owned cudaStream_t (torch stream). */
 bl_status bl_set_stream(bl_ctx* ctx, int tenant, void* cuda_stream);
 /* Append one kernel to the tenant's per-request kernel sequence.  Validates

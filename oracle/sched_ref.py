@@ -81,6 +81,17 @@ class Prof:
                 row.append(acc)
             self.tau.append(row)
         self.T = [row[-1] if row else 0 for row in self.tau]
+        # SLO mode (§6.5): "replacing the isolated latency
+        # T[n%] in §4.3.1 with the required QoS target".  In P~ = P_r / P_e,
+        # P_r = t_e / SLO and P_e = tau / T, so P~ = t_e / (tau * SLO / T);
+        # reading R30 floors tau * SLO / T to integer ns.  No SLO: tau itself.
+        self.slo = [int(getattr(tn, "slo_ns", 0)) for tn in pf.tenants]
+        self.tau_prog: List[List[int]] = []
+        for j in range(self.ntenants):
+            if self.slo[j] > 0 and self.T[j] > 0:
+                self.tau_prog.append([tk * self.slo[j] // self.T[j] for tk in self.tau[j]])
+            else:
+                self.tau_prog.append(list(self.tau[j]))
 
     def t(self, j: int, k: int, s: int) -> int:
         assert 1 <= s <= self.S, s
@@ -149,7 +160,8 @@ def generate_squad(now: int, active: Sequence[Active], prof: Prof, params: Param
     arr = {a.tenant: a.arrival for a in active}
 
     def tau_done(j: int) -> int:
-        return 0 if nxt[j] == 0 else prof.tau[j][nxt[j] - 1]
+        # pace of the request: tau (default) or tau * SLO / T (SLO mode, R30)
+        return 0 if nxt[j] == 0 else prof.tau_prog[j][nxt[j] - 1]
 
     def key(j: int):
         return behind_key(now, j, arr[j], tau_done(j))

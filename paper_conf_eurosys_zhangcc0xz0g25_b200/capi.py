@@ -97,6 +97,7 @@ _SIGS = {
     "bl_device_info_get": (C.c_int, [C.c_void_p, _P(bl_device_info)]),
     "bl_register_tenant": (C.c_int, [C.c_void_p, C.c_double, C.c_char_p, _P(C.c_int)]),
     "bl_set_stream": (C.c_int, [C.c_void_p, C.c_int, C.c_void_p]),
+    "bl_set_tenant_slo": (C.c_int, [C.c_void_p, C.c_int, C.c_int64]),
     "bl_append_kernel": (C.c_int, [C.c_void_p, C.c_int, _P(bl_op), _P(C.c_int)]),
     "bl_run_kernel": (C.c_int, [C.c_void_p, C.c_int, C.c_int, C.c_int, C.c_int]),
     "bl_set_tenant_io": (C.c_int, [C.c_void_p, C.c_int, C.c_void_p, C.c_void_p, C.c_size_t, C.c_void_p,
@@ -194,6 +195,9 @@ class Ctx:
         t = C.c_int()
         check("bl_register_tenant", lib().bl_register_tenant(self.h, float(quota), name.encode(), C.byref(t)))
         return t.value
+
+    def set_slo(self, tenant: int, slo_ns: int):
+        check("bl_set_tenant_slo", lib().bl_set_tenant_slo(self.h, tenant, int(slo_ns)))
 
     def set_stream(self, tenant: int, stream_ptr: int):
         check("bl_set_stream", lib().bl_set_stream(self.h, tenant, C.c_void_p(stream_ptr)))

@@ -88,6 +88,10 @@ bl_status bl_register_tenant(bl_ctx* ctx, double quota, const char* name, int* t
   GUARD(ctx);
   return wrap([&](std::string& e) { return ctx->eng->register_tenant(quota, name, tenant_out, e); });
 }
+bl_status bl_set_tenant_slo(bl_ctx* ctx, int tenant, int64_t slo_ns) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->set_slo(tenant, slo_ns, e); });
+}
 bl_status bl_set_stream(bl_ctx* ctx, int tenant, void* s) {
   GUARD(ctx);
   return wrap([&](std::string& e) { return ctx->eng->set_stream(tenant, s, e); });

@@ -4,18 +4,22 @@
 //
 //   Y[m, n] = act((sum_k X[m, k] W[n, k]) * scale[n] + shift[n] + R[m, n])
 //
-// A work tile is a block of up to 8 consecutive rows of W, i.e. one contiguous
-// rows*K*2-byte region.  Warp 0 (one thread) streams it into a ring of 16 KB
-// shared-memory stages with cp.async.bulk (TMA bulk copies, completion via
-// mbarrier transaction counts) and keeps streaming into the next claimed tile,
-// so an SM always has kStages*16 KB of weights in flight.  Warps 1..16 consume
-// stages: thread i owns the 16-element run at offset 16*i of every stage,
-// keeps one running dot product per X row, and folds it into shared-memory
-// row partials only when its run crosses into the next row of W.  HBM-bound:
-// no tensor cores (the contraction has M <= 8).
+// A work tile is a block of `rows` (1, 2, 4 or 8) consecutive rows of W, i.e.
+// one contiguous rows*K*2-byte region.  Warp 0 (one thread) streams it into a
+// ring of 16 KB shared-memory stages with cp.async.bulk (TMA bulk copies,
+// completion via mbarrier transaction counts) and keeps streaming into the
+// next claimed tile, so an SM always has kStages*16 KB of weights in flight.
+// A stage holds rows x (8192/rows) k-values, so it is full whatever the tile
+// height: 16/rows consumer warps share a row, each owning a 512-k window of
+// every stage (16 consecutive k per lane), and keep one running dot product
+// per X row that is folded into shared-memory row partials once per tile.
+// Short tiles (rows < 8) keep the dynamic queue's tail short: the last tile an
+// SM pulls is rows*K*2 bytes, ~9 us of one SM's HBM share at rows = 8 for VGG
+// FC1.  HBM-bound: no tensor cores (the contraction has M <= 8).
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 
@@ -45,7 +49,7 @@ constexpr int kGvStages = BLESS_GEMV_STAGES;
 constexpr int kGvElems = kGvStage / 2;        // bf16 elements per stage
 constexpr int kGvConsumers = 16;              // consumer warps
 constexpr int kGvRun = 16;                    // k values per lane per stage
-constexpr int kGvKc = kGvElems / 8;           // k values per stage (8 rows x 1024)
+constexpr int kGvWin = 32 * kGvRun;            // k values per consumer warp per stage (512)
 constexpr int kGvThreads = 32 * (1 + kGvConsumers);
 constexpr int kGvMaxRows = 8;
 constexpr int kGvSmem = kGvStages * kGvStage + 1024 + 8 * kGvMaxRows * 4 + 256;
@@ -155,13 +159,14 @@ __device__ void gemv_work(const GemvTmaParams& p, const GateArgs& g) {
         }
         const int n0 = t * p.rows;
         const int nr = min(p.rows, p.N - n0);
-        // stage = nr row segments of kGvKc k-values (row r at offset r*kGvKc*2)
-        for (long long k0 = 0; k0 < K; k0 += kGvKc) {
-          const uint32_t seg = (uint32_t)(min((long long)kGvKc, K - k0) * 2);
+        const int kc = kGvElems / p.rows;   // k values per row per stage
+        // stage = nr row segments of kc k-values (row r at offset r*kc*2)
+        for (long long k0 = 0; k0 < K; k0 += kc) {
+          const uint32_t seg = (uint32_t)(min((long long)kc, K - k0) * 2);
           gv_wait(&empty[stage], ph ^ 1);
           gv_expect(&full[stage], seg * nr);
           for (int r = 0; r < nr; ++r)
-            gv_bulk(stage_buf + stage * kGvStage + r * (kGvKc * 2), p.W + (size_t)(n0 + r) * K + k0, seg, &full[stage]);
+            gv_bulk(stage_buf + stage * kGvStage + r * (kc * 2), p.W + (size_t)(n0 + r) * K + k0, seg, &full[stage]);
           if (++stage == kGvStages) { stage = 0; ph ^= 1; }
         }
       }
@@ -179,19 +184,21 @@ __device__ void gemv_work(const GemvTmaParams& p, const GateArgs& g) {
       if (t < 0) break;
       const int n0 = t * p.rows;
       const int nr = min(p.rows, p.N - n0);
-      // consumer warp cw owns row (cw & 7) of the tile and k-half (cw >> 3) of
-      // every stage: 16 consecutive k per lane; the X slice of a stage (2 KB)
-      // is shared by all 8 rows through L1
-      const int row = (warp - 1) & 7, half = (warp - 1) >> 3;
-      const int koff = half * (kGvKc / 2) + lane * kGvRun;
+      // consumer warp cw owns row cw / wpr of the tile and the 512-k window
+      // cw % wpr of every stage (wpr = 16 / rows warps per row): 16
+      // consecutive k per lane; the X slice of a stage is shared by all rows
+      // through L1
+      const int kc = kGvElems / p.rows, wpr = kGvConsumers / p.rows;
+      const int row = (warp - 1) / wpr, part = (warp - 1) - row * wpr;
+      const int koff = part * kGvWin + lane * kGvRun;
       float acc[MAXM];
 #pragma unroll
       for (int m = 0; m < MAXM; ++m) acc[m] = 0.f;
-      for (long long k0 = 0; k0 < K; k0 += kGvKc) {
+      for (long long k0 = 0; k0 < K; k0 += kc) {
         gv_wait(&full[stage], ph);
         const long long k = k0 + koff;
         if (row < nr && k < K) {
-          const uint4* ws = reinterpret_cast<const uint4*>(stage_buf + stage * kGvStage + row * (kGvKc * 2) + koff * 2);
+          const uint4* ws = reinterpret_cast<const uint4*>(stage_buf + stage * kGvStage + row * (kc * 2) + koff * 2);
           const uint4 w0 = ws[0], w1 = ws[1];
 #pragma unroll
           for (int m = 0; m < MAXM; ++m)
@@ -277,10 +284,14 @@ bool build_gemv_tma(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std:
   p.act = op.act;
   p.invK = 1.0f / (float)p.K;
   p.warp_rows = (p.K % (32 * kGvRun)) == 0;
-  // rows per tile: as many as possible (<= 8; long streams amortise the
-  // per-tile fold) while keeping >= 2 tiles per SM
-  int rows = kGvMaxRows;
-  while (rows > 1 && (p.N + rows - 1) / rows < 2 * caps.S) rows /= 2;
+  // rows per tile: 4 (measured on B200, profiles/round1/gemv_rows.txt: VGG FC1
+  // 25088->4096 rows 8/4/2/1 = 52.0/40.7/46.8/53.7 us -- 8-row tiles (400 KB)
+  // leave a long tail in the dynamic queue, 1-2-row tiles pay the per-tile
+  // fold too often), fewer when that leaves under one tile per SM
+  int rows = 4;
+  while (rows > 1 && (long long)((p.N + rows - 1) / rows) < caps.S) rows /= 2;
+  if (const char* e = std::getenv("BLESS_GEMV_ROWS")) rows = std::atoi(e);
+  if (rows != 1 && rows != 2 && rows != 4 && rows != 8) rows = kGvMaxRows;
   p.rows = rows;
   const bool m1 = p.M == 1;
   if (!(m1 ? gemv_attr<1>(err) : gemv_attr<8>(err))) return false;

@@ -45,6 +45,7 @@ struct TcParams {
   int OH, OW, BH, BW, tiles_w, C, R_, S_, pad, kc_per_tap;
   // split-K: work unit u -> (tile u / splits, K blocks [ks*kbs, min(num_kb, (ks+1)*kbs)))
   int splits, kbs;
+  int stages;       // smem pipeline depth (runtime: budget / stage bytes, <= kMaxStages)
   float* ws;        // [tiles][128][BN] fp32 partial sums (zero between launches)
   unsigned* sem;    // [tiles] arrival counters (zero between launches)
 };
@@ -196,24 +197,30 @@ __device__ __forceinline__ void epi_store16(const TcParams& p, int m, int n0, fl
   }
 }
 
+constexpr int kMaxStages = 8;
+
 template <int BN, int BK>
 struct TcCfg {
   static constexpr int kStageA = 128 * BK * 2;
   static constexpr int kStageB = BN * BK * 2;
   static constexpr int kStageBytes = kStageA + kStageB;
+  // default pipeline: ~96 KB of stages, so two CTAs (the next kernel's, under
+  // programmatic dependent launch, or another tenant's) fit on one SM
   static constexpr int kStages = std::min(6, (96 * 1024) / kStageBytes);
   // TMEM accumulators: double buffered (epilogue of tile i overlaps the MMAs of
   // tile i+1) up to BN = 128; BN = 256 keeps one so a second co-resident CTA
   // (another tenant's kernel on the same SM) can still allocate.
   static constexpr int kAcc = BN >= 256 ? 1 : 2;
   static constexpr int kTmemCols = (kAcc * BN) < 32 ? 32 : kAcc * BN;
-  static constexpr int kSmem = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/ + 2 * BN * 4 /*sc, sh*/;
+  static constexpr int kFixed = 1024 /*align*/ + 256 /*barriers*/ + 2 * BN * 4 /*sc, sh*/;
+  static constexpr int kSmem = kStages * kStageBytes + kFixed;
+  static constexpr int kSmemMax = kMaxStages * kStageBytes + kFixed;
 };
 
 template <int BN, int BK>
 __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   using Cfg = TcCfg<BN, BK>;
-  constexpr int ST = Cfg::kStages;
+  const int ST = p.stages;
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   unsigned char* smem = (unsigned char*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   unsigned char* sA = smem;
@@ -521,18 +528,27 @@ static cudaError_t launch_tc(const KernelDesc& d, const GateArgs& g, cudaStream_
 }
 
 template <int BN, int BK>
-static bool prep(KernelDesc& d, std::string& err) {
+static bool prep(KernelDesc& d, TcParams& p, std::string& err) {
   static std::once_flag once;
   static cudaError_t attr_err = cudaSuccess;
   std::call_once(once, [] {
     attr_err = cudaFuncSetAttribute((const void*)k_tc_gemm<BN, BK>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    TcCfg<BN, BK>::kSmem);
+                                    std::min(TcCfg<BN, BK>::kSmemMax, 227 * 1024));
   });
   if (attr_err != cudaSuccess) {
     err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(attr_err);
     return false;
   }
-  d.smem = TcCfg<BN, BK>::kSmem;
+  // pipeline depth: BLESS_TC_SMEM_KB overrides the ~96 KB default budget (sweeps)
+  using Cfg = TcCfg<BN, BK>;
+  int st = Cfg::kStages;
+  if (const char* e = std::getenv("BLESS_TC_SMEM_KB")) {
+    const int kb = std::atoi(e);
+    st = std::max(2, std::min(kMaxStages, (kb * 1024 - Cfg::kFixed) / Cfg::kStageBytes));
+    while (st > 2 && st * Cfg::kStageBytes + Cfg::kFixed > 227 * 1024) --st;
+  }
+  p.stages = st;
+  d.smem = st * Cfg::kStageBytes + Cfg::kFixed;
   d.launch = launch_tc<BN, BK>;
   d.kernel_fn = (const void*)k_tc_gemm<BN, BK>;
   return true;
@@ -715,7 +731,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   d.grid = caps.S;
   bool ok = false;
 #define TC_CASE(bn, bk) \
-  if (BN == bn && BK == bk) ok = prep<bn, bk>(d, err);
+  if (BN == bn && BK == bk) ok = prep<bn, bk>(d, p, err);
   TC_CASE(16, 16) TC_CASE(16, 32) TC_CASE(16, 64)
   TC_CASE(32, 16) TC_CASE(32, 32) TC_CASE(32, 64)
   TC_CASE(64, 16) TC_CASE(64, 32) TC_CASE(64, 64)

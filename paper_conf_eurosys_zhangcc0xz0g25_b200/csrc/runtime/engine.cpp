@@ -89,6 +89,14 @@ bl_status Engine::register_tenant(double quota, const char* name, int* out, std:
   return BL_OK;
 }
 
+bl_status Engine::set_slo(int t, int64_t slo_ns, std::string& err) {
+  if (t < 0 || t >= nten() || slo_ns < 0) { err = "bad tenant/slo"; return BL_E_INVALID; }
+  if (started_) { err = "set_slo after bl_start"; return BL_E_STATE; }
+  prof_.ten[t].slo_ns = slo_ns;
+  prof_.derive();
+  return BL_OK;
+}
+
 bl_status Engine::set_stream(int t, void* s, std::string& err) {
   if (t < 0 || t >= nten() || !s) { err = "bad tenant/stream"; return BL_E_INVALID; }
   if (started_) { err = "set_stream after bl_start"; return BL_E_STATE; }
@@ -255,6 +263,7 @@ bl_status Engine::load_profile(const char* path, std::string& err) {
       err = "profile does not match tenant " + std::to_string(j);
       return BL_E_INVALID;
     }
+    if (p.ten[j].slo_ns > 0) prof_.ten[j].slo_ns = p.ten[j].slo_ns;
     for (size_t k = 0; k < p.ten[j].k.size(); ++k) {
       prof_.ten[j].k[k].t = p.ten[j].k[k].t;
       prof_.ten[j].k[k].d = p.ten[j].k[k].d;

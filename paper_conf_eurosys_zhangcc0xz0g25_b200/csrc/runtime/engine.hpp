@@ -60,6 +60,7 @@ class Engine {
   bl_status init(void* ws, size_t ws_bytes, std::string& err);
 
   bl_status register_tenant(double quota, const char* name, int* out, std::string& err);
+  bl_status set_slo(int t, int64_t slo_ns, std::string& err);
   bl_status set_stream(int t, void* s, std::string& err);
   bl_status append_kernel(int t, const bl_op* op, int* out, std::string& err);
   bl_status run_kernel(int t, int k, int lo, int hi, std::string& err);

@@ -48,6 +48,10 @@ void Profile::derive() {
       tn.tau[k] = acc;
     }
     tn.T = acc;
+    tn.tau_prog = tn.tau;
+    if (tn.slo_ns > 0 && tn.T > 0)
+      for (size_t k = 0; k < tn.k.size(); ++k)
+        tn.tau_prog[k] = (int64_t)(((__int128)tn.tau[k] * tn.slo_ns) / tn.T);
   }
 }
 
@@ -76,6 +80,16 @@ bool load_profile_text(const std::string& path, Profile& out, std::string& err) 
     int m = 0;
     f >> a >> tn.name >> tn.quota_ppm >> m;
     if (a != "tenant" || m < 0) { err = "bad tenant line"; return false; }
+    {  // optional "slo <ns>" line (SLO mode, R30)
+      const std::streampos pos = f.tellg();
+      if (f >> a && a == "slo") {
+        f >> tn.slo_ns;
+        if (!f || tn.slo_ns < 0) { err = "bad slo line"; return false; }
+      } else {
+        f.clear();
+        f.seekg(pos);
+      }
+    }
     for (int k = 0; k < m; ++k) {
       KernelProfile kp;
       f >> a >> kp.name >> kp.d;
@@ -98,6 +112,7 @@ bool save_profile_text(const std::string& path, const Profile& p, std::string& e
   f << "bless-profile 1\nS " << p.S << " g " << p.g << "\ntenants " << p.ten.size() << "\n";
   for (auto& tn : p.ten) {
     f << "tenant " << tn.name << " " << tn.quota_ppm << " " << tn.k.size() << "\n";
+    if (tn.slo_ns > 0) f << "slo " << tn.slo_ns << "\n";
     for (auto& k : tn.k) {
       f << "kernel " << k.name << " " << k.d;
       for (int64_t v : k.t) f << " " << v;
@@ -121,7 +136,7 @@ struct Order {
   const Profile* prof;
   int64_t tau(int j) const {
     int n = (*nxt)[j];
-    return n == 0 ? 0 : prof->ten[j].tau[n - 1];
+    return n == 0 ? 0 : prof->ten[j].tau_prog[n - 1];
   }
   bool more_behind(int x, int y) const {
     const int64_t tx = tau(x), ty = tau(y);

@@ -30,6 +30,13 @@ struct TenantProfile {
   int quota_sms = 0;
   std::vector<int64_t> tau;   // tau[k] = sum_{i<=k} t[i][quota_sms] (L157)
   int64_t T = 0;              // isolated latency T[n%] (L157)
+  // SLO mode (§6.5: "replacing the isolated latency T[n%] in §4.3.1
+  // with the required QoS target"): slo_ns > 0 replaces T in P_r = t_e/T, so
+  // P~ = t_e / (tau * slo / T); the progress order compares t_e against
+  // tau_prog[k] = floor(tau[k] * slo_ns / T) (reading R30).  slo_ns = 0:
+  // tau_prog = tau (the paper's default, pace = isolated latency).
+  int64_t slo_ns = 0;
+  std::vector<int64_t> tau_prog;
 };
 
 struct Profile {

@@ -7,6 +7,7 @@ both the C++ runtime ``bl_load_profile`` and the Python oracle)::
     S <S> g <g>
     tenants <n>
     tenant <name> <quota_ppm> <m>
+    slo <ns>                                     (optional: SLO mode target)
     kernel <name> <d> <t_1> <t_2> ... <t_S>      (m lines per tenant)
 
 ``t_s`` is the kernel's duration in integer ns when confined to s SMs
@@ -41,6 +42,7 @@ class TenantRows:
     name: str
     quota_ppm: int
     kernels: List[KernelRow] = field(default_factory=list)
+    slo_ns: int = 0   # optional "slo <ns>" line (SLO mode); 0 = none
 
 
 @dataclass
@@ -54,6 +56,8 @@ def save(path: str, pf: ProfileFile) -> None:
     lines = ["bless-profile 1", f"S {pf.S} g {pf.g}", f"tenants {len(pf.tenants)}"]
     for tn in pf.tenants:
         lines.append(f"tenant {tn.name} {int(tn.quota_ppm)} {len(tn.kernels)}")
+        if tn.slo_ns:
+            lines.append(f"slo {int(tn.slo_ns)}")
         for k in tn.kernels:
             assert len(k.t) == pf.S, (len(k.t), pf.S)
             lines.append("kernel %s %d %s" % (k.name, int(k.d), " ".join(str(int(v)) for v in k.t)))
@@ -73,6 +77,9 @@ def load(path: str) -> ProfileFile:
         _, name, ppm, m = toks[i]
         i += 1
         tn = TenantRows(name, int(ppm))
+        if i < len(toks) and toks[i][0] == "slo":
+            tn.slo_ns = int(toks[i][1])
+            i += 1
         for _ in range(int(m)):
             row = toks[i]
             i += 1

@@ -67,6 +67,20 @@ def test_gemv(ctx, M, N, K, dtype):
     run_and_check(ctx, m, dtype)
 
 
+@pytest.mark.parametrize("rows", ["1", "2", "4", "8"])
+@pytest.mark.parametrize("M,N,K", [(1, 4096, 25088), (1, 1000, 2048), (3, 37, 4112), (8, 129, 96)])
+def test_gemv_forced_rows(ctx, M, N, K, rows, monkeypatch):
+    """Every GEMV tile height (rows of W per tile, stage = rows x 8192/rows k)
+    is exact, including K tails shorter than a stage and N % rows != 0."""
+    monkeypatch.setenv("BLESS_GEMV_ROWS", rows)
+
+    def mk(b):
+        b.gemm(b.input((M, K)), N, act="none", bias=True)
+    m = one_layer(ctx, "bf16", mk)
+    assert ctx.kernel_info(m.tenant, 0).family.decode() == "gemv_tma_bf16"
+    run_and_check(ctx, m, "bf16")
+
+
 CONVS = [  # H, W, C, K, k, stride, pad, act, residual
     (56, 56, 64, 64, 3, 1, 1, "relu", False),
     (56, 56, 64, 256, 1, 1, 0, "relu", True),
