@@ -70,6 +70,7 @@ def parse():
     ap.add_argument("--profile-reps", type=int, default=5)
     ap.add_argument("--no-baselines", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-slo", action="store_true", help="skip the SLO-mode experiment (§6.5)")
     ap.add_argument("--load-profile", default="", help="reuse a saved profile table instead of profiling")
     ap.add_argument("--light", action="store_true", help="timed steps only (for ncu launch lists)")
     ap.add_argument("--out-dir", default=os.path.join(ROOT, "gpurun_out"))
@@ -329,26 +330,39 @@ def native(args):
         ctx.close()
         return
 
-    # ---------------- in-run baselines on the seed-1 trace
+    # ---------------- in-run baselines on the SAME traces as the timed steps
+    # (each distinct seed once, weighted by how often the timed steps used it),
+    # so attainment and the BLESS-vs-baseline ratios compare like with like
     per_tenant = {}
     base = {}
     iso_means = {}
+    seeds = [1 + k % 3 for k in range(args.steps)]
+    mult = {sd: seeds.count(sd) for sd in sorted(set(seeds))}
+
+    def run_seeds(pol, filt=None, extra=None):
+        out = {}
+        for sd, n in mult.items():
+            l, *_ = step(sd, pol, filt, extra)
+            for j, v in l.items():
+                out.setdefault(j, []).extend(v * n)
+        return out
+
     if not args.no_baselines:
         iso = {}
         for j in range(len(tms)):
-            l, *_ = step(1, "ISO", {j})
-            iso[j] = l[j]
-            iso_means[j] = float(np.mean(l[j]))
+            iso[j] = run_seeds("ISO", {j})[j]
+            iso_means[j] = float(np.mean(iso[j]))
         base["ISO"] = {names[j]: stats(iso[j]) for j in iso}
+        base["ISO"]["all_mean_ms"] = float(np.mean([x for v in iso.values() for x in v])) / 1e6
         runs = {"STATIC": ("STATIC", {}), "TEMPORAL_Tcap": ("TEMPORAL", {}),
                 "TEMPORAL_Twc": ("TEMPORAL", {"temporal_work_conserving": 1}), "UNBOUND": ("UNBOUND", {})}
+        base_lat = {}
         for label, (pol, extra) in runs.items():
-            l, *_ = step(1, pol, None, extra)
+            l = run_seeds(pol, None, extra)
+            base_lat[label] = l
             base[label] = {names[j]: stats(v) for j, v in l.items()}
             base[label]["all_mean_ms"] = float(np.mean([x for v in l.values() for x in v])) / 1e6
-        lb1, *_ = step(1)
-        base["BLESS_seed1"] = {names[j]: stats(v) for j, v in lb1.items()}
-        base["BLESS_seed1"]["all_mean_ms"] = float(np.mean([x for v in lb1.values() for x in v])) / 1e6
+        base["seeds"] = mult
     for j in range(len(tms)):
         s = stats(lat_all[j])
         if iso_means:
@@ -356,6 +370,29 @@ def native(args):
         s["quota_sms"] = quota_sms[j]
         s["T_iso_profile_ms"] = T_iso[j] / 1e6
         per_tenant[names[j]] = s
+
+    # ---------------- SLO mode (§6.5): QoS target replaces T[n%] in
+    # the progress order; violation rate = share of requests over the target,
+    # for BLESS with the targets, default BLESS, and the baselines (same traces)
+    slo = None
+    if not args.no_baselines and not args.no_slo:
+        slo = {}
+        for label, fac in (("tight", (1.2, 2.0)), ("loose", (1.5, 3.0))):
+            tgt = [int(fac[j % 2] * T_iso[j]) for j in range(len(tms))]
+            for m, q in zip(tms, tgt):
+                ctx.set_slo(m.tenant, q)
+            ls = run_seeds("BLESS")
+            for m in tms:
+                ctx.set_slo(m.tenant, 0)
+
+            def viol(l):
+                n = sum(len(v) for v in l.values())
+                return 100.0 * sum(sum(1 for x in v if x > tgt[j]) for j, v in l.items()) / max(1, n)
+            row = {"targets_ms": {names[j]: tgt[j] / 1e6 for j in range(len(tms))},
+                   "factors_x_T_iso": list(fac), "violation_pct": {"BLESS_SLO": viol(ls), "BLESS": viol(lat_all)}}
+            row["violation_pct"].update({k: viol(v) for k, v in base_lat.items()})
+            row["BLESS_SLO_mean_ms"] = {names[j]: float(np.mean(v)) / 1e6 for j, v in ls.items()}
+            slo[label] = row
 
     # ---------------- e2e: same metric with host buffers (H2D input, D2H output per request)
     e2e = None
@@ -421,8 +458,19 @@ def native(args):
     else:
         bound, unit, achieved, peak = "hbm", "GB/s", B / T, hbm_peak
     per_layer.sort(reverse=True)
+    # traffic: ncu dram bytes per launch of the same layers (committed capture,
+    # tools/traffic.py: each kernel alone on all SMs, cold L2), launch-weighted
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
+    if os.path.exists(tpath):
+        tl = json.load(open(tpath))["layers"]
+        keys = [(tk, f"{names[tk[0]]}[{tk[1]}]") for tk in busy if fam_of[tk] == fam]
+        if all(k in tl and tl[k]["dram_read"] is not None for _, k in keys):
+            nl = sum(nlaunch[tk] for tk, _ in keys)
+            traffic = sum(nlaunch[tk] * (tl[k]["dram_read"] + tl[k]["dram_write"]) for tk, k in keys) / max(1, nl)
     roofline = {"bound": bound, "achieved": achieved, "peak": peak, "unit": unit, "frac": achieved / peak,
-                "traffic": None, "kernel": fam, "layers": len(per_layer),
+                "traffic": traffic, "traffic_source": f"profiles/traffic_{args.config}.json" if traffic else None,
+                "kernel": fam, "layers": len(per_layer),
                 "algorithmic_flops_per_launch": F / max(1, sum(nlaunch[tk] for tk in busy if fam_of[tk] == fam)),
                 "algorithmic_bytes_per_launch": B / max(1, sum(nlaunch[tk] for tk in busy if fam_of[tk] == fam)),
                 "event_avg_ns_per_launch": T / max(1, sum(nlaunch[tk] for tk in busy if fam_of[tk] == fam)),
@@ -440,6 +488,10 @@ def native(args):
                                   "achieved": ki.bytes / ev, "peak": hbm_peak, "unit": "GB/s",
                                   "frac": ki.bytes / ev / hbm_peak, "algorithmic_bytes": ki.bytes,
                                   "event_ns": ev}
+        if os.path.exists(tpath):
+            rec = json.load(open(tpath))["layers"].get(f"{names[tk[0]]}[{tk[1]}]")
+            if rec and rec["dram_read"] is not None:
+                roofline["hbm_kernel"]["traffic"] = rec["dram_read"] + rec["dram_write"]
 
     # SM-share roofline per tenant: sum t_roof / sum t_meas over BLESS launches
     kinfo = {(m.tenant, k): ctx.kernel_info(m.tenant, k) for m in tms for k in range(len(m.layers))}
@@ -488,9 +540,9 @@ def native(args):
         "config": {"workload": f"{args.config}: {CONFIG_NAMES[args.config]}",
                    "trace": f"{'MMPP-2 bursty' if args.config == 'C4' else 'Poisson'} rho={args.rho} "
                    f"per tenant, {args.requests} requests/tenant/step, seeds 1-3", "squad_max": args.squad_max,
-                   "parallelism": f"replicas x{world} (no collective)",
+                   "split_pct": args.split_pct, "parallelism": f"replicas x{world} (no collective)",
                    "l2": "256 MiB buffer written between timed steps (> 126 MB L2); VGG11 weights 266 MB > L2"},
-        "per_tenant": per_tenant, "baselines": base, "requests_per_s": n_req / (step_ms * args.steps / 1e3),
+        "per_tenant": per_tenant, "baselines": base, "slo": slo, "requests_per_s": n_req / (step_ms * args.steps / 1e3),
         "e2e": e2e, "gpu_launches": gpu_launches, "roofline": roofline, "cpu_baseline": cpu,
         "clocks": clk.summary(),
         "scheduler": {"decisions": len(decisions_all), "sp_squads": sp_squads, "fallback_launches": fallbacks,

@@ -86,6 +86,10 @@ class Prof:
         # P_r = t_e / SLO and P_e = tau / T, so P~ = t_e / (tau * SLO / T);
         # reading R30 floors tau * SLO / T to integer ns.  No SLO: tau itself.
         self.slo = [int(getattr(tn, "slo_ns", 0)) for tn in pf.tenants]
+        # memory-management kernels: per-request H2D before
+        # kernel 0 and D2H after the last kernel, copy-engine ns
+        self.io_in = [int(getattr(tn, "io_in", 0)) for tn in pf.tenants]
+        self.io_out = [int(getattr(tn, "io_out", 0)) for tn in pf.tenants]
         self.tau_prog: List[List[int]] = []
         for j in range(self.ntenants):
             if self.slo[j] > 0 and self.T[j] > 0:
@@ -96,6 +100,12 @@ class Prof:
     def t(self, j: int, k: int, s: int) -> int:
         assert 1 <= s <= self.S, s
         return self._t[j][k][s - 1]
+
+    def io(self, j: int, k: int) -> int:
+        """L229: "the durations of memory management kernels (e.g., H2D, D2H
+        memcpy) are added" in both predictors.  Reading R31: the request's
+        input copy belongs to its kernel 0, its output copy to its last kernel."""
+        return (self.io_in[j] if k == 0 else 0) + (self.io_out[j] if k == self.m[j] - 1 else 0)
 
 
 @dataclass
@@ -224,6 +234,7 @@ def predict_nsp(ks: Dict[int, List[int]], prof: Prof) -> Tuple[int, List[int]]:
                 level += prof.t(j, k, x)
             else:
                 level += (prof.t(j, k, dk) * dk) // x
+            level += prof.io(j, k)                      # L229, R31
         total += level
         ends.append(total)
     return total, ends
@@ -244,7 +255,7 @@ def predict_sp(ks: Dict[int, List[int]], p: Sequence[int], prof: Prof) -> Tuple[
     chains = {}
     for idx, j in enumerate(parts):
         s = sp_sms(p, idx, prof)
-        chains[j] = sum(prof.t(j, k, s) for k in ks[j])
+        chains[j] = sum(prof.t(j, k, s) + prof.io(j, k) for k in ks[j])   # L229, R31
     return max(chains.values()), chains
 
 
@@ -277,7 +288,7 @@ def choose_config(ks: Dict[int, List[int]], prof: Prof) -> Tuple[Optional[Tuple[
 
         def chain(j: int, s: int) -> int:
             if (j, s) not in memo:
-                memo[(j, s)] = sum(prof.t(j, k, s) for k in ks[j])
+                memo[(j, s)] = sum(prof.t(j, k, s) + prof.io(j, k) for k in ks[j])
             return memo[(j, s)]
 
         for p in compositions(prof.N, K):

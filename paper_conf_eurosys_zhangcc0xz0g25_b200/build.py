@@ -50,7 +50,8 @@ def _obj_path(src):
 def _compile(src, verbose):
     out = _obj_path(src)
     if src.endswith(".cu"):
-        cmd = [NVCC] + NVFLAGS + INC + ["-c", src, "-o", out]
+        extra = os.environ.get("BLESS_EXTRA_NVFLAGS", "").split()   # debug builds (e.g. -DBLESS_TC_TRACE)
+        cmd = [NVCC] + NVFLAGS + extra + INC + ["-c", src, "-o", out]
     else:
         cmd = ["g++"] + CXXFLAGS + INC + ["-c", src, "-o", out]
     r = subprocess.run(cmd, capture_output=True, text=True)

@@ -54,6 +54,21 @@ struct TcParams {
 // ------------------------------------------------------------------ PTX helpers
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
+// Debug builds only (-DBLESS_TC_TRACE, tools/tctrace.py): per-CTA %globaltimer
+// stamps of the pipeline phases of the last launch.
+#ifdef BLESS_TC_TRACE
+constexpr int kTrMax = 2048, kTrN = 10;
+__device__ unsigned long long g_tc_trace[kTrMax][kTrN];
+__device__ __forceinline__ void tr_mark(int i) {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  if (blockIdx.x < kTrMax) g_tc_trace[blockIdx.x][i] = t;
+}
+#define TR(i) tr_mark(i)
+#else
+#define TR(i) ((void)0)
+#endif
+
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
 }
@@ -198,6 +213,7 @@ __device__ __forceinline__ void epi_store16(const TcParams& p, int m, int n0, fl
 }
 
 constexpr int kMaxStages = 8;
+constexpr int kDynSmemMax = 227 * 1024 - 2048;   // opt-in limit minus the executor's static smem
 
 template <int BN, int BK>
 struct TcCfg {
@@ -239,6 +255,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   float* epi_sh = epi_sc + BN;                                    // [BN] tile shift
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) TR(1);   // 1: work entry
   if (threadIdx.x == 0) {
     for (int i = 0; i < ST; ++i) {
       mbar_init(&full[i], 1);
@@ -262,6 +279,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  if (threadIdx.x == 0) TR(2);   // 2: barriers + TMEM ready
   // No grid-wide griddepcontrol.wait here: under programmatic dependent launch
   // the setup above, the first tile claim, the weight (B) loads and the
   // epilogue constants overlap the previous kernel; only reads of activations
@@ -280,6 +298,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       uint32_t rph = 0;
       for (;;) {
         const int t = gate_claim(g, marked);
+        if (!dep_waited) TR(3);          // 3: first claim returned
         mbar_wait(&rempty[rs], rph ^ 1);
         ring[rs] = t;
         mbar_arrive(&rfull[rs]);
@@ -335,6 +354,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
             load_B(kb0 + i, st);
           }
           pdl_wait();
+          TR(4);                         // 4: producer past griddepcontrol.wait
           dep_waited = true;
           for (int i = 0; i < npre; ++i) load_A(kb0 + i, (stage + i) % ST);
           for (int i = 0; i < npre; ++i)
@@ -374,6 +394,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       for (int kb = kb0; kb < kb1; ++kb) {
         mbar_wait(&full[stage], phase);
         tc_fence_after();
+        if (lane == 0 && kb == kb0) TR(5);   // 5: first stage landed (last tile of this CTA)
         if (lane == 0) {
           const uint32_t a0 = smem_u32(sA + stage * Cfg::kStageA);
           const uint32_t b0 = smem_u32(sB + stage * Cfg::kStageB);
@@ -438,6 +459,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       }
       mbar_wait(&tfull[acc], aph);
       tc_fence_after();
+      if (threadIdx.x == 64) TR(6);      // 6: accumulator ready (last tile)
       const uint32_t tbase = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN;
       if (p.splits == 1) {
 #pragma unroll 1
@@ -455,6 +477,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty[acc]);
+        if (threadIdx.x == 64) TR(7);    // 7: epilogue stores issued (last tile)
       } else {
         // split-K: add this unit's partial tile into the fp32 workspace
         float* wrow = p.ws + ((size_t)tile * 128 + row) * BN;
@@ -511,12 +534,15 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
 
 template <int BN, int BK>
 __global__ void __launch_bounds__(192, 1) k_tc_gemm(const __grid_constant__ TcParams p, const GateArgs g) {
+  if (threadIdx.x == 0) TR(0);   // 0: CTA start
   if (gate_in_range(g) || gate_linger(g)) tc_work<BN, BK>(p, g);
   pdl_trigger();
+  if (threadIdx.x == 0) TR(8);   // 8: work done, before the exit atomic
   int last = 0;
   const bool fb = gate_leave(g, last);
   if (fb) tc_work<BN, BK>(p, g);
   if (last) gate_finalize(g, fb);
+  if (threadIdx.x == 0) TR(9);   // 9: CTA exit
 }
 #endif  // __CUDACC__
 
@@ -533,7 +559,7 @@ static bool prep(KernelDesc& d, TcParams& p, std::string& err) {
   static cudaError_t attr_err = cudaSuccess;
   std::call_once(once, [] {
     attr_err = cudaFuncSetAttribute((const void*)k_tc_gemm<BN, BK>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    std::min(TcCfg<BN, BK>::kSmemMax, 227 * 1024));
+                                    std::min(TcCfg<BN, BK>::kSmemMax, kDynSmemMax));
   });
   if (attr_err != cudaSuccess) {
     err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(attr_err);
@@ -545,7 +571,7 @@ static bool prep(KernelDesc& d, TcParams& p, std::string& err) {
   if (const char* e = std::getenv("BLESS_TC_SMEM_KB")) {
     const int kb = std::atoi(e);
     st = std::max(2, std::min(kMaxStages, (kb * 1024 - Cfg::kFixed) / Cfg::kStageBytes));
-    while (st > 2 && st * Cfg::kStageBytes + Cfg::kFixed > 227 * 1024) --st;
+    while (st > 2 && st * Cfg::kStageBytes + Cfg::kFixed > kDynSmemMax) --st;
   }
   p.stages = st;
   d.smem = st * Cfg::kStageBytes + Cfg::kFixed;
@@ -792,3 +818,15 @@ int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int ma
 }
 
 }  // namespace bless
+
+#ifdef BLESS_TC_TRACE
+// debug builds only: copy the per-CTA phase stamps out (tools/tctrace.py)
+extern "C" int bl_debug_tc_trace(unsigned long long* host, int n_cta) {
+  const size_t n = (size_t)std::min(n_cta, bless::kTrMax) * bless::kTrN * sizeof(unsigned long long);
+  return (int)cudaMemcpyFromSymbol(host, bless::g_tc_trace, n);
+}
+extern "C" int bl_debug_tc_trace_clear() {
+  static unsigned long long z[bless::kTrMax][bless::kTrN];
+  return (int)cudaMemcpyToSymbol(bless::g_tc_trace, z, sizeof(z));
+}
+#endif

@@ -5,6 +5,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <vector>
 #include <atomic>
 #include <chrono>
 #include <cstring>
@@ -448,6 +449,26 @@ bool DeviceRT::overhead(int variant, int reps, int64_t* ns_out, std::string& err
   cudaEventDestroy(e0);
   cudaEventDestroy(e1);
   cudaStreamDestroy(s);
+  return true;
+}
+
+bool DeviceRT::time_copy(void* dst, const void* src, size_t n, int reps, void* stream, int64_t* ns) {
+  cudaStream_t st = (cudaStream_t)stream;
+  cudaEvent_t a, b;
+  if (cudaEventCreate(&a) != cudaSuccess || cudaEventCreate(&b) != cudaSuccess) return false;
+  std::vector<float> ms;
+  bool ok = true;
+  for (int i = 0; i < reps + 1 && ok; ++i) {   // first copy is a warm-up
+    ok = cudaEventRecord(a, st) == cudaSuccess && cudaMemcpyAsync(dst, src, n, cudaMemcpyDefault, st) == cudaSuccess &&
+         cudaEventRecord(b, st) == cudaSuccess && cudaEventSynchronize(b) == cudaSuccess;
+    float x = 0.f;
+    if (ok && i > 0 && cudaEventElapsedTime(&x, a, b) == cudaSuccess) ms.push_back(x);
+  }
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  if (!ok || ms.empty()) return false;
+  std::sort(ms.begin(), ms.end());
+  *ns = (int64_t)(ms[ms.size() / 2] * 1e6);
   return true;
 }
 

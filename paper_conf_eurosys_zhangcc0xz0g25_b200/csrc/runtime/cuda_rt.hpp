@@ -37,6 +37,8 @@ class DeviceRT {
   // One-CTA completion marker (stats only, no work) on stream; returns seq or 0.
   uint64_t launch_marker(void* stream, std::string& err);
   bool memcpy_async(void* dst, const void* src, size_t n, void* stream);
+  // median duration (ns, CUDA events) of reps copies of n bytes on stream
+  bool time_copy(void* dst, const void* src, size_t n, int reps, void* stream, int64_t* ns);
   // Diagnostics: per-launch time of back-to-back S-CTA launches.  variant 0:
   // empty kernel; 1: gate + tile queue + exit protocol; 2: 1 + host-mapped stamps.
   bool overhead(int variant, int reps, int64_t* ns_out, std::string& err);

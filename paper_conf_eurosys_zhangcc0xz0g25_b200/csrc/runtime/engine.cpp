@@ -154,6 +154,13 @@ bl_status Engine::set_io(int t, const void* hin, void* din, size_t inb, const vo
   tr.dev_out = dout;
   tr.host_out = hout;
   tr.out_bytes = outb;
+  // profile the memory-management kernels for the predictors (L229, R31)
+  rt_->set_device();
+  TenantProfile& tp = prof_.ten[t];
+  tp.io_in = tp.io_out = 0;
+  if (inb && !rt_->time_copy(din, hin, inb, 5, tr.stream, &tp.io_in)) { err = "H2D copy failed"; return BL_E_CUDA; }
+  if (outb && !rt_->time_copy(hout, dout, outb, 5, tr.stream, &tp.io_out)) { err = "D2H copy failed"; return BL_E_CUDA; }
+  prof_.derive();
   return BL_OK;
 }
 
@@ -264,6 +271,10 @@ bl_status Engine::load_profile(const char* path, std::string& err) {
       return BL_E_INVALID;
     }
     if (p.ten[j].slo_ns > 0) prof_.ten[j].slo_ns = p.ten[j].slo_ns;
+    if (p.ten[j].io_in > 0 || p.ten[j].io_out > 0) {
+      prof_.ten[j].io_in = p.ten[j].io_in;
+      prof_.ten[j].io_out = p.ten[j].io_out;
+    }
     for (size_t k = 0; k < p.ten[j].k.size(); ++k) {
       prof_.ten[j].k[k].t = p.ten[j].k[k].t;
       prof_.ten[j].k[k].d = p.ten[j].k[k].d;

@@ -80,14 +80,18 @@ bool load_profile_text(const std::string& path, Profile& out, std::string& err) 
     int m = 0;
     f >> a >> tn.name >> tn.quota_ppm >> m;
     if (a != "tenant" || m < 0) { err = "bad tenant line"; return false; }
-    {  // optional "slo <ns>" line (SLO mode, R30)
+    for (;;) {  // optional "slo <ns>" (SLO mode, R30) and "io <in_ns> <out_ns>" (R31) lines
       const std::streampos pos = f.tellg();
-      if (f >> a && a == "slo") {
+      if (!(f >> a)) { f.clear(); f.seekg(pos); break; }
+      if (a == "slo") {
         f >> tn.slo_ns;
         if (!f || tn.slo_ns < 0) { err = "bad slo line"; return false; }
+      } else if (a == "io") {
+        f >> tn.io_in >> tn.io_out;
+        if (!f || tn.io_in < 0 || tn.io_out < 0) { err = "bad io line"; return false; }
       } else {
-        f.clear();
         f.seekg(pos);
+        break;
       }
     }
     for (int k = 0; k < m; ++k) {
@@ -113,6 +117,7 @@ bool save_profile_text(const std::string& path, const Profile& p, std::string& e
   for (auto& tn : p.ten) {
     f << "tenant " << tn.name << " " << tn.quota_ppm << " " << tn.k.size() << "\n";
     if (tn.slo_ns > 0) f << "slo " << tn.slo_ns << "\n";
+    if (tn.io_in > 0 || tn.io_out > 0) f << "io " << tn.io_in << " " << tn.io_out << "\n";
     for (auto& k : tn.k) {
       f << "kernel " << k.name << " " << k.d;
       for (int64_t v : k.t) f << " " << v;
@@ -129,6 +134,12 @@ bool save_profile_text(const std::string& path, const Profile& p, std::string& e
 //   arrival; smaller tenant id (R4).  This is a total order.
 // ---------------------------------------------------------------------------
 namespace {
+// Memory-management kernel time attached to kernel k of tenant j (R31).
+inline int64_t io_of(const Profile& prof, int j, int k) {
+  const TenantProfile& tn = prof.ten[j];
+  return (k == 0 ? tn.io_in : 0) + (k == (int)tn.k.size() - 1 ? tn.io_out : 0);
+}
+
 struct Order {
   int64_t now;
   const std::vector<int>* nxt;
@@ -228,6 +239,7 @@ void decide(int64_t now, const ActiveReq* act, int n_act, const Profile& prof, c
       const int dk = prof.ten[j].k[k].d;
       if (x <= dk) level += prof.t(j, k, (int)x);
       else level += (prof.t(j, k, dk) * dk) / x;
+      level += io_of(prof, j, k);   // R31
     }
     t_nsp += level;
     level_end[lv] = t_nsp;
@@ -247,7 +259,7 @@ void decide(int64_t now, const ActiveReq* act, int n_act, const Profile& prof, c
       for (int p = 1; p <= N; ++p) {
         const int s = (i < K - 1) ? g * p : S - g * (N - p);
         int64_t sum = 0;
-        for (int k : sc.ks[i]) sum += prof.t(j, k, s);
+        for (int k : sc.ks[i]) sum += prof.t(j, k, s) + io_of(prof, j, k);   // R31
         sc.Sj[(size_t)i * W + p] = sum;
       }
     }

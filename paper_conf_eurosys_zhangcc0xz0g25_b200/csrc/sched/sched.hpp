@@ -37,6 +37,14 @@ struct TenantProfile {
   // tau_prog = tau (the paper's default, pace = isolated latency).
   int64_t slo_ns = 0;
   std::vector<int64_t> tau_prog;
+  // Memory-management kernels (L229: "the durations of memory management
+  // kernels (e.g., H2D, D2H memcpy) are added" in both predictors): the
+  // request's input copy before kernel 0 and output copy after its last
+  // kernel, profiled on the copy engine (ns, independent of the SM count).
+  // Reading R31: Eq. 1 adds io_in / io_out to a participant's chain when its
+  // picks include kernel 0 / the last kernel; Eq. 2 adds them to the level of
+  // that kernel.  0 = no per-request host I/O.
+  int64_t io_in = 0, io_out = 0;
 };
 
 struct Profile {

@@ -8,6 +8,7 @@ both the C++ runtime ``bl_load_profile`` and the Python oracle)::
     tenants <n>
     tenant <name> <quota_ppm> <m>
     slo <ns>                                     (optional: SLO mode target)
+    io <in_ns> <out_ns>                          (optional: per-request H2D / D2H copy time)
     kernel <name> <d> <t_1> <t_2> ... <t_S>      (m lines per tenant)
 
 ``t_s`` is the kernel's duration in integer ns when confined to s SMs
@@ -43,6 +44,8 @@ class TenantRows:
     quota_ppm: int
     kernels: List[KernelRow] = field(default_factory=list)
     slo_ns: int = 0   # optional "slo <ns>" line (SLO mode); 0 = none
+    io_in: int = 0    # optional "io <in_ns> <out_ns>" line: per-request H2D / D2H copy durations
+    io_out: int = 0
 
 
 @dataclass
@@ -58,6 +61,8 @@ def save(path: str, pf: ProfileFile) -> None:
         lines.append(f"tenant {tn.name} {int(tn.quota_ppm)} {len(tn.kernels)}")
         if tn.slo_ns:
             lines.append(f"slo {int(tn.slo_ns)}")
+        if tn.io_in or tn.io_out:
+            lines.append(f"io {int(tn.io_in)} {int(tn.io_out)}")
         for k in tn.kernels:
             assert len(k.t) == pf.S, (len(k.t), pf.S)
             lines.append("kernel %s %d %s" % (k.name, int(k.d), " ".join(str(int(v)) for v in k.t)))
@@ -77,8 +82,11 @@ def load(path: str) -> ProfileFile:
         _, name, ppm, m = toks[i]
         i += 1
         tn = TenantRows(name, int(ppm))
-        if i < len(toks) and toks[i][0] == "slo":
-            tn.slo_ns = int(toks[i][1])
+        while i < len(toks) and toks[i][0] in ("slo", "io"):
+            if toks[i][0] == "slo":
+                tn.slo_ns = int(toks[i][1])
+            else:
+                tn.io_in, tn.io_out = int(toks[i][1]), int(toks[i][2])
             i += 1
         for _ in range(int(m)):
             row = toks[i]

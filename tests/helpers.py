@@ -23,5 +23,6 @@ def golden_profile(fx) -> ProfileFile:
         else:
             for i in range(tn["m"]):
                 rows.append(KernelRow(f"{tn['name']}{i}", tn["d"], [tn["t_const"]] * S))
-        tenants.append(TenantRows(tn["name"], tn["quota_ppm"], rows, tn.get("slo_ns", 0)))
+        tenants.append(TenantRows(tn["name"], tn["quota_ppm"], rows, tn.get("slo_ns", 0), tn.get("io_in", 0),
+                                  tn.get("io_out", 0)))
     return ProfileFile(S, fx["g"], tenants)

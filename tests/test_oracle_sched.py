@@ -22,7 +22,7 @@ from tests.helpers import golden_profile, load_golden
 
 
 # --------------------------------------------------------------------------- golden E1/E2/E3
-@pytest.mark.parametrize("name", ["e1_nsp_wins.json", "e2_sp_wins.json"])
+@pytest.mark.parametrize("name", ["e1_nsp_wins.json", "e2_sp_wins.json", "e5_memory_kernels.json"])
 def test_predictors_golden(name):
     fx = load_golden(name)
     prof = Prof(golden_profile(fx))

@@ -1,0 +1,67 @@
+"""Phase timeline of the tcgen05 GEMM/conv kernel (debug build with
+-DBLESS_TC_TRACE): per-CTA %globaltimer stamps of the last of R back-to-back
+launches (programmatic dependent launch on, as in the engine).
+
+  BLESS_EXTRA_NVFLAGS=-DBLESS_TC_TRACE python tools/tctrace.py gemm 384 4096 1024
+  BLESS_EXTRA_NVFLAGS=-DBLESS_TC_TRACE python tools/tctrace.py conv 14 14 1024 256 1 1 0
+
+Phases: 0 CTA start, 1 work entry (in range), 2 barriers+TMEM ready, 3 first
+claim returned, 4 producer past griddepcontrol.wait, 5 first stage landed
+(MMA thread), 6 accumulator ready (epilogue), 7 epilogue stores issued,
+8 work done, 9 CTA exit.  Rebuilds the library with the flag (force).
+"""
+import ctypes as C
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+NAMES = ["start", "entry", "setup", "claim", "pdl_wait", "stage0", "acc_ready", "epi_done", "work_done", "exit"]
+
+
+def main():
+    assert "BLESS_TC_TRACE" in os.environ.get("BLESS_EXTRA_NVFLAGS", ""), "set BLESS_EXTRA_NVFLAGS=-DBLESS_TC_TRACE"
+    from paper_conf_eurosys_zhangcc0xz0g25_b200 import build, capi
+    from paper_conf_eurosys_zhangcc0xz0g25_b200.models import Builder
+    build.build(force=True, verbose=False)
+    kind, d = sys.argv[1], [int(x) for x in sys.argv[2:]]
+    ctx = capi.Ctx(0)
+    S = ctx.device_info().sm_count
+    t = ctx.register_tenant(1.0, "k")
+    b = Builder(ctx, t, "k", 1.0, "bf16", seed=7)
+    if kind == "gemm":
+        b.gemm(b.input((d[0], d[2])), d[1], act="gelu", bias=True)
+    else:
+        H, W, Cc, K, k, s, p = d
+        b.conv(b.input((1, H, W, Cc)), K, k, s, p, act="relu", bn=True)
+    ki = ctx.kernel_info(t, 0)
+    L = capi.lib()
+    L.bl_debug_tc_trace.argtypes = [C.c_void_p, C.c_int]
+    for reps in (1, 20):
+        L.bl_debug_tc_trace_clear()
+        ns, _ = ctx.profile_kernel(t, 0, S, reps)
+        buf = np.zeros((2048, 10), dtype=np.uint64)
+        L.bl_debug_tc_trace(buf.ctypes.data, 2048)
+        v = buf.astype(np.int64)
+        ok = (v[:, 0] > 0) & (v[:, 1] >= v[:, 0]) & (v[:, 9] >= v[:, 1]) & (v[:, 7] > 0)
+        w = v[ok]
+        t0 = int(v[v[:, 0] > 0, 0].min())
+        print(f"{kind} {d} {ki.family.decode()} tiles={ki.tiles} reps={reps}: event avg {ns / 1e3:.2f} us, "
+              f"{ok.sum()} working CTAs")
+        if not len(w):
+            continue
+        print("  phase       min(us)  med(us)  max(us)   (relative to the first CTA start of the last launch)")
+        for i, nm in enumerate(NAMES):
+            col = w[:, i]
+            col = col[col > 0] - t0
+            if len(col):
+                print(f"  {i} {nm:10s} {col.min() / 1e3:8.2f} {np.median(col) / 1e3:8.2f} {col.max() / 1e3:8.2f}")
+        allx = v[v[:, 9] > 0, 9] - t0
+        print(f"  last CTA exit (all CTAs) {allx.max() / 1e3:.2f} us")
+    ctx.close()
+
+
+if __name__ == "__main__":
+    main()
