@@ -311,7 +311,10 @@ bl_status bl_decide(bl_ctx* ctx, int64_t now, int n_active, const int32_t* tenan
 
 /* Diagnostics: mean per-launch device time of 'reps' back-to-back S-CTA
  * launches of an executor skeleton (variant 0: empty kernel, 1: SM gate + tile
- * queue + exit protocol, 2: 1 + host-mapped completion stamps). */
+ * queue + exit protocol, 2: 1 + device completion stamps, 3: 2 with
+ * programmatic dependent launch).  variant | 4 (4..7) returns instead the
+ * mean HOST time per launch call of the same loop (enqueue cost, ns).
+ * BL_E_INVALID for variant outside 0..7 or reps < 1. */
 bl_status bl_debug_overhead(bl_ctx* ctx, int variant, int reps, int64_t* ns_out);
 
 int64_t bl_now_ns(void);

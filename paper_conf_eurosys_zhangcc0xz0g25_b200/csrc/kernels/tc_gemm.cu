@@ -11,7 +11,7 @@
 // uses a rank-5 "parity" view of the input, (c, w%2, w/2, h%2, h/2), so every
 // tap is again a dense box.  B is the KRSC weight matrix [Kout, R*S*C].
 //
-// Warp roles (192 threads): warp 0 = tile scheduler + TMA producer, warp 1 =
+// Warp roles (320 threads): warp 0 = tile scheduler + TMA producer, warp 1 =
 // MMA issuer (one thread) and TMEM owner, warps 2-5 = epilogue (TMEM -> regs ->
 // fused epilogue -> global).  Tiles come from the executor's per-launch atomic
 // queue; the TMEM accumulator is double buffered so the epilogue of tile i
@@ -163,19 +163,21 @@ __device__ __forceinline__ uint32_t instr_desc() {
   return d;
 }
 
-__device__ __forceinline__ float act_f(float y, int act) {
-  switch (act) {
-    case BL_ACT_RELU: return fmaxf(y, 0.f);
-    case BL_ACT_RELU6: return fminf(fmaxf(y, 0.f), 6.f);
-    case BL_ACT_GELU: return 0.5f * y * (1.f + erff(y * 0.70710678118654752f));
-    default: return y;
-  }
+// Activation, resolved at compile time (the epilogue is instantiated per
+// activation: a per-element switch serialised the 16-wide chunk).
+template <int ACT>
+__device__ __forceinline__ float act_t(float y) {
+  if (ACT == BL_ACT_RELU) return fmaxf(y, 0.f);
+  if (ACT == BL_ACT_RELU6) return fminf(fmaxf(y, 0.f), 6.f);
+  if (ACT == BL_ACT_GELU) return 0.5f * y * (1.f + erff(y * 0.70710678118654752f));
+  return y;
 }
 
 // Fused epilogue for 16 consecutive columns of one output row:
 // y = act(acc * scale + shift + R), rounded to bf16 (RNE), vector stores.
 // sc/sh: the tile's per-column scale/shift staged in shared memory (1 / 0
 // where absent), indexed from this 16-column chunk.
+template <int ACT>
 __device__ __forceinline__ void epi_store16(const TcParams& p, int m, int n0, float (&y)[16], const float* sc,
                                             const float* sh) {
   const bool full16 = n0 + 16 <= p.N;
@@ -203,15 +205,62 @@ __device__ __forceinline__ void epi_store16(const TcParams& p, int m, int n0, fl
     uint4 o[2];
     __nv_bfloat162* ob = reinterpret_cast<__nv_bfloat162*>(o);
 #pragma unroll
-    for (int i = 0; i < 8; ++i) ob[i] = __floats2bfloat162_rn(act_f(y[2 * i], p.act), act_f(y[2 * i + 1], p.act));
+    for (int i = 0; i < 8; ++i) ob[i] = __floats2bfloat162_rn(act_t<ACT>(y[2 * i]), act_t<ACT>(y[2 * i + 1]));
     *reinterpret_cast<uint4*>(yy) = o[0];
     *reinterpret_cast<uint4*>(yy + 8) = o[1];
   } else {
     for (int i = 0; i < 16; ++i)
-      if (n0 + i < p.N) yy[i] = __float2bfloat16_rn(act_f(y[i], p.act));
+      if (n0 + i < p.N) yy[i] = __float2bfloat16_rn(act_t<ACT>(y[i]));
   }
 }
 
+// Unsplit epilogue of one row (m) over this warp's columns [c0, c1) of the
+// tile: TMEM -> registers (16 columns per wait) -> fused epilogue -> bf16.
+template <int ACT>
+__device__ __forceinline__ void epi_cols(const TcParams& p, uint32_t tbase, int c0, int c1, int tn, int BN, int m,
+                                         bool valid, const float* sc, const float* sh) {
+#pragma unroll 1
+  for (int c = c0; c < c1; c += 16) {
+    uint32_t v[16];
+    tmem_ld16(tbase + c, v);
+    tmem_ld_wait();
+    const int n0 = tn * BN + c;
+    if (!valid || n0 >= p.N) continue;
+    float y[16];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) y[i] = __uint_as_float(v[i]);
+    epi_store16<ACT>(p, m, n0, y, sc + c, sh + c);
+  }
+}
+
+template <int ACT>
+__device__ __forceinline__ void epi_ws(const TcParams& p, const float* wrow, int c0, int c1, int tn, int BN, int m,
+                                       const float* sc, const float* sh) {
+#pragma unroll 1
+  for (int c = c0; c < c1; c += 16) {
+    const int n0 = tn * BN + c;
+    if (n0 >= p.N) break;
+    float y[16];
+#pragma unroll
+    for (int i = 0; i < 16; i += 4) {
+      float4 f = __ldcg(reinterpret_cast<const float4*>(wrow + c + i));
+      y[i] = f.x; y[i + 1] = f.y; y[i + 2] = f.z; y[i + 3] = f.w;
+      __stcg(reinterpret_cast<float4*>(const_cast<float*>(wrow) + c + i), make_float4(0.f, 0.f, 0.f, 0.f));
+    }
+    epi_store16<ACT>(p, m, n0, y, sc + c, sh + c);
+  }
+}
+
+#define TC_ACT_DISPATCH(act, CALL)                         \
+  switch (act) {                                           \
+    case BL_ACT_RELU: { constexpr int A_ = BL_ACT_RELU; CALL; } break;   \
+    case BL_ACT_RELU6: { constexpr int A_ = BL_ACT_RELU6; CALL; } break; \
+    case BL_ACT_GELU: { constexpr int A_ = BL_ACT_GELU; CALL; } break;   \
+    default: { constexpr int A_ = BL_ACT_NONE; CALL; } break;           \
+  }
+
+constexpr int kEpiWarps = 8;   // 2 per SM sub-partition (TMEM lane quarter = warp % 4), split by columns
+constexpr int kTcThreads = 64 + 32 * kEpiWarps;
 constexpr int kMaxStages = 8;
 constexpr int kDynSmemMax = 227 * 1024 - 2048;   // opt-in limit minus the executor's static smem
 
@@ -263,9 +312,9 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
     }
     for (int i = 0; i < 2; ++i) {
       mbar_init(&tfull[i], 1);
-      mbar_init(&tempty[i], 4);
+      mbar_init(&tempty[i], kEpiWarps);
       mbar_init(&rfull[i], 1);
-      mbar_init(&rempty[i], 5);
+      mbar_init(&rempty[i], 1 + kEpiWarps);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -413,8 +462,13 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       if (++acc == Cfg::kAcc) { acc = 0; aph ^= 1; }
     }
   } else {
-    // ---------------- epilogue warps 2..5 (TMEM lane quarter = warp % 4)
+    // ---------------- epilogue warps 2..9: TMEM lane quarter = warp % 4, and
+    // half (warp - 2) / 4 of the tile's columns, so every SM sub-partition
+    // runs two epilogue warps
     const int q = warp & 3;
+    const int half = (warp - 2) >> 2;
+    const int c0 = BN >= 32 ? half * (BN / 2) : (half ? BN : 0);
+    const int c1 = BN >= 32 ? c0 + BN / 2 : BN;
     bool dep_waited = false;
     int rs = 0;
     uint32_t rph = 0;
@@ -442,38 +496,27 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         m = oh * p.OW + ow;
       }
       // stage this tile's scale/shift (independent of the previous kernel)
-      asm volatile("bar.sync 2, 128;" ::: "memory");   // previous tile's readers are done
-      for (int i = threadIdx.x - 64; i < BN; i += 128) {
+      asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiWarps) : "memory");   // previous tile's readers are done
+      for (int i = threadIdx.x - 64; i < BN; i += 32 * kEpiWarps) {
         const int n = tn * BN + i;
         epi_sc[i] = (p.scale && n < p.N) ? __ldg(p.scale + n) : 1.f;
         epi_sh[i] = (p.shift && n < p.N) ? __ldg(p.shift + n) : 0.f;
       }
-      asm volatile("bar.sync 2, 128;" ::: "memory");
+      asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiWarps) : "memory");
       if (!dep_waited) {   // residual reads / output writes depend on earlier kernels
         pdl_wait();
         dep_waited = true;
       }
-      if (p.R && valid) {  // pull this row's residual segment into L2 while the MMAs run
-        const char* rr = reinterpret_cast<const char*>(p.R + (size_t)m * p.ldr + tn * BN);
-        for (int b = 0; b < BN * 2; b += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(rr + b));
+      if (p.R && valid && c1 > c0) {  // pull this row's residual segment into L2 while the MMAs run
+        const char* rr = reinterpret_cast<const char*>(p.R + (size_t)m * p.ldr + tn * BN + c0);
+        for (int b = 0; b < (c1 - c0) * 2; b += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(rr + b));
       }
       mbar_wait(&tfull[acc], aph);
       tc_fence_after();
       if (threadIdx.x == 64) TR(6);      // 6: accumulator ready (last tile)
       const uint32_t tbase = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN;
       if (p.splits == 1) {
-#pragma unroll 1
-        for (int c = 0; c < BN; c += 16) {
-          uint32_t v[16];
-          tmem_ld16(tbase + c, v);
-          tmem_ld_wait();
-          const int n0 = tn * BN + c;
-          if (!valid || n0 >= p.N) continue;
-          float y[16];
-#pragma unroll
-          for (int i = 0; i < 16; ++i) y[i] = __uint_as_float(v[i]);
-          epi_store16(p, m, n0, y, epi_sc + c, epi_sh + c);
-        }
+        TC_ACT_DISPATCH(p.act, (epi_cols<A_>(p, tbase, c0, c1, tn, BN, m, valid, epi_sc, epi_sh)))
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty[acc]);
@@ -482,7 +525,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         // split-K: add this unit's partial tile into the fp32 workspace
         float* wrow = p.ws + ((size_t)tile * 128 + row) * BN;
 #pragma unroll 1
-        for (int c = 0; c < BN; c += 16) {
+        for (int c = c0; c < c1; c += 16) {
           uint32_t v[16];
           tmem_ld16(tbase + c, v);
           tmem_ld_wait();
@@ -497,26 +540,12 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty[acc]);  // TMEM no longer needed
         __threadfence();
-        asm volatile("bar.sync 1, 128;" ::: "memory");   // the 4 epilogue warps
+        asm volatile("bar.sync 1, %0;" ::"n"(32 * kEpiWarps) : "memory");   // all epilogue warps
         if (threadIdx.x == 64) *last_flag = (atomicAdd(p.sem + tile, 1u) == (unsigned)p.splits - 1) ? 1 : 0;
-        asm volatile("bar.sync 1, 128;" ::: "memory");
+        asm volatile("bar.sync 1, %0;" ::"n"(32 * kEpiWarps) : "memory");
         if (*last_flag) {
           __threadfence();
-          if (valid) {
-#pragma unroll 1
-            for (int c = 0; c < BN; c += 16) {
-              const int n0 = tn * BN + c;
-              if (n0 >= p.N) break;
-              float y[16];
-#pragma unroll
-              for (int i = 0; i < 16; i += 4) {
-                float4 f = __ldcg(reinterpret_cast<const float4*>(wrow + c + i));
-                y[i] = f.x; y[i + 1] = f.y; y[i + 2] = f.z; y[i + 3] = f.w;
-                __stcg(reinterpret_cast<float4*>(wrow + c + i), make_float4(0.f, 0.f, 0.f, 0.f));
-              }
-              epi_store16(p, m, n0, y, epi_sc + c, epi_sh + c);
-            }
-          }
+          if (valid) TC_ACT_DISPATCH(p.act, (epi_ws<A_>(p, wrow, c0, c1, tn, BN, m, epi_sc, epi_sh)))
           if (threadIdx.x == 64) p.sem[tile] = 0;
         }
       }
@@ -533,7 +562,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
 }
 
 template <int BN, int BK>
-__global__ void __launch_bounds__(192, 1) k_tc_gemm(const __grid_constant__ TcParams p, const GateArgs g) {
+__global__ void __launch_bounds__(kTcThreads, 2) k_tc_gemm(const __grid_constant__ TcParams p, const GateArgs g) {
   if (threadIdx.x == 0) TR(0);   // 0: CTA start
   if (gate_in_range(g) || gate_linger(g)) tc_work<BN, BK>(p, g);
   pdl_trigger();
@@ -753,7 +782,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   }
   d.op = op;
   d.tiles = (uint32_t)(tiles_m * p.tiles_n * p.splits);
-  d.block = 192;
+  d.block = kTcThreads;
   d.grid = caps.S;
   bool ok = false;
 #define TC_CASE(bn, bk) \

@@ -167,7 +167,7 @@ bl_status Engine::set_io(int t, const void* hin, void* din, size_t inb, const vo
 bl_status Engine::debug_overhead(int variant, int reps, int64_t* ns, std::string& err) {
   if (!rt_) { err = "no device"; return BL_E_STATE; }
   if (started_) { err = "diagnostics while running"; return BL_E_STATE; }
-  if (!ns || variant < 0 || variant > 3 || reps < 1) { err = "bad args"; return BL_E_INVALID; }
+  if (!ns || variant < 0 || variant > 7 || reps < 1) { err = "bad args"; return BL_E_INVALID; }
   rt_->set_device();
   return rt_->overhead(variant, reps, ns, err) ? BL_OK : BL_E_CUDA;
 }

@@ -28,7 +28,8 @@ def main():
     if a.mode == "time":
         for v, nm in [(0, "empty kernel"), (1, "gate+queue+exit"), (2, "gate+queue+exit+stamps"),
                       (3, "gate+queue+exit+stamps, PDL")]:
-            print(f"overhead {nm:32s} {ctx.debug_overhead(v, 500) / 1e3:7.2f} us/launch")
+            print(f"overhead {nm:32s} {ctx.debug_overhead(v, 500) / 1e3:7.2f} us/launch (device), "
+                  f"{ctx.debug_overhead(v | 4, 500) / 1e3:7.2f} us/launch call (host)")
     ms = models.build_config(ctx, a.config, "fp32" if a.config == "C1" else "bf16")
     tot = {}
     for m in ms:
