@@ -370,6 +370,31 @@ uint64_t DeviceRT::launch(int h, int lo, int hi, void* stream, std::string& err)
   return seq;
 }
 
+bool DeviceRT::launch_seq(int h, uint64_t seq, int lo, int hi, void* stream, std::string& err) {
+  const KernelDesc& kd = *kernels_[h];
+  const GateArgs g = make_gate(seq, kd.tiles, lo, hi);
+  const cudaError_t e = kd.launch(kd, g, (cudaStream_t)stream);
+  if (e != cudaSuccess) {
+    err = std::string("launch ") + kd.family + ": " + cudaGetErrorString(e);
+    return false;
+  }
+  return true;
+}
+
+__global__ void k_marker(const GateArgs g);
+
+bool DeviceRT::launch_marker_seq(uint64_t seq, void* stream, std::string& err) {
+  GateArgs g = make_gate(seq, 0, 0, 0);
+  g.lid_map = nullptr;
+  k_marker<<<1, 32, 0, (cudaStream_t)stream>>>(g);
+  const cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) {
+    err = std::string("marker: ") + cudaGetErrorString(e);
+    return false;
+  }
+  return true;
+}
+
 __global__ void k_marker(const GateArgs g) {
   // zero tiles: the single CTA is the last one and publishes the stamps
   int last = 0;

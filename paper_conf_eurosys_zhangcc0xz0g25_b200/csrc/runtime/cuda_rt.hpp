@@ -50,6 +50,11 @@ class DeviceRT {
   void refresh_async(uint64_t lo, uint64_t hi);
   void refresh_sync(uint64_t lo, uint64_t hi);
   uint64_t last_seq() const { return seq_; }
+  // Parallel launch (Engine launcher threads): the scheduler thread allocates
+  // the launch's seq; any thread may then launch it on its own stream.
+  uint64_t alloc_seq() { return ++seq_; }
+  bool launch_seq(int h, uint64_t seq, int lo, int hi, void* stream, std::string& err);
+  bool launch_marker_seq(uint64_t seq, void* stream, std::string& err);
 
   // Streams / events (thin wrappers so the engine does not include CUDA headers).
   void* stream_create();

@@ -6,6 +6,7 @@
 #include <chrono>
 #include <climits>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 
 #include "cuda_rt.hpp"
@@ -331,10 +332,15 @@ bl_status Engine::start(std::string& err) {
   if (rt_) run_first_seq_ = rt_->last_seq() + 1;
   inflight_.clear();
   prev_events_.clear();
+  prev_parts_.clear();
+  prev_squad_ = 0;
   stop_ = false;
   failed_ = false;
   t0_ = now_ns() + 1000000;  // VIRTUAL on a device: wall anchor of trace time 0
   started_ = true;
+  par_launch_ = true;
+  if (const char* e = std::getenv("BLESS_LAUNCH_THREADS")) par_launch_ = std::atoi(e) != 0;
+  start_launchers();
   th_ = std::thread([this] { thread_main(); });
   return BL_OK;
 }
@@ -396,6 +402,7 @@ bl_status Engine::drain(int64_t timeout_ns, std::string& err) {
 bl_status Engine::stop(std::string& err) {
   stop_ = true;
   if (th_.joinable()) th_.join();
+  stop_launchers();
   if (rt_ && started_) {
     rt_->set_device();
     if (!rt_->device_sync()) { err = "device error at stop"; started_ = false; return BL_E_CUDA; }
@@ -586,6 +593,119 @@ uint64_t Engine::launch_one(int t, int k, int lo, int hi, void* stream, int64_t 
   return seq;
 }
 
+// ------------------------------------------------------------------ parallel launch
+bool Engine::prepare_one(int t, int k, int lo, int hi, int64_t req, bool last, std::vector<LaunchItem>& items) {
+  const TenantRT& tr = ten_[t];
+  if (k == 0 && tr.in_bytes) items.push_back({LaunchItem::H2D, -1, 0, 0, 0});
+  const uint64_t seq = rt_->alloc_seq();
+  items.push_back({LaunchItem::KERNEL, tr.handles[k], seq, lo, hi});
+  bl_launch_rec rec{};
+  rec.seq = seq;
+  rec.tenant = t;
+  rec.kernel = k;
+  rec.lo = (int16_t)lo;
+  rec.hi = (int16_t)hi;
+  rec.req = req >= 0 ? (uint64_t)req : ~0ull;
+  size_t idx;
+  {
+    std::lock_guard<std::mutex> lk(log_mu_);
+    idx = llog_.size();
+    llog_.push_back(rec);
+  }
+  if (last && tr.out_bytes) {
+    // the request completes when its output has landed in host memory: a
+    // one-CTA marker after the D2H copy carries the completion stamp
+    const uint64_t mseq = rt_->alloc_seq();
+    items.push_back({LaunchItem::D2H, -1, 0, 0, 0});
+    items.push_back({LaunchItem::MARKER, -1, mseq, 0, 0});
+    pending_.push_back({seq, idx, req, k, 0});
+    pending_.push_back({mseq, (size_t)-1, req, -1, 1});
+  } else {
+    pending_.push_back({seq, idx, req, k, last ? 1 : 0});
+  }
+  return true;
+}
+
+bool Engine::exec_items(int t, const std::vector<LaunchItem>& items, void* stream, std::string& err) {
+  const TenantRT& tr = ten_[t];
+  for (const LaunchItem& it : items) {
+    switch (it.kind) {
+      case LaunchItem::KERNEL:
+        if (!rt_->launch_seq(it.handle, it.seq, it.lo, it.hi, stream, err)) return false;
+        break;
+      case LaunchItem::H2D:
+        if (!rt_->memcpy_async(tr.dev_in, tr.host_in, tr.in_bytes, stream)) { err = "H2D input copy failed"; return false; }
+        break;
+      case LaunchItem::D2H:
+        if (!rt_->memcpy_async(tr.host_out, tr.dev_out, tr.out_bytes, stream)) { err = "D2H output copy failed"; return false; }
+        break;
+      case LaunchItem::MARKER:
+        if (!rt_->launch_marker_seq(it.seq, stream, err)) return false;
+        break;
+    }
+  }
+  return true;
+}
+
+void Engine::push_job(int t, LaunchJob&& job) {
+  Launcher& L = *launchers_[t];
+  {
+    std::lock_guard<std::mutex> lk(L.mu);
+    L.q.push_back(std::move(job));
+  }
+  L.queued.fetch_add(1, std::memory_order_release);
+}
+
+void Engine::launcher_main(int t) {
+  rt_->set_device();
+  Launcher& L = *launchers_[t];
+  std::string err;
+  for (;;) {
+    if (L.queued.load(std::memory_order_acquire) == 0) {
+      if (L.quit.load()) return;
+      cpu_relax();
+      continue;
+    }
+    LaunchJob job;
+    {
+      std::lock_guard<std::mutex> lk(L.mu);
+      job = std::move(L.q.front());
+      L.q.pop_front();
+    }
+    L.queued.fetch_sub(1, std::memory_order_release);
+    if (job.wait_squad) {
+      // squad barrier: the previous squad's events must have been recorded
+      // (by their launchers) before this stream waits on them
+      for (int l : job.wait_parts)
+        while (launchers_[l]->recorded.load(std::memory_order_acquire) < job.wait_squad) {
+          if (L.quit.load() || failed_) return;
+          cpu_relax();
+        }
+      for (void* ev : job.wait_events) rt_->stream_wait(ten_[t].stream, ev);
+    }
+    if (!exec_items(t, job.items, ten_[t].stream, err)) {
+      fail(err);
+      return;
+    }
+    if (job.record_event) rt_->event_record(job.record_event, ten_[t].stream);
+    if (job.squad) L.recorded.store(job.squad, std::memory_order_release);
+  }
+}
+
+void Engine::start_launchers() {
+  launchers_.clear();
+  if (!use_launchers() || !par_launch_) return;
+  for (int j = 0; j < nten(); ++j) launchers_.emplace_back(new Launcher());
+  for (int j = 0; j < nten(); ++j) launchers_[j]->th = std::thread([this, j] { launcher_main(j); });
+}
+
+void Engine::stop_launchers() {
+  for (auto& L : launchers_) L->quit = true;
+  for (auto& L : launchers_)
+    if (L->th.joinable()) L->th.join();
+  launchers_.clear();
+}
+
 void Engine::harvest() {
   if (!rt_ || pending_.empty()) return;
   if (!harvest_all_) {
@@ -628,6 +748,10 @@ void Engine::harvest() {
 
 void Engine::retire_inflight() {
   while (!inflight_.empty()) {
+    // an event not yet recorded (its launcher is behind) queries as complete
+    if (!launchers_.empty())
+      for (int l : inflight_.front().parts)
+        if (launchers_[l]->recorded.load(std::memory_order_acquire) < inflight_.front().squad) return;
     bool all = true;
     for (void* e : inflight_.front().events) {
       const int q = rt_->event_query(e);
@@ -661,29 +785,49 @@ void Engine::thread_main() {
 
 // BLESS: squads on the event-barriered tenant streams (§4.3-§4.5).
 void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req, const std::vector<int>& act_next) {
+  (void)act_next;
   // Squad barrier: every participant waits for the previous squad's kernels
   // (the paper synchronises after each squad, L276; here a GPU-side event
   // wait instead of a host synchronisation, L432's 20 us switch).
-  for (int j : d.parts)
-    for (void* ev : prev_events_) rt_->stream_wait(ten_[j].stream, ev);
-  std::vector<int> cnt(nten(), 0);
-  for (const Pick& p : d.picks) {
-    const int j = p.tenant;
-    const int k = p.kernel;
-    const bool last = k == (int)prof_.ten[j].k.size() - 1;
-    const bool first = k == 0;
-    (void)act_next;
-    (void)cnt;
-    if (!launch_one(j, k, p.lo, p.hi, ten_[j].stream, (first || last) ? act_req[j] : -1, last)) return;
+  const uint64_t sq = ++squad_id_;
+  if (launchers_.empty()) {   // single launch thread (BLESS_LAUNCH_THREADS=0)
+    for (int j : d.parts)
+      for (void* ev : prev_events_) rt_->stream_wait(ten_[j].stream, ev);
+    for (const Pick& p : d.picks) {
+      const int j = p.tenant, k = p.kernel;
+      const bool last = k == (int)prof_.ten[j].k.size() - 1;
+      if (!launch_one(j, k, p.lo, p.hi, ten_[j].stream, (k == 0 || last) ? act_req[j] : -1, last)) return;
+    }
+  }
+  std::vector<LaunchJob> jobs(launchers_.empty() ? 0 : nten());
+  if (!launchers_.empty()) {
+    for (int j : d.parts) {
+      jobs[j].squad = sq;
+      jobs[j].wait_squad = prev_squad_;
+      jobs[j].wait_parts = prev_parts_;
+      jobs[j].wait_events = prev_events_;
+    }
+    for (const Pick& p : d.picks) {
+      const int j = p.tenant, k = p.kernel;
+      const bool last = k == (int)prof_.ten[j].k.size() - 1;
+      prepare_one(j, k, p.lo, p.hi, (k == 0 || last) ? act_req[j] : -1, last, jobs[j].items);
+    }
   }
   Inflight inf;
+  inf.squad = sq;
+  inf.parts = d.parts;
   for (int j : d.parts) {
     TenantRT& t = ten_[j];
     void* ev = t.events[t.ev_next++ % t.events.size()];
-    rt_->event_record(ev, t.stream);
+    if (launchers_.empty()) rt_->event_record(ev, t.stream);
+    else jobs[j].record_event = ev;
     inf.events.push_back(ev);
   }
+  for (int j : d.parts)
+    if (!launchers_.empty()) push_job(j, std::move(jobs[j]));
   prev_events_ = inf.events;
+  prev_parts_ = d.parts;
+  prev_squad_ = sq;
   inflight_.push_back(std::move(inf));
 }
 
@@ -804,8 +948,15 @@ void Engine::loop_at_arrival(bool unbound) {
         fifo_[j].pop_front();
         const int m = (int)prof_.ten[j].k.size();
         const int lo = unbound ? 0 : ten_[j].lo, hi = unbound ? S() : ten_[j].hi;
-        for (int k = 0; k < m; ++k)
-          if (!launch_one(j, k, lo, hi, ten_[j].stream, (k == 0 || k == m - 1) ? r : -1, k == m - 1)) return;
+        if (!launchers_.empty()) {
+          LaunchJob job;
+          for (int k = 0; k < m; ++k)
+            prepare_one(j, k, lo, hi, (k == 0 || k == m - 1) ? r : -1, k == m - 1, job.items);
+          push_job(j, std::move(job));
+        } else {
+          for (int k = 0; k < m; ++k)
+            if (!launch_one(j, k, lo, hi, ten_[j].stream, (k == 0 || k == m - 1) ? r : -1, k == m - 1)) return;
+        }
         launched = true;
       }
     }

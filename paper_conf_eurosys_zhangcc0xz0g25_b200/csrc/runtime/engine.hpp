@@ -45,6 +45,38 @@ struct TenantRT {
   size_t out_bytes = 0;
 };
 
+// Parallel launch path.  Host launch calls cost ~3 us each on the B200 boxes
+// (kprobe: cudaLaunchKernelExC ~ 3.0-3.4 us per call), about the device time
+// of a batch-1 kernel, so one host thread launching every tenant's kernels
+// serialises co-running tenants on the CPU.  Each tenant stream gets its own
+// launcher thread; the scheduler thread decides, allocates the launches' seqs
+// and logs them, and hands a LaunchJob to the tenant's launcher.
+struct LaunchItem {
+  enum Kind : uint8_t { KERNEL = 0, H2D = 1, D2H = 2, MARKER = 3 };
+  uint8_t kind = KERNEL;
+  int handle = -1;
+  uint64_t seq = 0;
+  int lo = 0, hi = 0;
+};
+
+struct LaunchJob {
+  uint64_t squad = 0;             // squad id (0: none -- baseline policies)
+  uint64_t wait_squad = 0;        // squad barrier: every launcher in wait_parts
+  std::vector<int> wait_parts;    //   must have recorded squad wait_squad first,
+  std::vector<void*> wait_events; //   then its stream waits on wait_events
+  std::vector<LaunchItem> items;
+  void* record_event = nullptr;   // recorded after the items (squad barrier)
+};
+
+struct Launcher {
+  std::thread th;
+  std::mutex mu;
+  std::deque<LaunchJob> q;
+  std::atomic<size_t> queued{0};
+  std::atomic<bool> quit{false};
+  std::atomic<uint64_t> recorded{0};   // last squad whose barrier event this launcher recorded
+};
+
 struct PendingLaunch {
   uint64_t seq;
   size_t log_idx;
@@ -98,6 +130,14 @@ class Engine {
   void retire_inflight();
   void launch_squad(const Decision& d, const std::vector<int64_t>& act_req, const std::vector<int>& act_next);
   uint64_t launch_one(int t, int k, int lo, int hi, void* stream, int64_t req, bool last);
+  // parallel launch path
+  bool prepare_one(int t, int k, int lo, int hi, int64_t req, bool last, std::vector<LaunchItem>& items);
+  bool exec_items(int t, const std::vector<LaunchItem>& items, void* stream, std::string& err);
+  void push_job(int t, LaunchJob&& job);
+  void launcher_main(int t);
+  void start_launchers();
+  void stop_launchers();
+  bool use_launchers() const { return rt_ && prm_.policy != BL_POLICY_TEMPORAL; }
   void log_decision(const Decision& d);
   void fail(const std::string& msg);
   int nten() const { return (int)ten_.size(); }
@@ -136,7 +176,14 @@ class Engine {
   bool harvest_all_ = false;
   struct Inflight {
     std::vector<void*> events;
+    std::vector<int> parts;
+    uint64_t squad = 0;
   };
+  std::vector<std::unique_ptr<Launcher>> launchers_;
+  uint64_t squad_id_ = 0;
+  bool par_launch_ = true;        // per-tenant launcher threads (BLESS_LAUNCH_THREADS=0 disables)
+  std::vector<int> prev_parts_;
+  uint64_t prev_squad_ = 0;
   std::deque<Inflight> inflight_;
   std::vector<void*> prev_events_;
   void* temporal_stream_ = nullptr;
