@@ -63,7 +63,9 @@ def parse():
     ap.add_argument("--requests", type=int, default=60, help="requests per tenant per step")
     # B200 operating point chosen by the c% x S_max sweep, the
     # way the paper picks its own empirically (§6.7).
-    ap.add_argument("--squad-max", type=int, default=20)
+    ap.add_argument("--squad-max", type=int, default=None,
+                    help="S_max (L406-L408); default per config from the B200 sweeps in "
+                         "profiles/round1/param_sweep: C1 4, C2 20, C3 10, C4 10")
     ap.add_argument("--split-pct", type=int, default=25)
     ap.add_argument("--lookahead-us", type=float, default=20.0)
     ap.add_argument("--max-inflight", type=int, default=2)
@@ -75,6 +77,12 @@ def parse():
     ap.add_argument("--light", action="store_true", help="timed steps only (for ncu launch lists)")
     ap.add_argument("--out-dir", default=os.path.join(ROOT, "gpurun_out"))
     return ap.parse_args()
+
+
+def default_squad_max(args):
+    """S_max per config unless given (B200 sweeps, profiles/round1/param_sweep)."""
+    if args.squad_max is None:
+        args.squad_max = {"C1": 4, "C2": 20, "C3": 10, "C4": 10}.get(args.config, 20)
 
 
 # ---------------------------------------------------------------------------- clocks
@@ -250,6 +258,7 @@ def native(args):
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     plan = replicas.plan(rank, world, local, args.config, sorted(models.CONFIGS))
     args.config = plan.config
+    default_squad_max(args)
 
     dtype = "fp32" if args.config == "C1" else "bf16"
     # tcgen05 tile configurations are autotuned at registration; a saved profile
@@ -567,6 +576,8 @@ def reference(args):
     from threadpoolctl import threadpool_info
 
     cfg = "C2" if args.config == "C5" else args.config
+    args.config = cfg
+    default_squad_max(args)
     tenants = REF_CONFIGS[cfg]
     names = [n for n, _ in tenants]
     # profile table: the last B200 profile committed under profiles/, else a synthetic stand-in

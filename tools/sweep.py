@@ -36,7 +36,7 @@ def main():
                 with open(gen) as f, open(prof.replace("profile_", kind + "_"), "w") as g:
                     g.write(f.read())
     for point in itertools.product(*axes):
-        args = [sys.executable, os.path.join(ROOT, "bench.py"), "--config", a.config, "--no-cpu-baseline",
+        args = [sys.executable, os.path.join(ROOT, "bench.py"), "--config", a.config, "--no-cpu-baseline", "--no-slo",
                 "--steps", str(a.steps), "--warmup", "1", "--requests", str(a.requests)]
         if os.path.exists(prof):
             args += ["--load-profile", prof]

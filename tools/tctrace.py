@@ -26,13 +26,15 @@ def main():
     from paper_conf_eurosys_zhangcc0xz0g25_b200 import build, capi
     from paper_conf_eurosys_zhangcc0xz0g25_b200.models import Builder
     build.build(force=True, verbose=False)
-    kind, d = sys.argv[1], [int(x) for x in sys.argv[2:]]
+    args = [a for a in sys.argv[1:] if not a.startswith("--act=")]
+    act = next((a.split("=")[1] for a in sys.argv[1:] if a.startswith("--act=")), "gelu")
+    kind, d = args[0], [int(x) for x in args[1:]]
     ctx = capi.Ctx(0)
     S = ctx.device_info().sm_count
     t = ctx.register_tenant(1.0, "k")
     b = Builder(ctx, t, "k", 1.0, "bf16", seed=7)
     if kind == "gemm":
-        b.gemm(b.input((d[0], d[2])), d[1], act="gelu", bias=True)
+        b.gemm(b.input((d[0], d[2])), d[1], act=act, bias=True)
     else:
         H, W, Cc, K, k, s, p = d
         b.conv(b.input((1, H, W, Cc)), K, k, s, p, act="relu", bn=True)
@@ -48,7 +50,7 @@ def main():
         ok = (v[:, 0] > 0) & (v[:, 1] >= v[:, 0]) & (v[:, 9] >= v[:, 1]) & (v[:, 7] > 0)
         w = v[ok]
         t0 = int(v[v[:, 0] > 0, 0].min())
-        print(f"{kind} {d} {ki.family.decode()} tiles={ki.tiles} reps={reps}: event avg {ns / 1e3:.2f} us, "
+        print(f"{kind} {d} act={act} {ki.family.decode()} tiles={ki.tiles} reps={reps}: event avg {ns / 1e3:.2f} us, "
               f"{ok.sum()} working CTAs")
         if not len(w):
             continue
