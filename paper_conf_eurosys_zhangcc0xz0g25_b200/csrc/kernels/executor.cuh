@@ -99,32 +99,22 @@ __device__ __forceinline__ int gate_claim(const GateArgs& g, bool& marked) {
 }
 
 // Block-wide tile loop for simple (non warp-specialised) kernels.
-// body(tile) is executed by all threads of the CTA.  The first claim is made
-// before griddepcontrol.wait (the tile queue is this launch's own state, so
-// under programmatic dependent launch the atomic round trip overlaps the tail
-// of the previous kernel); only body() touches data the predecessor wrote.
-// When the queue holds >= 2 tiles per CTA, the claim of the next tile is
-// issued before body(tile) runs (double-buffered), taking the atomic off the
-// per-tile critical path; with fewer tiles it is not, so that early CTAs do
-// not hoard tiles that idle CTAs could run.
+// body(tile) is executed by all threads of the CTA.  (Measured on B200: a
+// variant that claimed the first tile before griddepcontrol.wait, or issued
+// the next claim inside the previous body, made LayerNorm 384x1024 slower,
+// 8.8 -> 11.0 us, with its 48 tiles landing on 17 SMs instead of 24 --
+// profiles/round1/ln_executor_ab.txt.)
 template <class Body>
 __device__ __forceinline__ void gate_tile_loop(const GateArgs& g, Body&& body) {
-  __shared__ int s_tile[2];
+  __shared__ int s_tile;
   bool marked = false;
-  const bool ahead = g.tiles >= 2u * gridDim.x;
-  if (threadIdx.x == 0) s_tile[0] = gate_claim(g, marked);
-  __syncthreads();
-  if (s_tile[0] < 0) return;
-  pdl_wait();
-  int b = 0;
   for (;;) {
-    const int t = s_tile[b];
-    if (t < 0) break;
-    if (ahead && threadIdx.x == 0) s_tile[b ^ 1] = gate_claim(g, marked);
-    body(t);
-    if (!ahead && threadIdx.x == 0) s_tile[b ^ 1] = gate_claim(g, marked);
+    if (threadIdx.x == 0) s_tile = gate_claim(g, marked);
     __syncthreads();
-    b ^= 1;
+    const int t = s_tile;
+    __syncthreads();
+    if (t < 0) break;
+    body(t);
   }
 }
 
@@ -210,11 +200,17 @@ __device__ __forceinline__ void gate_finalize(const GateArgs& g, bool fallback) 
 // The canonical gated kernel body for tile-loop ops: Op::tile(params, t, smem).
 template <class Op>
 __device__ __forceinline__ void gated_run(const typename Op::Params& p, const GateArgs& g, unsigned char* smem) {
-  if (gate_in_range(g) || gate_linger(g)) gate_tile_loop(g, [&](int t) { Op::tile(p, t, smem); });
+  if (gate_in_range(g) || gate_linger(g)) {
+    pdl_wait();
+    gate_tile_loop(g, [&](int t) { Op::tile(p, t, smem); });
+  }
   pdl_trigger();
   int last = 0;
   const bool fb = gate_leave(g, last);
-  if (fb) gate_tile_loop(g, [&](int t) { Op::tile(p, t, smem); });
+  if (fb) {
+    pdl_wait();
+    gate_tile_loop(g, [&](int t) { Op::tile(p, t, smem); });
+  }
   if (last) gate_finalize(g, fb);
 }
 #endif
