@@ -295,6 +295,7 @@ __global__ void __launch_bounds__(attn::kThreads, 1) k_attn_tc(const __grid_cons
                                                                 const GateArgs g) {
   if (gate_in_range(g) || gate_linger(g)) attn_work(p, g);
   pdl_trigger();
+  if (!g.stamp) return;   // light exit
   int last = 0;
   const bool fb = gate_leave(g, last);
   if (fb) attn_work(p, g);

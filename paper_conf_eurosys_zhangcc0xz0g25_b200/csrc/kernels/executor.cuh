@@ -25,6 +25,18 @@
 // hardware placed every CTA elsewhere); it then processes the tiles itself and
 // flags the launch ("fallback"), so correctness never depends on placement.
 //
+// Light exit: most launches (a request's middle kernels) skip the exit
+// protocol (stamp = 0): no per-CTA atomic, no last-CTA publish, so the grid
+// completes as soon as its last tile's stores are issued (the exit protocol
+// was 1.5-2.4 us of a batch-1 kernel's critical path, profiles/round1/
+// tctrace_*).  Their end time is stamped by the successor on the same stream
+// when its griddepcontrol.wait returns (prev_stats); the slot and stats record
+// reuse is handled ahead of time by the tile-0 claimer.  Launches whose
+// completion the host must observe (a request's first/last kernel, the last
+// kernel of a tenant's chain in a squad, profiling) use the full protocol.
+// No tile is ever lost without the fallback: out-of-range CTAs linger and
+// help after a timeout, so every queue drains.
+//
 // Programmatic dependent launch: kernels are launched with programmatic stream
 // serialization; a CTA waits (griddepcontrol.wait) only right before touching
 // data produced by the previous kernel, and signals its dependents as soon as
@@ -54,11 +66,14 @@ constexpr uint64_t kMaskAhead = 32768;  // stats record zeroed this many launche
 struct GateArgs {
   DevSlot* slot;
   SlotStats* stats;        // this launch's record
-  SlotStats* stats_ahead;  // record of launch seq + kMaskAhead (mask zeroed here)
+  SlotStats* stats_ahead;  // record of launch seq + kMaskAhead (flags/mask zeroed here)
+  DevSlot* slot_ahead;     // slot of launch seq + kMaskAhead (zeroed here)
+  SlotStats* prev_stats;   // light predecessor on the stream (its end stamp is written here) or null
   const uint8_t* lid_map;  // logical SM index per %smid (255 = unusable); null = identity
   uint64_t seq;
   uint32_t tiles;
   int32_t lo, hi;
+  uint32_t stamp;          // 1: full exit protocol (last CTA publishes end + seq); 0: light exit
 };
 
 #ifdef __CUDACC__
@@ -86,10 +101,27 @@ __device__ __forceinline__ bool gate_in_range(const GateArgs& g) {
 
 // Claim the next tile (call from ONE thread).  Returns -1 when exhausted.
 // 'marked' tracks whether this CTA already set its SM bit in the mask.
-__device__ __forceinline__ int gate_claim(const GateArgs& g, bool& marked) {
+// The claimer of tile 0 stamps the start, zeroes the slot and the stats
+// flags/mask of the launch kMaskAhead later (no CTA of that ring position's
+// previous launch can still run), and -- if it claims after
+// griddepcontrol.wait (after_wait) -- writes the end stamp of a light
+// predecessor on the stream, which completed exactly when that wait returned.
+__device__ __forceinline__ void gate_prev_end(const GateArgs& g, int64_t now) {
+  if (g.prev_stats) g.prev_stats->end_gt = now;
+}
+__device__ __forceinline__ int gate_claim(const GateArgs& g, bool& marked, bool after_wait = true) {
   const uint32_t t = (uint32_t)atomicAdd(&g.slot->ctr, 1ull);
   if (t >= g.tiles) return -1;
-  if (t == 0) g.stats->start_gt = (int64_t)ptx_globaltimer();
+  if (t == 0) {
+    const int64_t now = (int64_t)ptx_globaltimer();
+    g.stats->start_gt = now;
+    g.slot_ahead->ctr = 0ull;
+    g.stats_ahead->flags = 0u;
+    uint4* fm = reinterpret_cast<uint4*>(g.stats_ahead->mask);
+    fm[0] = make_uint4(0, 0, 0, 0);
+    fm[1] = make_uint4(0, 0, 0, 0);
+    if (after_wait) gate_prev_end(g, now);
+  }
   if (!marked) {
     marked = true;
     const int lid = gate_lid(g);
@@ -186,11 +218,13 @@ __device__ __forceinline__ void gate_finalize(const GateArgs& g, bool fallback) 
     out->end_gt = (int64_t)end;
     if (g.tiles == 0) out->start_gt = (int64_t)end;
     if (fallback) atomicOr(&out->flags, 1u);
-    // zero the flags and mask of the record reused kMaskAhead launches from now
-    g.stats_ahead->flags = 0u;
-    uint4* fm = reinterpret_cast<uint4*>(g.stats_ahead->mask);
-    fm[0] = make_uint4(0, 0, 0, 0);
-    fm[1] = make_uint4(0, 0, 0, 0);
+    if (g.tiles == 0) {   // nothing was claimed: zero ahead here (marker launches)
+      g.slot_ahead->ctr = 0ull;
+      g.stats_ahead->flags = 0u;
+      uint4* fm = reinterpret_cast<uint4*>(g.stats_ahead->mask);
+      fm[0] = make_uint4(0, 0, 0, 0);
+      fm[1] = make_uint4(0, 0, 0, 0);
+    }
     g.slot->ctr = 0ull;
     __threadfence();
     *reinterpret_cast<volatile uint64_t*>(&out->seq) = g.seq;
@@ -205,6 +239,7 @@ __device__ __forceinline__ void gated_run(const typename Op::Params& p, const Ga
     gate_tile_loop(g, [&](int t) { Op::tile(p, t, smem); });
   }
   pdl_trigger();
+  if (!g.stamp) return;   // light exit (see header)
   int last = 0;
   const bool fb = gate_leave(g, last);
   if (fb) {

@@ -239,6 +239,7 @@ template <int MAXM>
 __global__ void __launch_bounds__(kGvThreads, 2) k_gemv_tma(const GemvTmaParams p, const GateArgs g) {
   if (gate_in_range(g) || gate_linger(g)) gemv_work<MAXM>(p, g);
   pdl_trigger();
+  if (!g.stamp) return;   // light exit
   int last = 0;
   const bool fb = gate_leave(g, last);
   if (fb) gemv_work<MAXM>(p, g);

@@ -327,7 +327,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   // the first tile claim (an L2 atomic round trip) overlaps the barrier/TMEM setup
   bool marked = false;
   int first_claim = -2;
-  if (threadIdx.x == 0) first_claim = gate_claim(g, marked);
+  if (threadIdx.x == 0) first_claim = gate_claim(g, marked, false);
   if (threadIdx.x == 0) {
     for (int i = 0; i < ST; ++i) {
       mbar_init(&full[i], 1);
@@ -368,7 +368,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       int rs = 0;
       uint32_t rph = 0;
       for (;;) {
-        const int t = first_claim != -2 ? first_claim : gate_claim(g, marked);
+        const int t = first_claim != -2 ? first_claim : gate_claim(g, marked, dep_waited);
         first_claim = -2;
         if (!dep_waited) TR(3);          // 3: first claim returned
         mbar_wait(&rempty[rs], rph ^ 1);
@@ -426,6 +426,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
             load_B(kb0 + i, st);
           }
           pdl_wait();
+          if (t == 0) gate_prev_end(g, (int64_t)ptx_globaltimer());   // predecessor just completed
           TR(4);                         // 4: producer past griddepcontrol.wait
           dep_waited = true;
           for (int i = 0; i < npre; ++i) load_A(kb0 + i, (stage + i) % ST);
@@ -590,6 +591,10 @@ __global__ void __launch_bounds__(kTcThreads, 2) k_tc_gemm(const __grid_constant
   if (gate_in_range(g) || gate_linger(g)) tc_work<BN, BK>(p, g);
   pdl_trigger();
   if (threadIdx.x == 0) TR(8);   // 8: work done, before the exit atomic
+  if (!g.stamp) {                // light exit
+    if (threadIdx.x == 0) TR(9);
+    return;
+  }
   int last = 0;
   const bool fb = gate_leave(g, last);
   if (fb) tc_work<BN, BK>(p, g);

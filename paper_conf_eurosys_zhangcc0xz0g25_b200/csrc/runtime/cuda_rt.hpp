@@ -33,7 +33,7 @@ class DeviceRT {
   const KernelDesc& kernel(int h) const { return *kernels_[h]; }
 
   // Launch kernel h confined to logical SMs [lo, hi) on stream; returns seq (>0) or 0 on error.
-  uint64_t launch(int h, int lo, int hi, void* stream, std::string& err);
+  uint64_t launch(int h, int lo, int hi, void* stream, std::string& err, bool stamp = true);
   // One-CTA completion marker (stats only, no work) on stream; returns seq or 0.
   uint64_t launch_marker(void* stream, std::string& err);
   bool memcpy_async(void* dst, const void* src, size_t n, void* stream);
@@ -44,6 +44,7 @@ class DeviceRT {
   bool overhead(int variant, int reps, int64_t* ns_out, std::string& err);
   // Non-blocking: true if launch seq's stats are in the host mirror.
   bool poll(uint64_t seq, LaunchStats* out);
+  void peek(uint64_t seq, LaunchStats* out);
   // Mirror the device stats of launches [lo, hi] (seq numbers) into host
   // memory: asynchronously (skipped while a previous copy is in flight) or
   // synchronously (after the launches are known complete).
@@ -53,7 +54,8 @@ class DeviceRT {
   // Parallel launch (Engine launcher threads): the scheduler thread allocates
   // the launch's seq; any thread may then launch it on its own stream.
   uint64_t alloc_seq() { return ++seq_; }
-  bool launch_seq(int h, uint64_t seq, int lo, int hi, void* stream, std::string& err);
+  bool launch_seq(int h, uint64_t seq, int lo, int hi, void* stream, std::string& err, bool stamp = true,
+                  uint64_t prev_light = 0);
   bool launch_marker_seq(uint64_t seq, void* stream, std::string& err);
 
   // Streams / events (thin wrappers so the engine does not include CUDA headers).
@@ -75,7 +77,7 @@ class DeviceRT {
 
   int64_t gt_to_host(int64_t gt) const { return gt - info_.clock_offset_ns; }
   bool calibrate_clock(std::string& err);
-  GateArgs make_gate(uint64_t seq, uint32_t tiles, int lo, int hi) const;
+  GateArgs make_gate(uint64_t seq, uint32_t tiles, int lo, int hi, bool stamp = true, uint64_t prev_light = 0) const;
 
  private:
   DeviceRT() = default;

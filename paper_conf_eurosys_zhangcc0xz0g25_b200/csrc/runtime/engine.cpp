@@ -417,7 +417,8 @@ bl_status Engine::stop(std::string& err) {
     std::lock_guard<std::mutex> lk(log_mu_);
     for (bl_launch_rec& r : llog_) {
       LaunchStats st;
-      if (r.seq >= lo && rt_->poll(r.seq, &st)) {
+      if (r.seq >= lo && r.seq <= hi) {
+        rt_->peek(r.seq, &st);   // light launches never publish their seq
         r.start_ns = st.start_host;
         r.end_ns = st.end_host;
         r.nsm = st.nsm;
@@ -537,45 +538,24 @@ void Engine::scan_submissions() {
   }
 }
 
-uint64_t Engine::launch_one(int t, int k, int lo, int hi, void* stream, int64_t req, bool last) {
+uint64_t Engine::launch_one(int t, int k, int lo, int hi, void* stream, int64_t req, bool last, bool stamp) {
   std::string err;
-  const TenantRT& tr = ten_[t];
-  if (k == 0 && tr.in_bytes && !rt_->memcpy_async(tr.dev_in, tr.host_in, tr.in_bytes, stream)) {
-    fail("H2D input copy failed");
-    return 0;
+  TenantRT& tr = ten_[t];
+  const bool own = stream == tr.stream;   // light-exit chaining only on the tenant's own stream
+  if (!own) stamp = true;
+  if (k == 0 && tr.in_bytes) {
+    if (!rt_->memcpy_async(tr.dev_in, tr.host_in, tr.in_bytes, stream)) {
+      fail("H2D input copy failed");
+      return 0;
+    }
+    if (own) tr.prev_light = 0;
   }
-  const uint64_t seq = rt_->launch(tr.handles[k], lo, hi, stream, err);
-  if (!seq) {
+  const uint64_t seq = rt_->alloc_seq();
+  if (!rt_->launch_seq(tr.handles[k], seq, lo, hi, stream, err, stamp, own ? tr.prev_light : 0)) {
     fail(err);
     return 0;
   }
-  if (last && tr.out_bytes) {
-    // the request completes when its output has landed in host memory: a
-    // one-CTA marker after the D2H copy carries the completion stamp
-    if (!rt_->memcpy_async(tr.host_out, tr.dev_out, tr.out_bytes, stream)) {
-      fail("D2H output copy failed");
-      return 0;
-    }
-    const uint64_t mseq = rt_->launch_marker(stream, err);
-    if (!mseq) {
-      fail(err);
-      return 0;
-    }
-    {
-      bl_launch_rec rec{};
-      rec.seq = seq;
-      rec.tenant = t;
-      rec.kernel = k;
-      rec.lo = (int16_t)lo;
-      rec.hi = (int16_t)hi;
-      rec.req = req >= 0 ? (uint64_t)req : ~0ull;
-      std::lock_guard<std::mutex> lk(log_mu_);
-      pending_.push_back({seq, llog_.size(), req, k, 0});
-      llog_.push_back(rec);
-    }
-    pending_.push_back({mseq, (size_t)-1, req, -1, 1});
-    return seq;
-  }
+  if (own) tr.prev_light = stamp ? 0 : seq;
   bl_launch_rec rec{};
   rec.seq = seq;
   rec.tenant = t;
@@ -589,16 +569,34 @@ uint64_t Engine::launch_one(int t, int k, int lo, int hi, void* stream, int64_t 
     idx = llog_.size();
     llog_.push_back(rec);
   }
-  pending_.push_back({seq, idx, req, k, last ? 1 : 0});
+  if (last && tr.out_bytes) {
+    // the request completes when its output has landed in host memory: a
+    // one-CTA marker after the D2H copy carries the completion stamp
+    if (!rt_->memcpy_async(tr.host_out, tr.dev_out, tr.out_bytes, stream)) {
+      fail("D2H output copy failed");
+      return 0;
+    }
+    const uint64_t mseq = rt_->launch_marker(stream, err);
+    if (!mseq) {
+      fail(err);
+      return 0;
+    }
+    if (own) tr.prev_light = 0;
+    pending_.push_back({seq, idx, req, k, 0});
+    pending_.push_back({mseq, (size_t)-1, req, -1, 1});
+    return seq;
+  }
+  if (stamp) pending_.push_back({seq, idx, req, k, last ? 1 : 0});
   return seq;
 }
 
 // ------------------------------------------------------------------ parallel launch
-bool Engine::prepare_one(int t, int k, int lo, int hi, int64_t req, bool last, std::vector<LaunchItem>& items) {
+bool Engine::prepare_one(int t, int k, int lo, int hi, int64_t req, bool last, std::vector<LaunchItem>& items,
+                         bool stamp) {
   const TenantRT& tr = ten_[t];
-  if (k == 0 && tr.in_bytes) items.push_back({LaunchItem::H2D, -1, 0, 0, 0});
+  if (k == 0 && tr.in_bytes) items.push_back({LaunchItem::H2D, 1, -1, 0, 0, 0});
   const uint64_t seq = rt_->alloc_seq();
-  items.push_back({LaunchItem::KERNEL, tr.handles[k], seq, lo, hi});
+  items.push_back({LaunchItem::KERNEL, (uint8_t)(stamp ? 1 : 0), tr.handles[k], seq, lo, hi});
   bl_launch_rec rec{};
   rec.seq = seq;
   rec.tenant = t;
@@ -616,22 +614,24 @@ bool Engine::prepare_one(int t, int k, int lo, int hi, int64_t req, bool last, s
     // the request completes when its output has landed in host memory: a
     // one-CTA marker after the D2H copy carries the completion stamp
     const uint64_t mseq = rt_->alloc_seq();
-    items.push_back({LaunchItem::D2H, -1, 0, 0, 0});
-    items.push_back({LaunchItem::MARKER, -1, mseq, 0, 0});
+    items.push_back({LaunchItem::D2H, 1, -1, 0, 0, 0});
+    items.push_back({LaunchItem::MARKER, 1, -1, mseq, 0, 0});
     pending_.push_back({seq, idx, req, k, 0});
     pending_.push_back({mseq, (size_t)-1, req, -1, 1});
-  } else {
+  } else if (stamp) {
     pending_.push_back({seq, idx, req, k, last ? 1 : 0});
   }
   return true;
 }
 
 bool Engine::exec_items(int t, const std::vector<LaunchItem>& items, void* stream, std::string& err) {
-  const TenantRT& tr = ten_[t];
+  TenantRT& tr = ten_[t];
   for (const LaunchItem& it : items) {
+    if (it.kind != LaunchItem::KERNEL) tr.prev_light = 0;
     switch (it.kind) {
       case LaunchItem::KERNEL:
-        if (!rt_->launch_seq(it.handle, it.seq, it.lo, it.hi, stream, err)) return false;
+        if (!rt_->launch_seq(it.handle, it.seq, it.lo, it.hi, stream, err, it.stamp != 0, tr.prev_light)) return false;
+        tr.prev_light = it.stamp ? 0 : it.seq;
         break;
       case LaunchItem::H2D:
         if (!rt_->memcpy_async(tr.dev_in, tr.host_in, tr.in_bytes, stream)) { err = "H2D input copy failed"; return false; }
@@ -790,13 +790,24 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
   // (the paper synchronises after each squad, L276; here a GPU-side event
   // wait instead of a host synchronisation, L432's 20 us switch).
   const uint64_t sq = ++squad_id_;
+  // full exit protocol only where the host observes completion: a request's
+  // first/last kernel and the last kernel of each participant's chain
+  std::vector<int> last_pick(nten(), -1);
+  for (size_t i = 0; i < d.picks.size(); ++i) last_pick[d.picks[i].tenant] = (int)i;
+  auto stamp_of = [&](size_t i) {
+    const Pick& p = d.picks[i];
+    return p.kernel == 0 || p.kernel == (int)prof_.ten[p.tenant].k.size() - 1 || last_pick[p.tenant] == (int)i;
+  };
   if (launchers_.empty()) {   // single launch thread (BLESS_LAUNCH_THREADS=0)
-    for (int j : d.parts)
+    for (int j : d.parts) {
       for (void* ev : prev_events_) rt_->stream_wait(ten_[j].stream, ev);
-    for (const Pick& p : d.picks) {
+      ten_[j].prev_light = 0;
+    }
+    for (size_t i = 0; i < d.picks.size(); ++i) {
+      const Pick& p = d.picks[i];
       const int j = p.tenant, k = p.kernel;
       const bool last = k == (int)prof_.ten[j].k.size() - 1;
-      if (!launch_one(j, k, p.lo, p.hi, ten_[j].stream, (k == 0 || last) ? act_req[j] : -1, last)) return;
+      if (!launch_one(j, k, p.lo, p.hi, ten_[j].stream, (k == 0 || last) ? act_req[j] : -1, last, stamp_of(i))) return;
     }
   }
   std::vector<LaunchJob> jobs(launchers_.empty() ? 0 : nten());
@@ -807,10 +818,11 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
       jobs[j].wait_parts = prev_parts_;
       jobs[j].wait_events = prev_events_;
     }
-    for (const Pick& p : d.picks) {
+    for (size_t i = 0; i < d.picks.size(); ++i) {
+      const Pick& p = d.picks[i];
       const int j = p.tenant, k = p.kernel;
       const bool last = k == (int)prof_.ten[j].k.size() - 1;
-      prepare_one(j, k, p.lo, p.hi, (k == 0 || last) ? act_req[j] : -1, last, jobs[j].items);
+      prepare_one(j, k, p.lo, p.hi, (k == 0 || last) ? act_req[j] : -1, last, jobs[j].items, stamp_of(i));
     }
   }
   Inflight inf;
@@ -951,11 +963,13 @@ void Engine::loop_at_arrival(bool unbound) {
         if (!launchers_.empty()) {
           LaunchJob job;
           for (int k = 0; k < m; ++k)
-            prepare_one(j, k, lo, hi, (k == 0 || k == m - 1) ? r : -1, k == m - 1, job.items);
+            prepare_one(j, k, lo, hi, (k == 0 || k == m - 1) ? r : -1, k == m - 1, job.items, k == 0 || k == m - 1);
           push_job(j, std::move(job));
         } else {
           for (int k = 0; k < m; ++k)
-            if (!launch_one(j, k, lo, hi, ten_[j].stream, (k == 0 || k == m - 1) ? r : -1, k == m - 1)) return;
+            if (!launch_one(j, k, lo, hi, ten_[j].stream, (k == 0 || k == m - 1) ? r : -1, k == m - 1,
+                            k == 0 || k == m - 1))
+              return;
         }
         launched = true;
       }

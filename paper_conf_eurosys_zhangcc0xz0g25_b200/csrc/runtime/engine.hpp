@@ -43,6 +43,7 @@ struct TenantRT {
   const void* dev_out = nullptr;
   void* host_out = nullptr;
   size_t out_bytes = 0;
+  uint64_t prev_light = 0;   // last launch on the stream if it used the light exit (owned by its launcher)
 };
 
 // Parallel launch path.  Host launch calls cost ~3 us each on the B200 boxes
@@ -54,6 +55,7 @@ struct TenantRT {
 struct LaunchItem {
   enum Kind : uint8_t { KERNEL = 0, H2D = 1, D2H = 2, MARKER = 3 };
   uint8_t kind = KERNEL;
+  uint8_t stamp = 1;    // full exit protocol (host observes completion); 0 = light exit
   int handle = -1;
   uint64_t seq = 0;
   int lo = 0, hi = 0;
@@ -129,9 +131,10 @@ class Engine {
   void harvest();
   void retire_inflight();
   void launch_squad(const Decision& d, const std::vector<int64_t>& act_req, const std::vector<int>& act_next);
-  uint64_t launch_one(int t, int k, int lo, int hi, void* stream, int64_t req, bool last);
+  uint64_t launch_one(int t, int k, int lo, int hi, void* stream, int64_t req, bool last, bool stamp = true);
   // parallel launch path
-  bool prepare_one(int t, int k, int lo, int hi, int64_t req, bool last, std::vector<LaunchItem>& items);
+  bool prepare_one(int t, int k, int lo, int hi, int64_t req, bool last, std::vector<LaunchItem>& items,
+                   bool stamp = true);
   bool exec_items(int t, const std::vector<LaunchItem>& items, void* stream, std::string& err);
   void push_job(int t, LaunchJob&& job);
   void launcher_main(int t);
