@@ -357,6 +357,23 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   // epilogue constants overlap the previous kernel; only reads of activations
   // (A operand, residual) and writes of the output wait for it.
 
+  // debug experiments (tools/tctrace.py builds): drop one operand's loads or the MMAs
+#ifdef BLESS_TC_SKIP_A
+  constexpr bool kSkipA = true;
+#else
+  constexpr bool kSkipA = false;
+#endif
+#ifdef BLESS_TC_SKIP_B
+  constexpr bool kSkipB = true;
+#else
+  constexpr bool kSkipB = false;
+#endif
+#ifdef BLESS_TC_SKIP_MMA
+  constexpr bool kSkipMma = true;
+#else
+  constexpr bool kSkipMma = false;
+#endif
+  constexpr uint32_t kTxBytes = (kSkipA ? 0u : (uint32_t)Cfg::kStageA) + (kSkipB ? 0u : (uint32_t)Cfg::kStageB);
   if (warp == 0) {
     // ---------------- tile scheduler + TMA producer
     if (lane == 0) {
@@ -422,23 +439,24 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           for (int i = 0; i < npre; ++i) {
             const int st = (stage + i) % ST;
             mbar_wait(&empty[st], (phase ^ (stage + i >= ST ? 1 : 0)) ^ 1);
-            mbar_expect_tx(&full[st], Cfg::kStageBytes);
-            load_B(kb0 + i, st);
+            mbar_expect_tx(&full[st], kTxBytes);
+            if (!kSkipB) load_B(kb0 + i, st);
           }
           pdl_wait();
           if (t == 0) gate_prev_end(g, (int64_t)ptx_globaltimer());   // predecessor just completed
           TR(4);                         // 4: producer past griddepcontrol.wait
           dep_waited = true;
-          for (int i = 0; i < npre; ++i) load_A(kb0 + i, (stage + i) % ST);
+          for (int i = 0; i < npre; ++i)
+            if (!kSkipA) load_A(kb0 + i, (stage + i) % ST);
           for (int i = 0; i < npre; ++i)
             if (++stage == ST) { stage = 0; phase ^= 1; }
           kb = kb0 + npre;
         }
         for (; kb < kb1; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
-          mbar_expect_tx(&full[stage], Cfg::kStageBytes);
-          load_B(kb, stage);
-          load_A(kb, stage);
+          mbar_expect_tx(&full[stage], kTxBytes);
+          if (!kSkipB) load_B(kb, stage);
+          if (!kSkipA) load_A(kb, stage);
           if (++stage == ST) { stage = 0; phase ^= 1; }
         }
       }
@@ -471,17 +489,24 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         if (lane == 0) {
           const uint32_t a0 = smem_u32(sA + stage * Cfg::kStageA);
           const uint32_t b0 = smem_u32(sB + stage * Cfg::kStageB);
+          if (kSkipMma) {
+            mbar_arrive(&empty[stage]);
+          } else {
 #pragma unroll
-          for (int k = 0; k < BK / 16; ++k) {
-            tc_mma(d_tmem, smem_desc<BK>(a0 + k * 32), smem_desc<BK>(b0 + k * 32), idesc,
-                   (kb != kb0 || k) ? 1u : 0u);
+            for (int k = 0; k < BK / 16; ++k) {
+              tc_mma(d_tmem, smem_desc<BK>(a0 + k * 32), smem_desc<BK>(b0 + k * 32), idesc,
+                     (kb != kb0 || k) ? 1u : 0u);
+            }
+            tc_commit(&empty[stage]);
           }
-          tc_commit(&empty[stage]);
         }
         __syncwarp();
         if (++stage == ST) { stage = 0; phase ^= 1; }
       }
-      if (lane == 0) tc_commit(&tfull[acc]);
+      if (lane == 0) {
+        if (kSkipMma) mbar_arrive(&tfull[acc]);
+        else tc_commit(&tfull[acc]);
+      }
       __syncwarp();
       if (++acc == Cfg::kAcc) { acc = 0; aph ^= 1; }
     }
@@ -563,12 +588,24 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty[acc]);  // TMEM no longer needed
+#ifdef BLESS_TC_SPLIT_FENCE_ALL   // A/B reference: every epilogue thread fences its own reds
         __threadfence();
+#endif
+        // release: the CTA barrier orders every epilogue thread's reds before
+        // thread 64's gpu-scope fence (fences are cumulative), which precedes
+        // its arrival on the tile's counter; one fence per unit instead of 256
         asm volatile("bar.sync 1, %0;" ::"n"(32 * kEpiWarps) : "memory");   // all epilogue warps
-        if (threadIdx.x == 64) *last_flag = (atomicAdd(p.sem + tile, 1u) == (unsigned)p.splits - 1) ? 1 : 0;
+        if (threadIdx.x == 64) {
+          __threadfence();
+          const bool last = atomicAdd(p.sem + tile, 1u) == (unsigned)p.splits - 1;
+          if (last) __threadfence();   // acquire: the other units' reds before our ld.cg reads
+          *last_flag = last ? 1 : 0;
+        }
         asm volatile("bar.sync 1, %0;" ::"n"(32 * kEpiWarps) : "memory");
         if (*last_flag) {
+#ifdef BLESS_TC_SPLIT_FENCE_ALL
           __threadfence();
+#endif
           if (valid) TC_ACT_DISPATCH(p.act, (epi_ws<A_>(p, wrow, c0, c1, tn, BN, m, epi_sc, epi_sh)))
           if (threadIdx.x == 64) p.sem[tile] = 0;
         }

@@ -58,7 +58,8 @@ def test_tc_gemm(ctx, M, N, K, act):
 
 @pytest.mark.parametrize("M,N,K,dtype", [(1, 4096, 25088, "bf16"), (1, 1000, 2048, "bf16"), (3, 100, 50, "bf16"),
                                          (2, 1000, 4096, "bf16"), (1, 37, 512, "bf16"), (8, 129, 96, "bf16"),
-                                         (1, 4096, 4096, "fp32"), (8, 64, 1000, "fp32")])
+                                         (1, 4096, 4096, "fp32"), (8, 64, 1000, "fp32"),
+                                         (1, 2050, 256, "bf16"), (2, 4100, 512, "bf16")])
 def test_gemv(ctx, M, N, K, dtype):
     def mk(b):
         x = b.input((M, K))
