@@ -48,6 +48,7 @@ struct TcParams {
   int stages;       // smem pipeline depth (runtime: budget / stage bytes, <= kMaxStages)
   float* ws;        // [tiles][128][BN] fp32 partial sums (zero between launches)
   unsigned* sem;    // [tiles] arrival counters (zero between launches)
+  int sk_tiles;     // output tiles (workspace layout)
 };
 
 #ifdef __CUDACC__
@@ -57,7 +58,7 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)_
 // Debug builds only (-DBLESS_TC_TRACE, tools/tctrace.py): per-CTA %globaltimer
 // stamps of the pipeline phases of the last launch.
 #ifdef BLESS_TC_TRACE
-constexpr int kTrMax = 2048, kTrN = 10;
+constexpr int kTrMax = 2048, kTrN = 12;
 __device__ unsigned long long g_tc_trace[kTrMax][kTrN];
 __device__ __forceinline__ void tr_mark(int i) {
   unsigned long long t;
@@ -252,19 +253,32 @@ __device__ __forceinline__ void epi_cols(const TcParams& p, uint32_t tbase, int 
   }
 }
 
+// Split-K fp32 workspace layout: [tile][BN/16 column chunks][4 float4
+// groups][128 rows][float4].  A thread owns one row (TMEM lane), so the four
+// float4 of its 16-column chunk lie 2 KB apart and the 32 rows of a warp
+// store/load 512 contiguous bytes per instruction (full sectors; the former
+// row-major [row][BN] layout cost 32 partial-sector transactions per warp
+// instruction and made the split-K epilogue ~4 us per 64 KB tile).
+__device__ __forceinline__ float4* ws_at(const TcParams& p, int slab, int tile, int c, int i, int row, int BN) {
+  const size_t chunk = ((size_t)slab * p.sk_tiles + tile) * (size_t)(BN >> 4) + (size_t)(c >> 4);
+  return reinterpret_cast<float4*>(p.ws) + (chunk * 4 + i) * 128 + row;
+}
+
 template <int ACT>
-__device__ __forceinline__ void epi_ws(const TcParams& p, const float* wrow, int c0, int c1, int tn, int BN, int m,
+__device__ __forceinline__ void epi_ws(const TcParams& p, int tile, int row, int c0, int c1, int tn, int BN, int m,
                                        const float* sc, const float* sh) {
 #pragma unroll 1
   for (int c = c0; c < c1; c += 16) {
     const int n0 = tn * BN + c;
     if (n0 >= p.N) break;
     float y[16];
+    float4 f[4];
 #pragma unroll
-    for (int i = 0; i < 16; i += 4) {
-      float4 f = __ldcg(reinterpret_cast<const float4*>(wrow + c + i));
-      y[i] = f.x; y[i + 1] = f.y; y[i + 2] = f.z; y[i + 3] = f.w;
-      __stcg(reinterpret_cast<float4*>(const_cast<float*>(wrow) + c + i), make_float4(0.f, 0.f, 0.f, 0.f));
+    for (int i = 0; i < 4; ++i) f[i] = __ldcg(ws_at(p, 0, tile, c, i, row, BN));
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {   // re-zero for the next launch (after all four loads are issued)
+      y[4 * i] = f[i].x; y[4 * i + 1] = f[i].y; y[4 * i + 2] = f[i].z; y[4 * i + 3] = f[i].w;
+      __stcg(ws_at(p, 0, tile, c, i, row, BN), make_float4(0.f, 0.f, 0.f, 0.f));
     }
     epi_store16<ACT>(p, m, n0, y, sc + c, sh + c);
   }
@@ -572,7 +586,6 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         if (threadIdx.x == 64) TR(7);    // 7: epilogue stores issued (last tile)
       } else {
         // split-K: add this unit's partial tile into the fp32 workspace
-        float* wrow = p.ws + ((size_t)tile * 128 + row) * BN;
 #pragma unroll 1
         for (int c = c0; c < c1; c += 16) {
           uint32_t v[16];
@@ -580,14 +593,16 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           tmem_ld_wait();
           if (!valid || tn * BN + c >= p.N) continue;
 #pragma unroll
-          for (int i = 0; i < 16; i += 4)
-            asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(wrow + c + i), "f"(__uint_as_float(v[i])),
-                         "f"(__uint_as_float(v[i + 1])), "f"(__uint_as_float(v[i + 2])), "f"(__uint_as_float(v[i + 3]))
+          for (int i = 0; i < 4; ++i)
+            asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(ws_at(p, 0, tile, c, i, row, BN)),
+                         "f"(__uint_as_float(v[4 * i])), "f"(__uint_as_float(v[4 * i + 1])),
+                         "f"(__uint_as_float(v[4 * i + 2])), "f"(__uint_as_float(v[4 * i + 3]))
                          : "memory");
         }
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty[acc]);  // TMEM no longer needed
+        if (threadIdx.x == 64) TR(7);      // 7: partial-sum reds issued (split-K)
 #ifdef BLESS_TC_SPLIT_FENCE_ALL   // A/B reference: every epilogue thread fences its own reds
         __threadfence();
 #endif
@@ -600,14 +615,18 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           const bool last = atomicAdd(p.sem + tile, 1u) == (unsigned)p.splits - 1;
           if (last) __threadfence();   // acquire: the other units' reds before our ld.cg reads
           *last_flag = last ? 1 : 0;
+          TR(10);                          // 10: fence + tile counter arrival done (split-K)
         }
         asm volatile("bar.sync 1, %0;" ::"n"(32 * kEpiWarps) : "memory");
         if (*last_flag) {
 #ifdef BLESS_TC_SPLIT_FENCE_ALL
           __threadfence();
 #endif
-          if (valid) TC_ACT_DISPATCH(p.act, (epi_ws<A_>(p, wrow, c0, c1, tn, BN, m, epi_sc, epi_sh)))
-          if (threadIdx.x == 64) p.sem[tile] = 0;
+          if (valid) TC_ACT_DISPATCH(p.act, (epi_ws<A_>(p, tile, row, c0, c1, tn, BN, m, epi_sc, epi_sh)))
+          if (threadIdx.x == 64) {
+            p.sem[tile] = 0;
+            TR(11);                        // 11: last unit's reduction epilogue done (split-K)
+          }
         }
       }
       if (++acc == Cfg::kAcc) { acc = 0; aph ^= 1; }
@@ -829,6 +848,9 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   p.splits = (p.num_kb + p.kbs - 1) / p.kbs;
   if (p.splits > 1) {
     const size_t nt = (size_t)ntiles(BN);
+    // (a per-unit fp32 slab variant -- plain stores summed by the last unit --
+    // was no faster on B200 and slower beyond 3 splits, profiles/round1/tc_splitk_*)
+    p.sk_tiles = (int)nt;
     const size_t wsb = nt * 128 * BN * sizeof(float);
     void* buf = nullptr;
     if (cudaMalloc(&buf, wsb + nt * sizeof(unsigned)) != cudaSuccess ||

@@ -18,7 +18,8 @@ import numpy as np
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
-NAMES = ["start", "entry", "setup", "claim", "pdl_wait", "stage0", "acc_ready", "epi_done", "work_done", "exit"]
+NAMES = ["start", "entry", "setup", "claim", "pdl_wait", "stage0", "acc_ready", "epi_done", "work_done", "exit",
+         "sk_arrived", "sk_reduced"]   # 10/11: split-K units only
 
 
 def main():
@@ -44,7 +45,7 @@ def main():
     for reps in (1, 20):
         L.bl_debug_tc_trace_clear()
         ns, _ = ctx.profile_kernel(t, 0, S, reps)
-        buf = np.zeros((2048, 10), dtype=np.uint64)
+        buf = np.zeros((2048, 12), dtype=np.uint64)
         L.bl_debug_tc_trace(buf.ctypes.data, 2048)
         v = buf.astype(np.int64)
         ok = (v[:, 0] > 0) & (v[:, 1] >= v[:, 0]) & (v[:, 9] >= v[:, 1]) & (v[:, 7] > 0)
