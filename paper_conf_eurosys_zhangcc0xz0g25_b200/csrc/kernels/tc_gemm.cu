@@ -236,6 +236,10 @@ __device__ __forceinline__ void epi_store16(const TcParams& p, int m, int n0, fl
 
 // Unsplit epilogue of one row (m) over this warp's columns [c0, c1) of the
 // tile: TMEM -> registers (16 columns per wait) -> fused epilogue -> bf16.
+// (Measured on B200, profiles/round1/tc_epilogue_ab.txt: the global stores
+// cost ~2-3 us per 128x128 tile (-DBLESS_TC_NOSTORE: ffn1 12.8 -> 9.4 us), but
+// warp-staging them through shared memory into full-sector row stores did not
+// change the time, so the per-thread row stores stay.)
 template <int ACT>
 __device__ __forceinline__ void epi_cols(const TcParams& p, uint32_t tbase, int c0, int c1, int tn, int BN, int m,
                                          bool valid, const float* sc, const float* sh) {
