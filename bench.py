@@ -60,6 +60,8 @@ def parse():
     ap.add_argument("--impl", default="native", choices=["native", "reference"])
     ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4", "C5"])
     ap.add_argument("--rho", type=float, default=0.5, help="per-tenant load relative to its ISO latency")
+    ap.add_argument("--rhos", default="", help="comma list: per-tenant rho (PAPER.md L298 workload E, biased load)")
+    ap.add_argument("--quotas", default="", help="comma list: per-tenant quota override (PAPER.md Table 2 quota sets)")
     ap.add_argument("--requests", type=int, default=60, help="requests per tenant per step")
     # B200 operating point chosen by the c% x S_max sweep, the
     # way the paper picks its own empirically (§6.7).
@@ -67,6 +69,8 @@ def parse():
                     help="S_max (L406-L408); default per config from the B200 sweeps in "
                          "profiles/round1/param_sweep: C1 4, C2 20, C3 10, C4 10")
     ap.add_argument("--split-pct", type=int, default=25)
+    ap.add_argument("--ablate", type=int, default=0,
+                    help="PAPER.md §6.8 ablation (R32): 1 = no multi-task scheduler, 2 = no determiner, 3 = both")
     ap.add_argument("--lookahead-us", type=float, default=20.0)
     ap.add_argument("--max-inflight", type=int, default=2)
     ap.add_argument("--profile-reps", type=int, default=5)
@@ -176,8 +180,10 @@ def squad_timeline(decisions, launches):
 
 def make_trace(T_iso, rho, n, seed, bursty=False):
     """Poisson (C1-C3, C5) or bursty MMPP-2 (C4: ON 20% at 4x, OFF at 0.25x the
-    mean rate, exponential dwell 20 / 80 ms) per tenant."""
-    gaps = [T / rho for T in T_iso]
+    mean rate, exponential dwell 20 / 80 ms) per tenant.
+    ``rho`` is one load for every tenant or a per-tenant list."""
+    rhos = list(rho) if isinstance(rho, (list, tuple)) else [rho] * len(T_iso)
+    gaps = [T / r for T, r in zip(T_iso, rhos)]
     if bursty:
         return syntrace.mmpp2(gaps, n, seed)
     return syntrace.poisson(gaps, n, seed)
@@ -277,7 +283,9 @@ def native(args):
     ctx = capi.Ctx(local, params)
     info = ctx.device_info()
     S = info.sm_count
-    tms = models.build_config(ctx, args.config, dtype)
+    quotas = [float(x) for x in args.quotas.split(",")] if args.quotas else None
+    tms = models.build_config(ctx, args.config, dtype, quotas)
+    rho = [float(x) for x in args.rhos.split(",")] if args.rhos else args.rho
     names = [m.name for m in tms]
     t_prof = time.perf_counter()
     if args.load_profile:
@@ -295,10 +303,10 @@ def native(args):
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 
     def step(seed, pol="BLESS", filt=None, extra=None):
-        p = capi.default_params(squad_max=args.squad_max, policy=pol, split_pct=args.split_pct,
+        p = capi.default_params(squad_max=args.squad_max, policy=pol, split_pct=args.split_pct, ablate=args.ablate,
                                 lookahead_ns=int(args.lookahead_us * 1000), max_inflight_squads=args.max_inflight,
                                 **(extra or {}))
-        return run_policy(ctx, capi, p, make_trace(T_iso, args.rho, args.requests, seed + plan.trace_seed_offset,
+        return run_policy(ctx, capi, p, make_trace(T_iso, rho, args.requests, seed + plan.trace_seed_offset,
                                                    args.config == "C4"), filt)
 
     for w in range(args.warmup):
@@ -524,7 +532,7 @@ def native(args):
         prof = Prof(synprof.load(prof_path))
         sq = len(decisions_all) / max(1, n_local)
         cpu = oracle_timing(names, decisions_all, prof, [len(lat_all[j]) for j in range(len(tms))], sq * 2,
-                            Params(squad_max=args.squad_max, split_pct=args.split_pct))
+                            Params(squad_max=args.squad_max, split_pct=args.split_pct, ablate=args.ablate))
 
     # decisions replayed bit-exactly through the oracle (sample)
     replay_ok = None
@@ -534,7 +542,7 @@ def native(args):
         replay_ok = 0
         for rec in decisions_all[:200]:
             got = capi.decision_to_tuple(rec)
-            ref = decide_ref(got["now"], [Active(*a) for a in got["active"]], prof, Params(squad_max=args.squad_max, split_pct=args.split_pct))
+            ref = decide_ref(got["now"], [Active(*a) for a in got["active"]], prof, Params(squad_max=args.squad_max, split_pct=args.split_pct, ablate=args.ablate))
             replay_ok += int(got["picks"] == [tuple(p) for p in ref.picks] and got["config"] == ref.config
                              and got["t_hat"] == ref.t_hat)
         replay_ok = f"{replay_ok}/{min(200, len(decisions_all))}"
@@ -547,9 +555,11 @@ def native(args):
         "warmup": args.warmup, "ms_per_step": step_ms, "higher_is_better": False, "scaling": "weak",
         "vs_baseline": None, "dtype": "bf16" if dtype == "bf16" else "f32", "data": "synthetic",
         "config": {"workload": f"{args.config}: {CONFIG_NAMES[args.config]}",
-                   "trace": f"{'MMPP-2 bursty' if args.config == 'C4' else 'Poisson'} rho={args.rho} "
+                   "trace": f"{'MMPP-2 bursty' if args.config == 'C4' else 'Poisson'} rho={args.rhos or args.rho} "
                    f"per tenant, {args.requests} requests/tenant/step, seeds 1-3", "squad_max": args.squad_max,
-                   "split_pct": args.split_pct, "parallelism": f"replicas x{world} (no collective)",
+                   "split_pct": args.split_pct, "ablate": args.ablate,
+                   "parallelism": f"replicas x{world} (no collective)",
+                   "quotas": [m.quota for m in tms],
                    "l2": "256 MiB buffer written between timed steps (> 126 MB L2); VGG11 weights 266 MB > L2"},
         "per_tenant": per_tenant, "baselines": base, "slo": slo, "requests_per_s": n_req / (step_ms * args.steps / 1e3),
         "e2e": e2e, "gpu_launches": gpu_launches, "roofline": roofline, "cpu_baseline": cpu,
@@ -594,7 +604,7 @@ def reference(args):
     for it in range(args.warmup + args.steps):
         t0 = time.perf_counter()
         trace = make_trace(prof.T, args.rho, max(4, args.requests // 10), 1 + it % 3, cfg == "C4")
-        res = des.run_bless(trace, prof, Params(squad_max=args.squad_max, split_pct=args.split_pct))
+        res = des.run_bless(trace, prof, Params(squad_max=args.squad_max, split_pct=args.split_pct, ablate=args.ablate))
         t_dec = time.perf_counter() - t0
         fw = {}
         for i, n in enumerate(names):

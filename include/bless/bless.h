@@ -96,6 +96,13 @@ typedef struct {
   int64_t lookahead_ns;       /* WALL: decide the next squad this long before the
                                  predicted end of the in-flight one (default 20 us) */
   int64_t max_requests;       /* request-table capacity (default 1<<20) */
+  int32_t ablate;             /* §6.8 ablation study (L424-L426, reading R32; default 0):
+                                 bit 0 = no multi-task scheduler (picks round-robin over
+                                 the active requests, one kernel each per round, no
+                                 progress order); bit 1 = no execution configuration
+                                 determiner (every squad NSP on [0,S)).  BL_E_INVALID
+                                 outside 0..3 at bl_create. */
+  int32_t reserved0;          /* 0 */
 } bl_params;
 
 /* Fill *p with the defaults listed above. */

@@ -114,11 +114,16 @@ class Params:
     split_pct: int = 50        # Semi-SP split ratio c% (L255, L410; R16)
     seed_all: bool = True      # every active request seeded first (R6)
     squad_overhead_ns: int = 0  # DES only: GPU idle per squad switch (L432)
+    # Ablation (§6.8; reading R32): bit 0 = no multi-task scheduler
+    # (picks taken round-robin over the active requests in tenant-id order,
+    # one kernel each per round, no progress ordering); bit 1 = no execution
+    # configuration determiner (no search: every squad runs NSP on [0, S)).
+    ablate: int = 0
 
     @staticmethod
     def from_dict(d: dict) -> "Params":
         return Params(int(d.get("squad_max", 50)), int(d.get("split_pct", 50)),
-                      bool(d.get("seed_all", True)), int(d.get("squad_overhead_ns", 0)))
+                      bool(d.get("seed_all", True)), int(d.get("squad_overhead_ns", 0)), int(d.get("ablate", 0)))
 
 
 @dataclass(frozen=True)
@@ -189,6 +194,17 @@ def generate_squad(now: int, active: Sequence[Active], prof: Prof, params: Param
 
     closed = False
     tenants = sorted(nxt)
+    if params.ablate & 1:
+        # §6.8 "BLESS without the multi-task scheduler can not dynamically
+        # control the kernel number from each active request" (L426): equal
+        # shares, one kernel per active request per round, tenant-id order;
+        # the same closing rules (R5, R7).
+        while not closed:
+            for j in tenants:
+                if nxt[j] < prof.m[j] and pick(j):
+                    closed = True
+                    break
+        return picks
     if params.seed_all and len(tenants) >= 2:             # R6
         for j in sorted(tenants, key=key):
             if pick(j):
@@ -270,7 +286,7 @@ def compositions(N: int, K: int) -> Iterator[Tuple[int, ...]]:
             yield (first,) + rest
 
 
-def choose_config(ks: Dict[int, List[int]], prof: Prof) -> Tuple[Optional[Tuple[int, ...]], int, int]:
+def choose_config(ks: Dict[int, List[int]], prof: Prof, search: bool = True) -> Tuple[Optional[Tuple[int, ...]], int, int]:
     """argmin over {NSP} U {all strict spatial splits} (L205, L237).
 
     R13: NSP is the incumbent and is replaced only by a strictly smaller
@@ -282,7 +298,7 @@ def choose_config(ks: Dict[int, List[int]], prof: Prof) -> Tuple[Optional[Tuple[
     t_nsp, _ = predict_nsp(ks, prof)
     K = len(ks)
     best, best_t = None, t_nsp
-    if K >= 2:
+    if K >= 2 and search:   # search = False: the §6.8 ablation without the determiner (R32)
         parts = sorted(ks)
         memo: Dict[Tuple[int, int], int] = {}   # (participant, s) -> sum_i t[k_i][s]; same Eq. 1 terms
 
@@ -335,7 +351,7 @@ def decide_ref(now: int, active: Sequence[Active], prof: Prof, params: Params) -
     picks = generate_squad(now, act, prof, params)
     ks = per_participant(picks)
     parts = sorted(ks)
-    config, t_hat, t_nsp = choose_config(ks, prof)
+    config, t_hat, t_nsp = choose_config(ks, prof, search=not (params.ablate & 2))
     ranged = semi_sp_ranges(picks, parts, config, prof, params.split_pct)
     if config is None:
         _, ends = predict_nsp(ks, prof)

@@ -194,7 +194,15 @@ void decide(int64_t now, const ActiveReq* act, int n_act, const Profile& prof, c
     return (int)out.picks.size() >= prm.squad_max || k == (int)prof.ten[j].k.size() - 1;  // R5, R7
   };
   bool closed = false;
-  if (prm.seed_all && tenants.size() >= 2) {  // R6
+  if (prm.ablate & 1) {
+    // §6.8 ablation (L426, R32): no multi-task scheduler -- one kernel per
+    // active request per round in tenant-id order, same closing rules
+    while (!closed) {
+      for (int j : tenants)
+        if (sc.nxt[j] < (int)prof.ten[j].k.size() && pick(j)) { closed = true; break; }
+    }
+  }
+  if (!closed && prm.seed_all && tenants.size() >= 2) {  // R6
     std::vector<int> seed = tenants;
     std::sort(seed.begin(), seed.end(), [&](int x, int y) { return ord.more_behind(x, y); });
     for (int j : seed)
@@ -249,8 +257,9 @@ void decide(int64_t now, const ActiveReq* act, int n_act, const Profile& prof, c
   out.sp = false;
   out.p.clear();
 
-  // Eq. 1 (L211) over all compositions by exact DP over suffixes (R9-R14).
-  if (K >= 2) {
+  // Eq. 1 (L211) over all compositions by exact DP over suffixes (R9-R14);
+  // skipped by the §6.8 ablation without the determiner (R32: always NSP).
+  if (K >= 2 && !(prm.ablate & 2)) {
     const int W = N + 1;
     sc.Sj.assign((size_t)K * W, 0);
     sc.F.assign((size_t)K * W, INT64_MAX);

@@ -62,6 +62,7 @@ struct SchedParams {
   int squad_max = 50;   // R5
   int split_pct = 50;   // R16
   bool seed_all = true; // R6
+  int ablate = 0;       // §6.8 ablation (R32): bit0 no multi-task scheduler, bit1 no determiner
 };
 
 struct ActiveReq {

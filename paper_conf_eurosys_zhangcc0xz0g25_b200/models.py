@@ -14,7 +14,7 @@ Layouts: activations NHWC, conv weights KRSC, GEMM weights [N, K].
 from __future__ import annotations
 
 from dataclasses import dataclass, field
-from typing import Dict, List, Optional
+from typing import Dict, List, Optional, Sequence
 
 import numpy as np
 import torch
@@ -427,9 +427,16 @@ CONFIGS = {
 }
 
 
-def build_config(ctx: capi.Ctx, cfg: str, dtype: str) -> List[TenantModel]:
+def build_config(ctx: capi.Ctx, cfg: str, dtype: str, quotas: Optional[Sequence[float]] = None) -> List[TenantModel]:
+    """Register and build the tenants of a config; ``quotas`` overrides the
+    config's quota per tenant (Table 2's two-model quota sets, L295)."""
     models = []
-    for i, (name, q) in enumerate(CONFIGS[cfg]):
+    spec = CONFIGS[cfg]
+    if quotas is not None:
+        if len(quotas) != len(spec):
+            raise ValueError(f"{cfg} has {len(spec)} tenants, got {len(quotas)} quotas")
+        spec = [(name, float(q)) for (name, _), q in zip(spec, quotas)]
+    for i, (name, q) in enumerate(spec):
         t = ctx.register_tenant(q, name)
         models.append(BUILDERS[name](ctx, t, q, dtype=dtype, seed=1000 + i))
     return models

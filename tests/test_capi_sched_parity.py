@@ -120,7 +120,7 @@ def world(draw):
     active = [(j, draw(st.integers(0, 300)), draw(st.integers(0, m[j] - 1))) for j in who]
     now = draw(st.integers(0, 1500))
     params = dict(squad_max=draw(st.integers(1, 12)), split_pct=draw(st.sampled_from([0, 30, 50, 75, 100])),
-                  seed_all=int(draw(st.booleans())))
+                  seed_all=int(draw(st.booleans())), ablate=draw(st.sampled_from([0, 0, 1, 2, 3])))
     return pf, active, now, params
 
 
@@ -131,7 +131,8 @@ def test_decide_bit_exact_small(tmp_path_factory, w):
     tmp = tmp_path_factory.mktemp("d")
     ctx = _ctx_from(pf, tmp, **params)
     ref = decide_ref(now, [Active(*a) for a in active], Prof(pf),
-                     Params(params["squad_max"], params["split_pct"], bool(params["seed_all"])))
+                     Params(params["squad_max"], params["split_pct"], bool(params["seed_all"]),
+                            ablate=params["ablate"]))
     assert _cpp_tuple(ctx.decide(now, active)) == _ref_tuple(ref)
     ctx.close()
 
@@ -172,7 +173,7 @@ def _virtual_run(ctx, trace):
     return recs, out
 
 
-@pytest.mark.parametrize("case", ["fig1_like", "c3_like", "random_small"])
+@pytest.mark.parametrize("case", ["fig1_like", "c3_like", "random_small", "ablate_sched", "ablate_both"])
 def test_whole_trace_virtual_bit_exact(tmp_path, case):
     """Whole trace, VIRTUAL clock (R17): every decision record (now, admitted
     set, picks, config, SM ranges, predictions) and every model completion time
@@ -190,6 +191,13 @@ def test_whole_trace_virtual_bit_exact(tmp_path, case):
                    for j, (q, m) in enumerate(zip([400000, 300000, 200000, 100000], [55, 21, 30, 25]))]
         params = dict(squad_max=50, split_pct=50, seed_all=1, squad_overhead_ns=2000)
         n = 10
+    elif case.startswith("ablate"):   # §6.8 ablation (R32) on a C2-like pair
+        S, g = 148, 4
+        tenants = [sp.random_tenant("vgg", 333333, 16, S, rng, 5e5, 0.85, 0.1, 1500),
+                   sp.random_tenant("r50", 666667, 55, S, rng, 3e5, 0.85, 0.1, 1500)]
+        params = dict(squad_max=20, split_pct=25, seed_all=1, squad_overhead_ns=2000,
+                      ablate=1 if case == "ablate_sched" else 3)
+        n = 20
     else:
         S, g = 16, 4
         tenants = [sp.random_tenant(f"t{j}", q, m, S, rng, 2e4, 0.5, 0.3, 200)
@@ -202,7 +210,7 @@ def test_whole_trace_virtual_bit_exact(tmp_path, case):
     ctx = _ctx_from(pf, tmp_path, **params)
     recs, fin = _virtual_run(ctx, trace)
     ref = des.run_bless(trace, prof, Params(params["squad_max"], params["split_pct"], bool(params["seed_all"]),
-                                            params["squad_overhead_ns"]))
+                                            params["squad_overhead_ns"], params.get("ablate", 0)))
     assert len(recs) == len(ref.decisions)
     for i, (r, d) in enumerate(zip(recs, ref.decisions)):
         got = capi.decision_to_tuple(r)

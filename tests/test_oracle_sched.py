@@ -332,3 +332,36 @@ def test_iso_lindley_closed_form():
     trace = [tr.Arrival(0, 0), tr.Arrival(50, 0), tr.Arrival(1000, 0)]
     r = des.run_iso(trace, prof)
     assert [r.finish[i] for i in range(3)] == [T, 2 * T, 1000 + T]
+
+
+# --------------------------------------------------------------------------- §6.8 ablation (R32)
+def test_ablation_without_scheduler_round_robin():
+    """PAPER.md §6.8: without the multi-task scheduler BLESS "can not
+    dynamically control the kernel number from each active request" -- reading
+    R32: one kernel per active request per round in tenant-id order, the same
+    closing rules (R5 cap, R7 last kernel).  Hand-derived on fixture E3:
+    progress would pick b1 first at now = 1000 (B is further behind), the
+    ablation takes A's kernel first and A's last kernel closes the squad."""
+    fx = load_golden("e3_squad_generation.json")
+    prof = Prof(golden_profile(fx))
+    p = Params(squad_max=fx["squad_max"], seed_all=True, ablate=1)
+    assert generate_squad(0, [Active(0, 0, 0), Active(1, 0, 0)], prof, p) == [(0, 0), (1, 0), (0, 1), (1, 1)]
+    assert generate_squad(1000, [Active(0, 0, 3), Active(1, 0, 1)], prof, p) == [(0, 3)]
+    # a single active request: its kernels in order up to the cap
+    assert generate_squad(0, [Active(1, 0, 0)], prof, p) == [(1, 0), (1, 1), (1, 2), (1, 3)]
+
+
+def test_ablation_without_determiner_is_nsp():
+    """§6.8 L426 without the execution configuration determiner (reading R32:
+    no search, every squad NSP on [0, S)).  Fixture E2 picks the split (2, 2)
+    with t_hat 400 when searching; without the determiner the squad is NSP
+    with the Eq. 2 prediction 525 and every range is the full GPU."""
+    fx = load_golden("e2_sp_wins.json")
+    prof = Prof(golden_profile(fx))
+    ks = {int(j): v for j, v in fx["squad"].items()}
+    assert choose_config(ks, prof)[0] == tuple(fx["expected"]["config"])
+    config, t_hat, t_nsp = choose_config(ks, prof, search=False)
+    assert config is None and t_hat == t_nsp == fx["expected"]["nsp"]
+    picks = [tuple(p) for p in fx["picks_order"]]
+    assert all((lo, hi) == (0, prof.S) for _, _, lo, hi in semi_sp_ranges(picks, sorted(ks), config, prof,
+                                                                            fx["split_pct"]))
