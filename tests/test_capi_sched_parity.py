@@ -220,3 +220,10 @@ def test_whole_trace_virtual_bit_exact(tmp_path, case):
     for i in range(len(trace)):
         assert fin[i] == (ref.start[i], ref.finish[i]), i
     ctx.close()
+
+
+def test_ablate_out_of_range_rejected():
+    """bl_params.ablate outside 0..3 is BL_E_INVALID at bl_create (header)."""
+    with pytest.raises(capi.BlessError) as e:
+        capi.Ctx(capi.BL_DEVICE_NONE, clock=capi.BL_CLOCK_VIRTUAL, ablate=4)
+    assert e.value.status == capi.BL_E_INVALID

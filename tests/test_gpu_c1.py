@@ -98,13 +98,14 @@ def _run_trace(ctx, trace, t_base):
     return ids
 
 
-@pytest.mark.parametrize("dtype", ["fp32", "bf16"])
-def test_c1_bless_wall_replay_bit_exact(lib_built, dtype, tmp_path):
+@pytest.mark.parametrize("dtype,ablate", [("fp32", 0), ("bf16", 0), ("fp32", 1), ("fp32", 2)])
+def test_c1_bless_wall_replay_bit_exact(lib_built, dtype, ablate, tmp_path):
     """C1 end to end under BLESS on the wall clock: every request completes,
     every decision replays bit-exactly through decide_ref, all restricted
     kernels stay inside their windows, and the whole-model output matches the
-    fp64 oracle forward (fp32: 1e-4, bf16: 1e-2 per layer)."""
-    ctx = capi.Ctx(0, squad_max=4)
+    fp64 oracle forward (fp32: 1e-4, bf16: 1e-2 per layer).  ablate 1/2: the
+    §6.8 ablation variants (reading R32) replay bit-exactly as well."""
+    ctx = capi.Ctx(0, squad_max=4, ablate=ablate)
     ms = models.build_config(ctx, "C1", dtype)
     for m in ms:
         ctx.profile_tenant(m.tenant, reps=5)
@@ -123,7 +124,7 @@ def test_c1_bless_wall_replay_bit_exact(lib_built, dtype, tmp_path):
         assert st == capi.BL_OK and info.finish_ns > info.arrival_ns
     recs = ctx.decisions()
     assert recs
-    pr = Params(squad_max=4)
+    pr = Params(squad_max=4, ablate=ablate)
     for i, rec in enumerate(recs):
         got = capi.decision_to_tuple(rec)
         ref = decide_ref(got["now"], [Active(*a) for a in got["active"]], prof, pr)
