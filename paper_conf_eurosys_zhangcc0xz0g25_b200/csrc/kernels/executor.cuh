@@ -44,6 +44,7 @@
 // tail of its predecessor on the tenant's stream.
 #pragma once
 #include <cstdint>
+#include <cstdlib>
 
 namespace bless {
 
@@ -253,11 +254,19 @@ __device__ __forceinline__ void gated_run(const typename Op::Params& p, const Ga
 // Host: launch with programmatic stream serialization (PDL) unless disabled.
 extern int g_use_pdl;
 #ifdef __CUDACC__
-// Grid = S x (resident blocks per SM for this kernel), capped at 8 per SM.
-inline int full_occupancy_grid(const void* fn, int block, size_t smem, int S) {
+// Grid = S x (resident blocks per SM for this kernel), capped at 8 per SM and
+// at the kernel's own cap (small-work SIMT kernels run faster with fewer CTAs:
+// fewer claims on the tile queue and fewer idle CTAs to launch and retire).
+inline int full_occupancy_grid(const void* fn, int block, size_t smem, int S, int max_occ = 8) {
   int occ = 1;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, block, smem) != cudaSuccess || occ < 1) occ = 1;
-  return S * (occ > 8 ? 8 : occ);
+  static const int cap = [] {   // BLESS_MAX_OCC: blocks-per-SM cap (sweeps; default 8)
+    const char* e = std::getenv("BLESS_MAX_OCC");
+    const int v = e ? std::atoi(e) : 8;
+    return v < 1 ? 1 : (v > 8 ? 8 : v);
+  }();
+  const int c = cap < max_occ ? cap : max_occ;
+  return S * (occ > c ? c : occ);
 }
 inline cudaError_t launch_kernel(const void* fn, dim3 grid, dim3 block, size_t smem, cudaStream_t st, void** args) {
   cudaLaunchConfig_t cfg = {};

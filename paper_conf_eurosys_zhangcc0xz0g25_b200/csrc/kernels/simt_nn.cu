@@ -335,7 +335,7 @@ __global__ void __launch_bounds__(256) k_nn(const typename Op::Params p, const G
 template <class Op>
 static cudaError_t launch_nn(const KernelDesc& d, const GateArgs& g, cudaStream_t st) {
   void* args[2] = {(void*)d.params, (void*)&g};
-  return launch_kernel((const void*)k_nn<Op>, dim3(d.grid), dim3(d.block), (size_t)d.smem, st, args);
+  return launch_kernel((const void*)k_nn<Op>, dim3(launch_grid(d, g)), dim3(d.block), (size_t)d.smem, st, args);
 }
 
 template <class Op>
@@ -391,6 +391,7 @@ bool build_nn(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::strin
     std::memcpy(d.params, &p, sizeof(p));
     use_nn<LayerNorm>(d);
     d.family = p.embed ? "embed_ln_bf16" : "layernorm_bf16";
+    d.max_occ = 1;   // B200 sweep: fastest with 1 CTA/SM (profiles/round1/occ_cap.txt)
     d.bytes = 2.0 * p.rows * p.C * (p.R ? 3 : 2);
     return true;
   }
@@ -446,6 +447,7 @@ bool build_nn(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::strin
     std::memcpy(d.params, &p, sizeof(p));
     use_nn<DwConv>(d);
     d.family = "dwconv_bf16";
+    d.max_occ = 1;   // B200 sweep: fastest with 1 CTA/SM (profiles/round1/occ_cap.txt)
     d.flops = 2.0 * p.OH * p.OW * p.C * p.R_ * p.S_;
     d.bytes = 2.0 * ((double)p.H * p.Wd * p.C + (double)p.OH * p.OW * p.C * (p.R ? 2 : 1));
     return true;
@@ -470,6 +472,7 @@ bool build_nn(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::strin
   std::memcpy(d.params, &p, sizeof(p));
   use_nn<Eltwise>(d);
   d.family = "eltwise_bf16";
+  d.max_occ = 1;   // B200 sweep: fastest with 1 CTA/SM (profiles/round1/occ_cap.txt)
   d.bytes = 2.0 * p.rows * p.C * (p.R ? 3 : 2);
   return true;
 }

@@ -253,7 +253,11 @@ int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
   std::unique_ptr<KernelDesc> kd(new KernelDesc());
   if (!build_kernel(op, caps_, *kd, err)) return -1;
   // grid = S x (resident blocks per SM): see gate_linger in executor.cuh
-  if (kd->kernel_fn) kd->grid = full_occupancy_grid(kd->kernel_fn, kd->block, (size_t)kd->smem, caps_.S);
+  if (kd->kernel_fn) {
+    kd->grid = full_occupancy_grid(kd->kernel_fn, kd->block, (size_t)kd->smem, caps_.S, kd->max_occ);
+    kd->grid_full = full_occupancy_grid(kd->kernel_fn, kd->block, (size_t)kd->smem, caps_.S);
+    kd->S = caps_.S;
+  }
   if (kd->choice_bn && autotune_ && !std::getenv("BLESS_TC_CFG")) {
     const std::string sig = tc_signature(op);
     auto it = tune_cache_.find(sig);
@@ -262,7 +266,9 @@ int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
         std::unique_ptr<KernelDesc> k2(new KernelDesc());
         std::string e2;
         if (build_tc_gemm(op, caps_, *k2, e2, &it->second)) {
-          k2->grid = full_occupancy_grid(k2->kernel_fn, k2->block, (size_t)k2->smem, caps_.S);
+          k2->grid = full_occupancy_grid(k2->kernel_fn, k2->block, (size_t)k2->smem, caps_.S, k2->max_occ);
+          k2->grid_full = full_occupancy_grid(k2->kernel_fn, k2->block, (size_t)k2->smem, caps_.S);
+          k2->S = caps_.S;
           if (kd->owned) cudaFree(kd->owned);
           kd = std::move(k2);
         }
@@ -320,7 +326,9 @@ bool DeviceRT::autotune_tc(const bl_op& op, std::unique_ptr<KernelDesc>& best, s
       if (kd->owned) cudaFree(kd->owned);
       continue;
     }
-    kd->grid = full_occupancy_grid(kd->kernel_fn, kd->block, (size_t)kd->smem, caps_.S);
+    kd->grid = full_occupancy_grid(kd->kernel_fn, kd->block, (size_t)kd->smem, caps_.S, kd->max_occ);
+    kd->grid_full = full_occupancy_grid(kd->kernel_fn, kd->block, (size_t)kd->smem, caps_.S);
+    kd->S = caps_.S;
     kernels_.push_back(std::move(kd));
     const int h = (int)kernels_.size() - 1;
     int64_t ns = 0;

@@ -23,6 +23,9 @@ struct KernelDesc {
   const char* family = "";
   uint32_t tiles = 1;
   int grid = 0, block = 0, smem = 0;
+  int max_occ = 8;         // blocks-per-SM cap of the grid (measured per family, profiles/round1/occ_cap.txt)
+  int grid_full = 0;       // uncapped full-occupancy grid: used whenever the launch range is restricted
+  int S = 0;               // SMs of the device (a launch over [0, S) may use the capped grid)
   double flops = 0;        // algorithmic FLOPs per launch (roofline)
   double bytes = 0;        // algorithmic HBM bytes per launch (roofline)
   LaunchFn launch = nullptr;
@@ -31,6 +34,13 @@ struct KernelDesc {
   int choice_bn = 0, choice_splits = 0;  // tcgen05 tile configuration (0 = not a tc kernel)
   alignas(128) unsigned char params[4096];  // family-specific parameter block
 };
+
+// Grid of one launch: the capped grid only for an unrestricted range -- a
+// restricted launch needs the full-occupancy grid so that lingering
+// out-of-range CTAs can never absorb it (gate_linger in executor.cuh).
+inline int launch_grid(const KernelDesc& d, const GateArgs& g) {
+  return (d.grid_full > 0 && g.hi - g.lo < d.S) ? d.grid_full : d.grid;
+}
 
 struct DeviceCaps {
   int S = 148;             // SMs
