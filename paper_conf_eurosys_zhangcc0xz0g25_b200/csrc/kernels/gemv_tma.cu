@@ -298,7 +298,14 @@ bool build_gemv_tma(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std:
   // rows per tile: 4 (measured on B200, profiles/round1/gemv_rows.txt: VGG FC1
   // 25088->4096 rows 8/4/2/1 = 52.0/40.7/46.8/53.7 us -- 8-row tiles (400 KB)
   // leave a long tail in the dynamic queue, 1-2-row tiles pay the per-tile
-  // fold too often), fewer when that leaves under one tile per SM
+  // fold too often), fewer when that leaves under one tile per SM.  Three
+  // other schedules were measured and dropped: a flat weight stream whose
+  // 16-64 KB tiles cut rows (fp32 row sums completed through a global k
+  // counter: half the bandwidth -- the gpu-scope fences also invalidate L1
+  // and the X reloads), guided tile heights 4 -> 2 -> 1 (10% slower: partial
+  // stages), and the last wave's row tiles cut into K halves joined by fp32
+  // atomics (18% slower); profiles/round1/gemv_{stream_sweep,guided_ab,
+  // split_tail_ab}.txt
   int rows = 4;
   while (rows > 1 && (long long)((p.N + rows - 1) / rows) < caps.S) rows /= 2;
   if (const char* e = std::getenv("BLESS_GEMV_ROWS")) rows = std::atoi(e);
