@@ -667,7 +667,7 @@ __global__ void __launch_bounds__(kTcThreads, 2) k_tc_gemm(const __grid_constant
 template <int BN, int BK>
 static cudaError_t launch_tc(const KernelDesc& d, const GateArgs& g, cudaStream_t st) {
   void* args[2] = {(void*)d.params, (void*)&g};
-  return launch_kernel((const void*)k_tc_gemm<BN, BK>, dim3(d.grid), dim3(d.block), (size_t)d.smem, st, args);
+  return launch_kernel((const void*)k_tc_gemm<BN, BK>, dim3(launch_grid(d, g)), dim3(d.block), (size_t)d.smem, st, args);
 }
 
 template <int BN, int BK>
@@ -875,6 +875,11 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   d.tiles = (uint32_t)(tiles_m * p.tiles_n * p.splits);
   d.block = kTcThreads;
   d.grid = caps.S;
+  // one CTA per SM on unrestricted launches (B200 kprobe: 0-4% faster than
+  // two, profiles/round1/tc_occ.txt); restricted launches keep the
+  // full-occupancy grid (launch_grid in kdesc.hpp)
+  d.max_occ = 1;
+  if (const char* e = std::getenv("BLESS_TC_MAX_OCC")) d.max_occ = std::max(1, std::atoi(e));   // sweeps
   bool ok = false;
 #define TC_CASE(bn, bk) \
   if (BN == bn && BK == bk) ok = prep<bn, bk>(d, p, err);
