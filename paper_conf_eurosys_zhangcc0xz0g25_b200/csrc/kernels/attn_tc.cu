@@ -13,9 +13,9 @@
 //   4. tcgen05.mma: O = P V into TMEM (64 columns);
 //   5. epilogue: O / rowsum -> bf16 -> out[q, h*64 : h*64 + 64].
 // Warp 0: TMA producer + MMA issuer (one thread); warps 1..8: softmax and
-// epilogue, two warps per TMEM lane quarter (quarter = warp % 4), each taking
-// one half of the keys (and of O's columns); the row max and row sum of the
-// two halves meet in shared memory.  (With one warp per quarter the softmax
+// epilogue, four warps per TMEM lane quarter (quarter = warp % 4), each taking
+// one quarter of the keys (and of O's columns); the row max and row sum of the
+// parts meet in shared memory.  (With one warp per quarter the softmax
 // was the serial part of a BERT-large tile: 16.6 us per launch.)  Under the
 // SM-gated executor.
 #include <cuda.h>
@@ -40,13 +40,14 @@ struct AttnTcParams {
 };
 
 namespace attn {
-constexpr int kSoftWarps = 8;             // two per TMEM lane quarter (key halves)
+constexpr int kParts = 4;                 // key parts per TMEM lane quarter
+constexpr int kSoftWarps = 4 * kParts;    // softmax/epilogue warps
 constexpr int kThreads = 32 + 32 * kSoftWarps;   // warp 0 producer/MMA, warps 1-8 softmax/epilogue
 constexpr int kMaxL = 384;                // S (L fp32 columns) + O (64 columns at 448) fit in 512 TMEM columns
 constexpr int kQBytes = 128 * 128;        // 128 rows x 128 B
 constexpr int kKVBytes = kMaxL * 128;     // L rows x 128 B (K, later V)
 constexpr int kPBytes = (kMaxL / 64) * 128 * 128;  // L/64 K-blocks of [128 rows x 128 B]
-constexpr int kSmem = kQBytes + kKVBytes + kPBytes + 1024 + 256 + 2 * 2 * 128 * 4;   // + row max/sum halves
+constexpr int kSmem = kQBytes + kKVBytes + kPBytes + 1024 + 256 + 2 * kParts * 128 * 4;   // + row max/sum parts
 }  // namespace attn
 
 #ifdef __CUDACC__
@@ -143,8 +144,8 @@ __device__ void attn_work(const AttnTcParams& p, const GateArgs& g) {
   uint64_t* b_o1 = bars + 7;   // P_hi MMAs done (MMA commit)
   int* tile_slot = (int*)(bars + 8);
   uint32_t* tmem_slot = (uint32_t*)(tile_slot + 1);
-  float* red_max = (float*)(bars + 32);   // [2][128] per key half
-  float* red_sum = red_max + 256;         // [2][128]
+  float* red_max = (float*)(bars + 32);   // [kParts][128] per key part
+  float* red_sum = red_max + kParts * 128;  // [kParts][128]
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     bar_init(b_qk, 1);
@@ -217,9 +218,9 @@ __device__ void attn_work(const AttnTcParams& p, const GateArgs& g) {
     } else {
       // ---- softmax: thread = query row (TMEM lane) x key half
       const int q = warp & 3;
-      const int half = (warp - 1) >> 2;
+      const int part = (warp - 1) >> 2;
       const int row = q * 32 + lane;
-      const int c0 = half * (L >> 1), c1 = c0 + (L >> 1);   // L % 128 == 0: halves are whole 64-key blocks
+      const int c0 = part * (L / kParts), c1 = c0 + L / kParts;   // L % 128 == 0: parts are whole 16-key chunks
       const uint32_t trow = tmem + ((uint32_t)(q * 32) << 16);
       bar_wait(b_s, ph);
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
@@ -230,9 +231,10 @@ __device__ void attn_work(const AttnTcParams& p, const GateArgs& g) {
 #pragma unroll
         for (int i = 0; i < 16; ++i) mx = fmaxf(mx, __uint_as_float(v[i]));
       }
-      red_max[half * 128 + row] = mx;
-      asm volatile("bar.sync 1, %0;" ::"n"(32 * kSoftWarps) : "memory");   // both halves' maxima
-      mx = fmaxf(red_max[row], red_max[128 + row]);
+      red_max[part * 128 + row] = mx;
+      asm volatile("bar.sync 1, %0;" ::"n"(32 * kSoftWarps) : "memory");   // every part's maximum
+#pragma unroll
+      for (int i = 0; i < kParts; ++i) mx = fmaxf(mx, red_max[i * 128 + row]);
       const float moff = mx * p.scale_log2e;
       float sum = 0.f;
       const int rr = row & 7;
@@ -269,16 +271,19 @@ __device__ void attn_work(const AttnTcParams& p, const GateArgs& g) {
         __syncwarp();
         if (lane == 0) bar_arrive(pass == 0 ? b_p : b_p2);
       }
-      red_sum[half * 128 + row] = sum;
-      // ---- epilogue (this warp: O columns [32 * half, 32 * half + 32))
+      red_sum[part * 128 + row] = sum;
+      // ---- epilogue (this warp: O columns [16 * part, 16 * part + 16))
       bar_wait(b_o, ph);
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-      asm volatile("bar.sync 1, %0;" ::"n"(32 * kSoftWarps) : "memory");   // both halves' sums
-      const float inv = 1.f / (red_sum[row] + red_sum[128 + row]);
+      asm volatile("bar.sync 1, %0;" ::"n"(32 * kSoftWarps) : "memory");   // every part's sum
+      float tot = 0.f;
+#pragma unroll
+      for (int i = 0; i < kParts; ++i) tot += red_sum[i * 128 + row];
+      const float inv = 1.f / tot;
       const int qrow = qb * 128 + row;
       __nv_bfloat16* out = p.O + (size_t)qrow * p.ldo + h * 64;
 #pragma unroll 1
-      for (int c = 32 * half; c < 32 * half + 32; c += 16) {
+      for (int c = 16 * part; c < 16 * part + 16; c += 16) {
         uint32_t v[16];
         ld16(trow + 448 + c, v);
         uint32_t pk[8];
