@@ -95,6 +95,13 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, u
       "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
       : "memory");
 }
+__device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1, int c2) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(
+          smem_u32(dst)),
+      "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2)
+      : "memory");
+}
 __device__ __forceinline__ void tma_load_4d(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1, int c2,
                                             int c3) {
   asm volatile(
@@ -138,11 +145,13 @@ __device__ __forceinline__ void tmem_ld_wait() { asm volatile("tcgen05.wait::ld.
 // UMMA shared-memory descriptor, K-major, swizzled (SW128/64/32: rows of
 // BK*2 bytes, 8-row atoms; LBO = 16 B (unused for swizzled K-major), SBO =
 // 8 rows * row bytes; version 1 = tcgen05; layout type 2/4/6).
+// BK = 128 stages hold two 64-deep SW128 slabs (one TMA box each operand), so
+// their descriptors are those of BK = 64.
 template <int BK>
 __device__ __forceinline__ uint64_t smem_desc(uint32_t saddr) {
-  constexpr uint64_t row_bytes = BK * 2;
+  constexpr uint64_t row_bytes = (BK > 64 ? 64 : BK) * 2;
   constexpr uint64_t sbo = 8 * row_bytes;
-  constexpr uint64_t layout = (BK == 64) ? 2 : (BK == 32 ? 4 : 6);
+  constexpr uint64_t layout = (BK >= 64) ? 2 : (BK == 32 ? 4 : 6);
   uint64_t d = 0;
   d |= (uint64_t)((saddr >> 4) & 0x3FFF);
   d |= (uint64_t)1 << 16;                    // LBO (16 B)
@@ -308,7 +317,7 @@ struct TcCfg {
   static constexpr int kStageBytes = kStageA + kStageB;
   // default pipeline: ~96 KB of stages, so two CTAs (the next kernel's, under
   // programmatic dependent launch, or another tenant's) fit on one SM
-  static constexpr int kStages = std::min(6, (96 * 1024) / kStageBytes);
+  static constexpr int kStages = std::max(2, std::min(6, (96 * 1024) / kStageBytes));
   // TMEM accumulators: double buffered (epilogue of tile i overlaps the MMAs of
   // tile i+1) up to BN = 128; BN = 256 keeps one so a second co-resident CTA
   // (another tenant's kernel on the same SM) can still allocate.
@@ -425,7 +434,10 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         }
         auto load_B = [&](int kb, int st) {
           unsigned char* b = sB + st * Cfg::kStageB;
-          if (p.mode == 0) {
+          if (BK > 64) {   // 3-D view (64, N, K/64): one box = two 64-deep slabs
+            const int kc = p.mode == 0 ? kb * 2 : (kb / p.kc_per_tap) * (p.C / 64) + (kb % p.kc_per_tap) * 2;
+            tma_load_3d(b, &p.tmB, &full[st], 0, tn * BN, kc);
+          } else if (p.mode == 0) {
             tma_load_2d(b, &p.tmB, &full[st], kb * BK, tn * BN);
           } else {
             const int tap = kb / p.kc_per_tap, c0 = (kb - tap * p.kc_per_tap) * BK;
@@ -434,7 +446,13 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         };
         auto load_A = [&](int kb, int st) {
           unsigned char* a = sA + st * Cfg::kStageA;
-          if (p.mode == 0) {
+          if (BK > 64 && p.mode == 0) {   // 3-D view (64, M, K/64)
+            tma_load_3d(a, &p.tmA, &full[st], 0, tm * 128, kb * 2);
+          } else if (BK > 64) {            // 4-D view (64, W, H, C/64), stride 1 only
+            const int tap = kb / p.kc_per_tap, ch = (kb - tap * p.kc_per_tap) * 2;
+            const int r = tap / p.S_, s = tap - r * p.S_;
+            tma_load_4d(a, &p.tmA, &full[st], 0, ow0 - p.pad + s, oh0 - p.pad + r, ch);
+          } else if (p.mode == 0) {
             tma_load_2d(a, &p.tmA, &full[st], kb * BK, tm * 128);
           } else {
             const int tap = kb / p.kc_per_tap, c0 = (kb - tap * p.kc_per_tap) * BK;
@@ -512,7 +530,10 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           } else {
 #pragma unroll
             for (int k = 0; k < BK / 16; ++k) {
-              tc_mma(d_tmem, smem_desc<BK>(a0 + k * 32), smem_desc<BK>(b0 + k * 32), idesc,
+              // BK = 128: slab k / 4 (128 x 64 of A, BN x 64 of B), K step k % 4
+              const uint32_t ao = BK > 64 ? (k >> 2) * (128 * 128) + (k & 3) * 32 : k * 32;
+              const uint32_t bo = BK > 64 ? (k >> 2) * (BN * 128) + (k & 3) * 32 : k * 32;
+              tc_mma(d_tmem, smem_desc<BK>(a0 + ao), smem_desc<BK>(b0 + bo), idesc,
                      (kb != kb0 || k) ? 1u : 0u);
             }
             tc_commit(&empty[stage]);
@@ -721,7 +742,7 @@ static bool encode(CUtensorMap* map, int rank, const void* base, const cuuint64_
   if (!fn) return false;
   cuuint32_t es[5] = {1, 1, 1, 1, 1};
   const CUtensorMapSwizzle sw =
-      BK == 64 ? CU_TENSOR_MAP_SWIZZLE_128B : (BK == 32 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B);
+      BK >= 64 ? CU_TENSOR_MAP_SWIZZLE_128B : (BK == 32 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B);
   const CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, (cuuint32_t)rank, const_cast<void*>(base), dims,
                         strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
@@ -748,7 +769,15 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   // BLESS_TC_CFG="BN,BK,splits" forces a tile configuration (sweeps only, tools/tcsweep.py)
   int fbn = 0, fbk = 0, fs = 0;
   if (const char* f = std::getenv("BLESS_TC_CFG")) std::sscanf(f, "%d,%d,%d", &fbn, &fbk, &fs);
-  const bool fbk_ok = fbk == 16 || fbk == 32 || fbk == 64;
+  const bool fbk_ok = fbk == 16 || fbk == 32 || fbk == 64 || fbk == 128;
+  // BK = 128 stages (two 64-deep slabs per one 3-D/4-D TMA box): the K loop
+  // pays a fixed cost per box, not per byte (profiles/round1/s4/tc_bk_sweep.txt),
+  // so halving the boxes per K cuts 3x3 conv time 38-42% on B200
+  // (s4/tc_bk128_ab.txt).  BLESS_TC_BK128=0 restores BK = 64 (A/B sweeps).
+  static const bool bk128 = [] {
+    const char* e = std::getenv("BLESS_TC_BK128");
+    return !e || std::atoi(e) != 0;
+  }();
   if (op.kind == BL_OP_GEMM) {
     p.M = (int)op.dims[0];
     p.N = (int)op.dims[1];
@@ -759,11 +788,18 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     if (p.M <= 8 || p.N % 16 || p.K % 8 || ldx % 8 || p.ldy % 8 || p.ldr % 8) return false;  // GEMV / SIMT
     if (((uintptr_t)X | (uintptr_t)W) & 15) return false;
     p.mode = 0;
-    BK = fbk_ok ? fbk : 64;
+    BK = fbk_ok ? fbk : ((bk128 && p.K % 64 == 0) ? 128 : 64);
+    if (BK == 128 && p.K % 64) BK = 64;
     p.num_kb = (p.K + BK - 1) / BK;
-    cuuint64_t da[2] = {(cuuint64_t)p.K, (cuuint64_t)p.M}, sa[1] = {(cuuint64_t)ldx * 2};
-    cuuint32_t ba[2] = {(cuuint32_t)BK, 128};
-    if (!encode(&p.tmA, 2, X, da, sa, ba, BK, err)) return false;
+    if (BK == 128) {   // (64, M, K/64): a box of two 64-deep slabs
+      cuuint64_t da[3] = {64, (cuuint64_t)p.M, (cuuint64_t)(p.K / 64)}, sa[2] = {(cuuint64_t)ldx * 2, 128};
+      cuuint32_t ba[3] = {64, 128, 2};
+      if (!encode(&p.tmA, 3, X, da, sa, ba, BK, err)) return false;
+    } else {
+      cuuint64_t da[2] = {(cuuint64_t)p.K, (cuuint64_t)p.M}, sa[1] = {(cuuint64_t)ldx * 2};
+      cuuint32_t ba[2] = {(cuuint32_t)BK, 128};
+      if (!encode(&p.tmA, 2, X, da, sa, ba, BK, err)) return false;
+    }
   } else if (op.kind == BL_OP_CONV) {
     const int Nb = (int)op.dims[0], H = (int)op.dims[1], Wd = (int)op.dims[2], C = (int)op.dims[3];
     const int K = (int)op.dims[4], R = (int)op.dims[5], S = (int)op.dims[6];
@@ -779,7 +815,9 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     if (((uintptr_t)X | (uintptr_t)W) & 15) return false;
     // 1x1 stride-1 convs are plain GEMMs over pixels: any C % 8, K tail zero-filled by TMA
     BK = one_by_one ? 64 : ((C % 64 == 0) ? 64 : (C % 32 == 0 ? 32 : 16));
+    if (bk128 && stride == 1 && (one_by_one ? C % 64 == 0 : C % 128 == 0)) BK = 128;
     if (fbk_ok && fbk < BK) BK = fbk;
+    if (fbk == 128 && stride == 1 && (one_by_one ? C % 64 == 0 : C % 128 == 0)) BK = 128;
     p.OH = (H + 2 * pad - R) / stride + 1;
     p.OW = (Wd + 2 * pad - S) / stride + 1;
     p.M = p.OH * p.OW;
@@ -799,7 +837,18 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     p.BH = 128 / BW;
     p.tiles_w = (p.OW + BW - 1) / BW;
     const int tiles_h = (p.OH + p.BH - 1) / p.BH;
-    if (one_by_one) {
+    if (one_by_one && BK == 128) {
+      p.mode = 0;
+      cuuint64_t da[3] = {64, (cuuint64_t)(H * Wd), (cuuint64_t)(C / 64)}, sa[2] = {(cuuint64_t)ldx * 2, 128};
+      cuuint32_t ba[3] = {64, 128, 2};
+      if (!encode(&p.tmA, 3, X, da, sa, ba, BK, err)) return false;
+    } else if (stride == 1 && BK == 128) {
+      p.mode = 1;
+      cuuint64_t da[4] = {64, (cuuint64_t)Wd, (cuuint64_t)H, (cuuint64_t)(C / 64)};
+      cuuint64_t sa[3] = {(cuuint64_t)ldx * 2, (cuuint64_t)Wd * ldx * 2, 128};
+      cuuint32_t ba[4] = {64, (cuuint32_t)BW, (cuuint32_t)p.BH, 2};
+      if (!encode(&p.tmA, 4, X, da, sa, ba, BK, err)) return false;
+    } else if (one_by_one) {
       // 1x1 stride-1: plain GEMM over pixels
       p.mode = 0;
       cuuint64_t da[2] = {(cuuint64_t)C, (cuuint64_t)(H * Wd)}, sa[1] = {(cuuint64_t)ldx * 2};
@@ -847,6 +896,14 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     BN = fbn;
     p.tiles_n = (p.N + BN - 1) / BN;
   }
+  if (BK == 128 && BN > 64) {
+    // two BK = 128 stages must fit the ~96 KB budget that lets a second CTA
+    // (another tenant's kernel under NSP) share the SM: BN <= 64.  BN = 128
+    // stages of 64 KB cost co-residency and wrecked the C3/C4 squads on B200
+    // (profiles/round1/s4/bench_bk128_bn128_*.json).
+    BN = 64;
+    p.tiles_n = (p.N + BN - 1) / BN;
+  }
   if (fs >= 1) splits = std::min(fs, p.num_kb);
   p.kbs = (p.num_kb + splits - 1) / splits;
   p.splits = (p.num_kb + p.kbs - 1) / p.kbs;
@@ -866,7 +923,12 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     p.sem = (unsigned*)((char*)buf + wsb);
     d.owned = buf;
   }
-  {
+  if (BK == 128) {
+    if (p.K % 64) { err = "BK 128 needs K % 64 == 0"; return false; }
+    cuuint64_t db[3] = {64, (cuuint64_t)p.N, (cuuint64_t)(p.K / 64)}, sb[2] = {(cuuint64_t)p.K * 2, 128};
+    cuuint32_t bb[3] = {64, (cuuint32_t)BN, 2};
+    if (!encode(&p.tmB, 3, W, db, sb, bb, BK, err)) return false;
+  } else {
     cuuint64_t db[2] = {(cuuint64_t)p.K, (cuuint64_t)p.N}, sb[1] = {(cuuint64_t)p.K * 2};
     cuuint32_t bb[2] = {(cuuint32_t)BK, (cuuint32_t)BN};
     if (!encode(&p.tmB, 2, W, db, sb, bb, BK, err)) return false;
@@ -888,6 +950,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   TC_CASE(64, 16) TC_CASE(64, 32) TC_CASE(64, 64)
   TC_CASE(128, 16) TC_CASE(128, 32) TC_CASE(128, 64)
   TC_CASE(256, 16) TC_CASE(256, 32) TC_CASE(256, 64)
+  TC_CASE(16, 128) TC_CASE(32, 128) TC_CASE(64, 128) TC_CASE(128, 128)
 #undef TC_CASE
   if (!ok) {
     if (err.empty()) err = "no tc instantiation";

@@ -111,13 +111,16 @@ def test_conv_bf16(ctx, H, W, C, K, k, s, p, act, res):
     run_and_check(ctx, m, "bf16")
 
 
-@pytest.mark.parametrize("cfg", ["256,64,1", "256,32,3", "128,64,5", "64,32,2", "32,64,1"])
+@pytest.mark.parametrize("cfg", ["256,64,1", "256,32,3", "128,64,5", "64,32,2", "32,64,1", "128,128,1", "64,128,3"])
 @pytest.mark.parametrize("shape", [("conv", (56, 56, 64, 256, 3, 1, 1)), ("conv", (28, 28, 128, 256, 3, 2, 1)),
+                                   ("conv", (20, 27, 256, 96, 3, 1, 1)), ("conv", (9, 9, 192, 64, 1, 1, 0)),
                                    ("conv", (14, 14, 256, 512, 1, 1, 0)), ("gemm", (384, 1024, 320)),
                                    ("gemm", (200, 272, 136))])
 def test_tc_forced_configs(ctx, cfg, shape, monkeypatch):
     """Every tile configuration the selector may pick (BN 32..256, BK 32/64,
-    split-K) is exact on convs (stride 1/2, 1x1) and ragged GEMMs."""
+    BK 128 = two 64-deep slabs per TMA box where C % 128 == 0 (3x3) or
+    K % 64 == 0 (GEMM, 1x1; the K tail zero-filled), split-K) is exact on convs
+    (stride 1/2, 1x1) and ragged GEMMs."""
     monkeypatch.setenv("BLESS_TC_CFG", cfg)
     kind, dims = shape
 
