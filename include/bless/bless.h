@@ -201,13 +201,33 @@ typedef struct {
   int32_t tenant;
   int32_t kernel;
   int16_t lo, hi;     /* logical SM range */
-  int32_t nsm;        /* distinct SMs that processed >= 1 tile */
+  int32_t nsm;        /* distinct SMs that processed >= 1 tile; -1 = unknown (a light-exit
+                         launch older than the last 2^18 of the run: its stats record was
+                         reused, so no times or mask are reported) */
   int32_t fallback;   /* 1 if no in-range CTA ran and the last CTA did the work */
   int64_t start_ns;   /* first tile claimed */
   int64_t end_ns;     /* last CTA exit */
   uint64_t req;
   uint32_t sm_mask[8]; /* logical SMs that processed >= 1 tile (bit i = SM i) */
 } bl_launch_rec;
+
+/* One TEMPORAL-policy launch decision (reading R22), for
+ * replay by the oracle's slice rule.  Times are ns relative to the loop's
+ * start (host clock).  A record is written for every kernel the loop launches. */
+typedef struct {
+  int64_t t;           /* host time of the decision */
+  int64_t gpu_free;    /* predicted time the GPU becomes free before this launch */
+  int64_t slice_end;   /* end of the slice the launch is charged to */
+  int64_t dur;         /* predicted kernel duration t[j][k][S] */
+  int64_t sid;         /* slice id (T-cap: cycle * n_tenants + j; T-wc: turn counter) */
+  int64_t last_sid;    /* slice id of the previous launch (-1 before the first) */
+  int64_t turn_end;    /* T-wc: end of the running turn before this decision (0 if none) */
+  int32_t turn;        /* T-wc: tenant of the running turn before this decision (-1 if none) */
+  int32_t work_mask;   /* bit j: tenant j had an active or arrived request at t */
+  int32_t tenant, kernel;
+  int32_t work_conserving;
+  int32_t reserved;
+} bl_temporal_rec;
 
 /* Launch descriptor summary of one appended kernel (roofline accounting). */
 typedef struct {
@@ -236,7 +256,8 @@ typedef struct {
  * bl_create: device >= 0 selects a CUDA device and runs the SM probe (A1);
  * BL_DEVICE_NONE makes a CUDA-free ctx (S, g come from bl_load_profile).
  * workspace/ws_bytes: optional caller-owned device buffer for the launch-slot
- * ring (>= 4 MiB); NULL lets the library cudaMalloc it.  Errors: BL_E_INVALID,
+ * ring (>= 8 MiB: 2^19 slots x 16 B; more with BLESS_STATS_RING_LOG2); NULL
+ * lets the library cudaMalloc it.  Errors: BL_E_INVALID,
  * BL_E_CUDA, BL_E_OOM. */
 bl_status bl_create(int device, const bl_params* params, void* workspace, size_t ws_bytes, bl_ctx** out);
 bl_status bl_destroy(bl_ctx* ctx);               /* stops threads, frees library memory */
@@ -307,6 +328,8 @@ bl_status bl_stop(bl_ctx* ctx);
 /* Copy out decision records / launch records (from index 'first'). */
 bl_status bl_decisions(bl_ctx* ctx, size_t first, bl_decision* buf, size_t cap, size_t* n_out);
 bl_status bl_launches(bl_ctx* ctx, size_t first, bl_launch_rec* buf, size_t cap, size_t* n_out);
+/* TEMPORAL launch decisions of the last run (policy BL_POLICY_TEMPORAL). */
+bl_status bl_temporal_log(bl_ctx* ctx, size_t first, bl_temporal_rec* buf, size_t cap, size_t* n_out);
 /* Reset request table, logs and queues (between runs with the same tenants). */
 bl_status bl_reset(bl_ctx* ctx, const bl_params* params);
 
@@ -315,6 +338,32 @@ bl_status bl_reset(bl_ctx* ctx, const bl_params* params);
  * n_active (tenant ids, arrivals, next kernel indices). */
 bl_status bl_decide(bl_ctx* ctx, int64_t now, int n_active, const int32_t* tenants,
                     const int64_t* arrivals, const int32_t* next_kernel, bl_decision* out);
+
+/* Host cost of the C++ scheduler (3.7 + 2 + 1 us per kernel on
+ * the paper's host): re-runs decide() 'reps' times on the inputs (now, active
+ * set) of each of the n logged records on the calling thread and returns the
+ * total wall time and the total number of kernels those decisions picked
+ * (so ns/decision = total_ns / (n * reps), ns/kernel = total_ns / total_picks).
+ * BL_E_INVALID on a record whose active set does not fit the ctx. */
+bl_status bl_time_decide(bl_ctx* ctx, const bl_decision* recs, size_t n, int reps, int64_t* total_ns,
+                         int64_t* total_picks);
+
+/* ---- box-wide trace dispatcher ("replicating
+ * its runtime components for each active GPU") -----------------------------------
+ * One host thread routes a merged trace of several GPUs' tenants: entry i goes
+ * to ctxs[entries[i].ctx] as a request of entries[i].tenant.  Entries must be
+ * sorted by arrival_ns (trace time).  WALL-clock ctxs: the call busy-waits on
+ * the host clock until base_ns + arrival_ns, then submits with that arrival
+ * (the ctxs must be started); VIRTUAL ctxs: submits at once with arrival_ns
+ * (before bl_start).  req_out[i] receives the request id (may be NULL).
+ * Returns when every entry is submitted; errors stop at the failing entry. */
+typedef struct {
+  int32_t ctx;
+  int32_t tenant;
+  int64_t arrival_ns;
+} bl_dispatch_entry;
+bl_status bl_dispatch(bl_ctx* const* ctxs, int n_ctx, const bl_dispatch_entry* entries, size_t n, int64_t base_ns,
+                      uint64_t* req_out);
 
 /* Diagnostics: mean per-launch device time of 'reps' back-to-back S-CTA
  * launches of an executor skeleton (variant 0: empty kernel, 1: SM gate + tile

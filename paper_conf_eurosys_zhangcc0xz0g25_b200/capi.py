@@ -71,6 +71,17 @@ class bl_launch_rec(C.Structure):
                 ("sm_mask", C.c_uint32 * 8)]
 
 
+class bl_temporal_rec(C.Structure):
+    _fields_ = [("t", C.c_int64), ("gpu_free", C.c_int64), ("slice_end", C.c_int64), ("dur", C.c_int64),
+                ("sid", C.c_int64), ("last_sid", C.c_int64), ("turn_end", C.c_int64), ("turn", C.c_int32),
+                ("work_mask", C.c_int32), ("tenant", C.c_int32), ("kernel", C.c_int32),
+                ("work_conserving", C.c_int32), ("reserved", C.c_int32)]
+
+
+class bl_dispatch_entry(C.Structure):
+    _fields_ = [("ctx", C.c_int32), ("tenant", C.c_int32), ("arrival_ns", C.c_int64)]
+
+
 class bl_kernel_info(C.Structure):
     _fields_ = [("family", C.c_char * 32), ("tiles", C.c_int32), ("grid", C.c_int32), ("block", C.c_int32),
                 ("smem", C.c_int32), ("flops", C.c_double), ("bytes", C.c_double)]
@@ -121,6 +132,10 @@ _SIGS = {
     "bl_reset": (C.c_int, [C.c_void_p, _P(bl_params)]),
     "bl_decide": (C.c_int, [C.c_void_p, C.c_int64, C.c_int, _P(C.c_int32), _P(C.c_int64), _P(C.c_int32),
                             _P(bl_decision)]),
+    "bl_temporal_log": (C.c_int, [C.c_void_p, C.c_size_t, _P(bl_temporal_rec), C.c_size_t, _P(C.c_size_t)]),
+    "bl_time_decide": (C.c_int, [C.c_void_p, _P(bl_decision), C.c_size_t, C.c_int, _P(C.c_int64), _P(C.c_int64)]),
+    "bl_dispatch": (C.c_int, [_P(C.c_void_p), C.c_int, _P(bl_dispatch_entry), C.c_size_t, C.c_int64,
+                              _P(C.c_uint64)]),
     "bl_debug_overhead": (C.c_int, [C.c_void_p, C.c_int, C.c_int, _P(C.c_int64)]),
     "bl_now_ns": (C.c_int64, []),
     "bl_last_error": (C.c_char_p, []),
@@ -298,6 +313,21 @@ class Ctx:
         lib().bl_launches(self.h, 0, buf, n.value, C.byref(got))
         return [buf[i] for i in range(got.value)]
 
+    def temporal_log(self):
+        n = C.c_size_t()
+        lib().bl_temporal_log(self.h, 0, None, 0, C.byref(n))
+        buf = (bl_temporal_rec * max(1, n.value))()
+        got = C.c_size_t()
+        lib().bl_temporal_log(self.h, 0, buf, n.value, C.byref(got))
+        return [buf[i] for i in range(got.value)]
+
+    def time_decide(self, recs, reps: int = 1):
+        """Native timing of decide() on logged records: (total_ns, total_picks)."""
+        arr = (bl_decision * max(1, len(recs)))(*recs)
+        ns, picks = C.c_int64(), C.c_int64()
+        check("bl_time_decide", lib().bl_time_decide(self.h, arr, len(recs), int(reps), C.byref(ns), C.byref(picks)))
+        return ns.value, picks.value
+
     def decide(self, now: int, active):
         """active: list of (tenant, arrival, next_kernel)."""
         n = len(active)
@@ -311,6 +341,18 @@ class Ctx:
 
 def now_ns() -> int:
     return lib().bl_now_ns()
+
+
+def dispatch(ctxs, entries, base_ns: int = 0):
+    """Box-wide trace dispatcher (bl_dispatch): entries = [(ctx_index, tenant,
+    arrival_ns)] sorted by arrival; returns the request ids.  Blocks (busy-waits
+    in native code, GIL released) until every entry is submitted."""
+    hs = (C.c_void_p * len(ctxs))(*[c.h.value for c in ctxs])
+    ent = (bl_dispatch_entry * max(1, len(entries)))(*[bl_dispatch_entry(int(c), int(t), int(a))
+                                                        for c, t, a in entries])
+    out = (C.c_uint64 * max(1, len(entries)))()
+    check("bl_dispatch", lib().bl_dispatch(hs, len(ctxs), ent, len(entries), int(base_ns), out))
+    return [out[i] for i in range(len(entries))]
 
 
 def decision_to_tuple(d: bl_decision):

@@ -169,6 +169,48 @@ bl_status bl_launches(bl_ctx* ctx, size_t first, bl_launch_rec* buf, size_t cap,
   GUARD(ctx);
   return ctx->eng->launches(first, buf, cap, n);
 }
+bl_status bl_temporal_log(bl_ctx* ctx, size_t first, bl_temporal_rec* buf, size_t cap, size_t* n) {
+  GUARD(ctx);
+  return ctx->eng->temporal_log(first, buf, cap, n);
+}
+bl_status bl_time_decide(bl_ctx* ctx, const bl_decision* recs, size_t n, int reps, int64_t* total_ns,
+                         int64_t* total_picks) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->time_decide(recs, n, reps, total_ns, total_picks, e); });
+}
+bl_status bl_dispatch(bl_ctx* const* ctxs, int n_ctx, const bl_dispatch_entry* ent, size_t n, int64_t base_ns,
+                      uint64_t* req_out) {
+  if (!ctxs || n_ctx < 1 || (n && !ent)) {
+    g_err = "bad dispatcher args";
+    return BL_E_INVALID;
+  }
+  for (int i = 0; i < n_ctx; ++i) GUARD(ctxs[i]);
+  return wrap([&](std::string& e) {
+    int64_t prev = INT64_MIN;
+    for (size_t i = 0; i < n; ++i) {
+      const bl_dispatch_entry& x = ent[i];
+      if (x.ctx < 0 || x.ctx >= n_ctx) { e = "entry " + std::to_string(i) + ": bad ctx index"; return BL_E_INVALID; }
+      if (x.arrival_ns < prev) { e = "entries not sorted by arrival"; return BL_E_INVALID; }
+      prev = x.arrival_ns;
+      bless::Engine* eng = ctxs[x.ctx]->eng;
+      int64_t arr = x.arrival_ns;
+      if (!eng->virtual_clock()) {
+        // a steady-clock busy-wait: the request is handed over at its arrival
+        arr = base_ns + x.arrival_ns;
+        while (bl_now_ns() < arr) {
+#if defined(__x86_64__)
+          __builtin_ia32_pause();
+#endif
+        }
+      }
+      uint64_t id = 0;
+      const bl_status st = eng->submit(x.tenant, arr, &id, e);
+      if (st != BL_OK) return st;
+      if (req_out) req_out[i] = id;
+    }
+    return BL_OK;
+  });
+}
 bl_status bl_reset(bl_ctx* ctx, const bl_params* p) {
   GUARD(ctx);
   return wrap([&](std::string& e) { return ctx->eng->reset(p, e); });

@@ -20,7 +20,7 @@
 //   stats.mask   logical SMs that processed >= 1 tile (atomicOr per CTA; R19)
 //   stats.end / flags / seq   written by the last CTA (seq last, after a fence)
 // The last CTA also zeroes the mask of the stats record it will reuse
-// kMaskAhead launches later and resets its slot word.
+// DeviceRT::ahead() launches later and resets its slot word.
 // Safety net: if the last CTA finds unclaimed tiles, no in-range CTA ran (the
 // hardware placed every CTA elsewhere); it then processes the tiles itself and
 // flags the launch ("fallback"), so correctness never depends on placement.
@@ -62,13 +62,12 @@ struct __align__(16) DevSlot {  // device memory, zero between launches
   unsigned long long pad;
 };
 
-constexpr uint64_t kMaskAhead = 32768;  // stats record zeroed this many launches ahead
 
 struct GateArgs {
   DevSlot* slot;
   SlotStats* stats;        // this launch's record
-  SlotStats* stats_ahead;  // record of launch seq + kMaskAhead (flags/mask zeroed here)
-  DevSlot* slot_ahead;     // slot of launch seq + kMaskAhead (zeroed here)
+  SlotStats* stats_ahead;  // record of launch seq + ahead (flags/mask zeroed here; ahead = ring / 2)
+  DevSlot* slot_ahead;     // slot of launch seq + ahead (zeroed here)
   SlotStats* prev_stats;   // light predecessor on the stream (its end stamp is written here) or null
   const uint8_t* lid_map;  // logical SM index per %smid (255 = unusable); null = identity
   uint64_t seq;
@@ -103,7 +102,7 @@ __device__ __forceinline__ bool gate_in_range(const GateArgs& g) {
 // Claim the next tile (call from ONE thread).  Returns -1 when exhausted.
 // 'marked' tracks whether this CTA already set its SM bit in the mask.
 // The claimer of tile 0 stamps the start, zeroes the slot and the stats
-// flags/mask of the launch kMaskAhead later (no CTA of that ring position's
+// flags/mask of the launch `ahead` seqs later (no CTA of that ring position's
 // previous launch can still run), and -- if it claims after
 // griddepcontrol.wait (after_wait) -- writes the end stamp of a light
 // predecessor on the stream, which completed exactly when that wait returned.

@@ -769,6 +769,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   // BLESS_TC_CFG="BN,BK,splits" forces a tile configuration (sweeps only, tools/tcsweep.py)
   int fbn = 0, fbk = 0, fs = 0;
   if (const char* f = std::getenv("BLESS_TC_CFG")) std::sscanf(f, "%d,%d,%d", &fbn, &fbk, &fs);
+  if (force && force->bk) fbk = force->bk;   // autotuner candidate (tc_candidates)
   const bool fbk_ok = fbk == 16 || fbk == 32 || fbk == 64 || fbk == 128;
   // BK = 128 stages (two 64-deep slabs per one 3-D/4-D TMA box): the K loop
   // pays a fixed cost per box, not per byte (profiles/round1/s4/tc_bk_sweep.txt),
@@ -950,7 +951,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   TC_CASE(64, 16) TC_CASE(64, 32) TC_CASE(64, 64)
   TC_CASE(128, 16) TC_CASE(128, 32) TC_CASE(128, 64)
   TC_CASE(256, 16) TC_CASE(256, 32) TC_CASE(256, 64)
-  TC_CASE(16, 128) TC_CASE(32, 128) TC_CASE(64, 128) TC_CASE(128, 128)
+  TC_CASE(16, 128) TC_CASE(32, 128) TC_CASE(64, 128)
 #undef TC_CASE
   if (!ok) {
     if (err.empty()) err = "no tc instantiation";
@@ -960,6 +961,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   std::memcpy(d.params, &p, sizeof(p));
   d.choice_bn = BN;
   d.choice_splits = p.splits;
+  d.choice_bk = BK;
   d.family = op.kind == BL_OP_GEMM ? "tc_gemm_bf16" : (p.mode == 0 ? "tc_conv1x1_bf16" : "tc_conv_bf16");
   d.flops = 2.0 * p.M * p.N * p.K;
   double a_bytes = (op.kind == BL_OP_CONV) ? 2.0 * op.dims[1] * op.dims[2] * op.dims[3] : 2.0 * p.M * p.K;
@@ -968,38 +970,50 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
 }
 
 // Candidate tile configurations for the registration-time autotuner
-// (DeviceRT::add_kernel): BN in {32, 64, 128} (narrower when N is small), each
-// unsplit and split-K to about S work units.  Measured on B200 (tools/tcsweep.py,
-// profiles/round1/tcsweep.txt) no single rule picks the fastest: unsplit tiles
-// below S often win (split-K's fp32 reduction costs several us), wide tiles win
-// on large convs; BN = 256 never won with 96 KB of pipeline stages.
+// (DeviceRT::add_kernel): BN in {32, 64, 128} (narrower when N is small) x BK
+// in {64, 128} (128 only where build_tc_gemm takes it -- K % 64 == 0 for GEMMs
+// and 1x1 convs, C % 128 == 0 for stride-1 3x3 convs -- and only with
+// BN <= 64, which keeps two stages in the ~96 KB co-residency budget), each
+// unsplit and split-K to about S work units.  Measured on B200
+// (tools/tcsweep.py, profiles/round1/tcsweep.txt, s4/tc_bk128_ab.txt) no single
+// rule picks the fastest: unsplit tiles below S often win (split-K's fp32
+// reduction costs several us), BK = 128 wins the 3x3 convs, BN = 128 with
+// BK = 64 wins large GEMMs; BN = 256 never won with 96 KB of stages.
 int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int max) {
   long long M, N, num_kb, tiles_m;
+  bool bk128_ok = false;
   if (op.kind == BL_OP_GEMM) {
     M = op.dims[0], N = op.dims[1];
     num_kb = (op.dims[2] + 63) / 64;
     tiles_m = (M + 127) / 128;
+    bk128_ok = op.dims[2] % 64 == 0;
   } else if (op.kind == BL_OP_CONV) {
     const long long H = op.dims[1], W = op.dims[2], C = op.dims[3], R = op.dims[5], S = op.dims[6];
     const long long st = op.dims[7] ? op.dims[7] : 1, pad = op.dims[8];
     const long long OH = (H + 2 * pad - R) / st + 1, OW = (W + 2 * pad - S) / st + 1;
+    const bool one = R == 1 && S == 1 && st == 1 && pad == 0;
     N = op.dims[4];
     num_kb = R * S * std::max(1LL, C / 64);
     long long BW = 8;
     while (BW < OW && BW < 128) BW <<= 1;
     tiles_m = ((OW + BW - 1) / BW) * ((OH + (128 / BW) - 1) / (128 / BW));
+    bk128_ok = st == 1 && (one ? C % 64 == 0 : C % 128 == 0);
   } else {
     return 0;
   }
   int n = 0;
   const int nmax = N <= 16 ? 16 : (N <= 32 ? 32 : (N <= 64 ? 64 : 128));
-  for (int bn = std::min(32, nmax); bn <= nmax && n < max; bn <<= 1) {
-    const long long tiles = tiles_m * ((N + bn - 1) / bn);
-    out[n++] = TcChoice{bn, 1};
-    if (tiles < caps.S && num_kb >= 6 && n < max) {
-      const long long want = std::min<long long>((caps.S + tiles - 1) / tiles, num_kb / 3);
-      if (want >= 2) out[n++] = TcChoice{bn, (int)want};
-      if (want >= 6 && n < max) out[n++] = TcChoice{bn, (int)(want / 2)};
+  for (int bn = std::min(32, nmax); bn <= nmax; bn <<= 1) {
+    for (int bk = 64; bk <= 128; bk += 64) {
+      if (bk == 128 && (!bk128_ok || bn > 64)) continue;
+      const long long kbs = bk == 128 ? (num_kb + 1) / 2 : num_kb;   // K blocks at this depth
+      const long long tiles = tiles_m * ((N + bn - 1) / bn);
+      if (n < max) out[n++] = TcChoice{bn, 1, bk};
+      if (tiles < caps.S && kbs >= 6) {
+        const long long want = std::min<long long>((caps.S + tiles - 1) / tiles, kbs / 3);
+        if (want >= 2 && n < max) out[n++] = TcChoice{bn, (int)want, bk};
+        if (want >= 6 && n < max) out[n++] = TcChoice{bn, (int)(want / 2), bk};
+      }
     }
   }
   return n;

@@ -110,6 +110,12 @@ std::unique_ptr<DeviceRT> DeviceRT::create(int device, void* ws, size_t ws_bytes
   rt->caps_.cc_major = prop.major;
   rt->caps_.cc_minor = prop.minor;
   rt->caps_.smem_optin = (int)prop.sharedMemPerBlockOptin;
+  if (const char* e = std::getenv("BLESS_STATS_RING_LOG2")) {
+    const int l2 = std::atoi(e);
+    if (l2 >= 10 && l2 <= 22) rt->ring_ = 1ull << l2;
+  }
+  rt->ahead_ = rt->ring_ / 2;
+  const uint64_t kSlotRing = rt->ring_;
   const size_t slot_bytes = kSlotRing * sizeof(DevSlot);
   if (ws && ws_bytes >= slot_bytes) {
     rt->slots_ = ws;
@@ -141,8 +147,8 @@ std::unique_ptr<DeviceRT> DeviceRT::create(int device, void* ws, size_t ws_bytes
     rt->tune_file_ = e;
     if (FILE* f = std::fopen(e, "r")) {
       char sig[512];
-      int bn = 0, sp = 0;
-      while (std::fscanf(f, "%511s %d %d", sig, &bn, &sp) == 3) rt->tune_cache_[sig] = TcChoice{bn, sp};
+      int bn = 0, sp = 0, bk = 0;
+      while (std::fscanf(f, "%511s %d %d %d", sig, &bn, &sp, &bk) == 4) rt->tune_cache_[sig] = TcChoice{bn, sp, bk};
       std::fclose(f);
     }
   }
@@ -262,7 +268,8 @@ int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
     const std::string sig = tc_signature(op);
     auto it = tune_cache_.find(sig);
     if (it != tune_cache_.end()) {
-      if (it->second.bn != kd->choice_bn || it->second.splits != kd->choice_splits) {
+      if (it->second.bn != kd->choice_bn || it->second.splits != kd->choice_splits ||
+          it->second.bk != kd->choice_bk) {
         std::unique_ptr<KernelDesc> k2(new KernelDesc());
         std::string e2;
         if (build_tc_gemm(op, caps_, *k2, e2, &it->second)) {
@@ -275,10 +282,10 @@ int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
       }
     } else {
       if (!autotune_tc(op, kd, err)) return -1;
-      tune_cache_[sig] = TcChoice{kd->choice_bn, kd->choice_splits};
+      tune_cache_[sig] = TcChoice{kd->choice_bn, kd->choice_splits, kd->choice_bk};
       if (!tune_file_.empty()) {
         if (FILE* f = std::fopen(tune_file_.c_str(), "a")) {
-          std::fprintf(f, "%s %d %d\n", sig.c_str(), kd->choice_bn, kd->choice_splits);
+          std::fprintf(f, "%s %d %d %d\n", sig.c_str(), kd->choice_bn, kd->choice_splits, kd->choice_bk);
           std::fclose(f);
         }
       }
@@ -290,7 +297,8 @@ int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
 
 // Shape signature of a tc op for the tuning cache (pointers excluded).
 std::string DeviceRT::tc_signature(const bl_op& op) const {
-  std::string s = "k" + std::to_string(op.kind) + "_t" + std::to_string(op.dtype) + "_r" + (op.ptr[4] ? "1" : "0");
+  // "v2": tune files since the autotuner also picks BK (older lines never match)
+  std::string s = "v2k" + std::to_string(op.kind) + "_t" + std::to_string(op.dtype) + "_r" + (op.ptr[4] ? "1" : "0");
   for (int i = 0; i < 12; ++i) s += "_" + std::to_string(op.dims[i]);
   return s;
 }
@@ -301,8 +309,8 @@ std::string DeviceRT::tc_signature(const bl_op& op) const {
 // events, all S SMs) on the layer's own buffers; the fastest wins, and within
 // 3 % of it the one with fewer tiles (smaller d leaves more SMs to co-runners).
 bool DeviceRT::autotune_tc(const bl_op& op, std::unique_ptr<KernelDesc>& best, std::string& err) {
-  TcChoice cand[8];
-  const int nc = tc_candidates(op, caps_, cand, 8);
+  TcChoice cand[16];
+  const int nc = tc_candidates(op, caps_, cand, 16);
   if (nc <= 1) return true;
   if (!tune_stream_ && cudaStreamCreateWithFlags((cudaStream_t*)&tune_stream_, cudaStreamNonBlocking) != cudaSuccess) {
     err = "autotune stream";
@@ -318,11 +326,13 @@ bool DeviceRT::autotune_tc(const bl_op& op, std::unique_ptr<KernelDesc>& best, s
     if (!ok) return false;
   }
   for (int i = 0; i < nc; ++i) {
-    if (cand[i].bn == best->choice_bn && cand[i].splits == best->choice_splits) continue;
+    if (cand[i].bn == best->choice_bn && cand[i].splits == best->choice_splits && cand[i].bk == best->choice_bk)
+      continue;
     std::unique_ptr<KernelDesc> kd(new KernelDesc());
     std::string e2;
     if (!build_tc_gemm(op, caps_, *kd, e2, &cand[i])) continue;
-    if (kd->choice_bn == best->choice_bn && kd->choice_splits == best->choice_splits) {
+    if (kd->choice_bn == best->choice_bn && kd->choice_splits == best->choice_splits &&
+        kd->choice_bk == best->choice_bk) {
       if (kd->owned) cudaFree(kd->owned);
       continue;
     }
@@ -355,11 +365,12 @@ bool DeviceRT::autotune_tc(const bl_op& op, std::unique_ptr<KernelDesc>& best, s
 
 GateArgs DeviceRT::make_gate(uint64_t seq, uint32_t tiles, int lo, int hi, bool stamp, uint64_t prev_light) const {
   GateArgs g;
-  g.slot = reinterpret_cast<DevSlot*>(slots_) + seq % kSlotRing;
-  g.stats = reinterpret_cast<SlotStats*>(stats_dev_) + seq % kSlotRing;
-  g.stats_ahead = reinterpret_cast<SlotStats*>(stats_dev_) + (seq + kMaskAhead) % kSlotRing;
-  g.slot_ahead = reinterpret_cast<DevSlot*>(slots_) + (seq + kMaskAhead) % kSlotRing;
-  g.prev_stats = prev_light ? reinterpret_cast<SlotStats*>(stats_dev_) + prev_light % kSlotRing : nullptr;
+  const uint64_t R = ring_;
+  g.slot = reinterpret_cast<DevSlot*>(slots_) + seq % R;
+  g.stats = reinterpret_cast<SlotStats*>(stats_dev_) + seq % R;
+  g.stats_ahead = reinterpret_cast<SlotStats*>(stats_dev_) + (seq + ahead_) % R;
+  g.slot_ahead = reinterpret_cast<DevSlot*>(slots_) + (seq + ahead_) % R;
+  g.prev_stats = prev_light ? reinterpret_cast<SlotStats*>(stats_dev_) + prev_light % R : nullptr;
   g.lid_map = identity_map_ ? nullptr : lid_map_dev_;
   g.seq = seq;
   g.tiles = tiles;
@@ -521,6 +532,7 @@ bool DeviceRT::memcpy_async(void* dst, const void* src, size_t n, void* stream) 
 
 void DeviceRT::copy_range(uint64_t lo, uint64_t hi) {
   if (hi < lo) return;
+  const uint64_t kSlotRing = ring_;
   uint64_t n = std::min<uint64_t>(hi - lo + 1, kSlotRing);
   const uint64_t s0 = lo % kSlotRing;
   const uint64_t n1 = std::min<uint64_t>(n, kSlotRing - s0);
@@ -556,7 +568,7 @@ void DeviceRT::refresh_sync(uint64_t lo, uint64_t hi) {
 // publish): valid once the launch and its stream successor have finished and
 // the mirror was refreshed (Engine::stop after a device sync).
 void DeviceRT::peek(uint64_t seq, LaunchStats* out) {
-  const volatile SlotStats* s = reinterpret_cast<const volatile SlotStats*>(stats_host_) + (seq % kSlotRing);
+  const volatile SlotStats* s = reinterpret_cast<const volatile SlotStats*>(stats_host_) + (seq % ring_);
   out->start_host = gt_to_host(s->start_gt);
   out->end_host = gt_to_host(s->end_gt);
   int nsm = 0;
@@ -568,7 +580,7 @@ void DeviceRT::peek(uint64_t seq, LaunchStats* out) {
 
 bool DeviceRT::poll(uint64_t seq, LaunchStats* out) {
   if (!reader_idle()) return false;  // never read the mirror while a copy is landing
-  const volatile SlotStats* s = reinterpret_cast<const volatile SlotStats*>(stats_host_) + (seq % kSlotRing);
+  const volatile SlotStats* s = reinterpret_cast<const volatile SlotStats*>(stats_host_) + (seq % ring_);
   if (s->seq != seq) return false;
   std::atomic_thread_fence(std::memory_order_acquire);
   if (out) {

@@ -13,6 +13,12 @@
 
 namespace bless {
 
+// Default launch-slot/stats ring: 2^19 records (8 MiB of slots, 32 MiB of
+// stats on the device plus a 32 MiB pinned mirror); records stay readable for
+// 2^18 launches, more than one bench step of any config (C4: ~31k launches).
+// BLESS_STATS_RING_LOG2 (10..22) overrides it (tests).
+constexpr uint64_t kSlotRingDefault = 1ull << 19;
+
 struct LaunchStats {
   int64_t start_host, end_host;  // host clock (CLOCK_MONOTONIC ns)
   int nsm;
@@ -51,6 +57,12 @@ class DeviceRT {
   void refresh_async(uint64_t lo, uint64_t hi);
   void refresh_sync(uint64_t lo, uint64_t hi);
   uint64_t last_seq() const { return seq_; }
+  // Launch-slot / stats ring: ring() records; a launch zeroes the record
+  // ahead() seqs in front of it, so a record stays readable until ahead()
+  // later launches have started (Engine::stop reports older light launches
+  // as unknown instead of reading a reused record).
+  uint64_t ring() const { return ring_; }
+  uint64_t ahead() const { return ahead_; }
   // Parallel launch (Engine launcher threads): the scheduler thread allocates
   // the launch's seq; any thread may then launch it on its own stream.
   uint64_t alloc_seq() { return ++seq_; }
@@ -98,6 +110,8 @@ class DeviceRT {
   uint8_t* lid_map_dev_ = nullptr;
   bool identity_map_ = true;
   uint64_t seq_ = 0;
+  uint64_t ring_ = kSlotRingDefault;
+  uint64_t ahead_ = kSlotRingDefault / 2;
   std::vector<std::unique_ptr<KernelDesc>> kernels_;
   bool autotune_ = true;          // BLESS_TC_AUTOTUNE=0 keeps the builder's heuristic
   void* tune_stream_ = nullptr;
@@ -106,7 +120,5 @@ class DeviceRT {
   std::map<std::string, TcChoice> tune_cache_;   // BLESS_TC_TUNE_FILE
   std::string tune_file_;
 };
-
-constexpr uint64_t kSlotRing = 65536;
 
 }  // namespace bless

@@ -409,8 +409,13 @@ bl_status Engine::stop(std::string& err) {
     if (!rt_->device_sync()) { err = "device error at stop"; started_ = false; return BL_E_CUDA; }
     // every launch of the run has finished: mirror the whole stats range once
     // (includes the SM masks) and complete the logs
+    // Records older than ahead() launches have been zeroed for reuse by later
+    // launches: only the last ahead() seqs are read back; an older light
+    // launch (never published, so not harvested during the run) is reported
+    // as unknown (nsm = -1, no times) instead of from a reused record.
     const uint64_t hi = rt_->last_seq();
-    const uint64_t lo = hi >= run_first_seq_ ? std::max<uint64_t>(run_first_seq_, hi > kSlotRing ? hi - kSlotRing + 1 : 1) : hi + 1;
+    const uint64_t win = rt_->ahead();
+    const uint64_t lo = hi >= run_first_seq_ ? std::max<uint64_t>(run_first_seq_, hi > win ? hi - win + 1 : 1) : hi + 1;
     rt_->refresh_sync(lo, hi);
     harvest_all_ = true;
     harvest();
@@ -418,7 +423,10 @@ bl_status Engine::stop(std::string& err) {
     std::lock_guard<std::mutex> lk(log_mu_);
     for (bl_launch_rec& r : llog_) {
       LaunchStats st;
-      if (r.seq >= lo && r.seq <= hi) {
+      if (r.seq < lo && r.end_ns == 0) {
+        r.nsm = -1;
+        r.start_ns = 0;
+      } else if (r.seq >= lo && r.seq <= hi) {
         rt_->peek(r.seq, &st);   // light launches never publish their seq
         r.start_ns = st.start_host;
         r.end_ns = st.end_host;
@@ -455,6 +463,52 @@ bl_status Engine::reset(const bl_params* p, std::string& err) {
   std::lock_guard<std::mutex> lk(log_mu_);
   dlog_.clear();
   llog_.clear();
+  tlog_.clear();
+  return BL_OK;
+}
+
+bl_status Engine::temporal_log(size_t first, bl_temporal_rec* buf, size_t cap, size_t* n) {
+  std::lock_guard<std::mutex> lk(log_mu_);
+  size_t c = 0;
+  for (size_t i = first; i < tlog_.size() && c < cap; ++i) buf[c++] = tlog_[i];
+  if (n) *n = (buf == nullptr) ? tlog_.size() : c;
+  return BL_OK;
+}
+
+// Host cost of decide() (L436): the logged inputs of each record replayed reps
+// times on this thread, timed with the steady clock.
+bl_status Engine::time_decide(const bl_decision* recs, size_t n, int reps, int64_t* total_ns, int64_t* picks,
+                              std::string& err) {
+  if (!recs || reps < 1) { err = "bad args"; return BL_E_INVALID; }
+  if (!prof_.complete()) { err = "profile incomplete"; return BL_E_STATE; }
+  prof_.g = prm_.sm_unit;
+  prof_.derive();
+  std::vector<std::vector<ActiveReq>> in(n);
+  for (size_t r = 0; r < n; ++r) {
+    const bl_decision& d = recs[r];
+    if (d.n_active < 1 || d.n_active > nten()) { err = "bad active set"; return BL_E_INVALID; }
+    for (int i = 0; i < d.n_active; ++i) {
+      const int t = d.act_tenant[i];
+      if (t < 0 || t >= nten() || d.act_next[i] < 0 || d.act_next[i] >= (int)prof_.ten[t].k.size()) {
+        err = "bad active entry";
+        return BL_E_INVALID;
+      }
+      in[r].push_back({t, d.act_arrival[i], d.act_next[i]});
+    }
+  }
+  SchedParams sp{prm_.squad_max, prm_.split_pct, prm_.seed_all != 0, prm_.ablate};
+  Decision d;
+  DecideScratch sc;
+  int64_t np = 0;
+  const int64_t t0 = now_ns();
+  for (int rep = 0; rep < reps; ++rep)
+    for (size_t r = 0; r < n; ++r) {
+      decide(recs[r].now, in[r].data(), (int)in[r].size(), prof_, sp, d, sc);
+      np += (int64_t)d.picks.size();
+    }
+  const int64_t t1 = now_ns();
+  if (total_ns) *total_ns = t1 - t0;
+  if (picks) *picks = np;
   return BL_OK;
 }
 
@@ -1016,6 +1070,13 @@ void Engine::loop_temporal() {
     const int64_t host = now_ns();
     int j = -1;
     int64_t slice_end = 0, sid = 0;
+    // decision inputs for the log (bl_temporal_rec): which tenants have work
+    // now, and the T-wc turn state before this iteration
+    int32_t work_mask = 0;
+    for (int q = 0; q < nt; ++q)
+      if (act_req[q] >= 0 || (!fifo_[q].empty() && reqs_[fifo_[q].front()].arrival <= host)) work_mask |= 1 << q;
+    const int rec_turn = turn;
+    const int64_t rec_turn_end = turn_end;
     if (!prm_.temporal_work_conserving) {
       const int64_t cyc = (host - base) / P, pos = (host - base) % P;
       for (int q = 0; q < nt; ++q)
@@ -1033,7 +1094,8 @@ void Engine::loop_temporal() {
         }
         if (pick < 0) { turn = -1; cpu_relax(); continue; }
         turn = pick;
-        turn_end = host + len[pick];
+        // the turn starts when the GPU is free (the oracle DES, des.run_temporal)
+        turn_end = std::max(host, F) + len[pick];
         ++sid_wc;
       }
       j = turn;
@@ -1046,6 +1108,23 @@ void Engine::loop_temporal() {
     const int64_t st = std::max(F, host);
     const bool first = sid != last_sid;
     if (st < slice_end && (first || st + dur <= slice_end)) {
+      bl_temporal_rec rec{};
+      rec.t = host - base;
+      rec.gpu_free = F - base;
+      rec.slice_end = slice_end - base;
+      rec.dur = dur;
+      rec.sid = sid;
+      rec.last_sid = last_sid;
+      rec.turn = prm_.temporal_work_conserving ? rec_turn : -1;
+      rec.turn_end = prm_.temporal_work_conserving && rec_turn >= 0 ? rec_turn_end - base : 0;
+      rec.work_mask = work_mask;
+      rec.tenant = j;
+      rec.kernel = k;
+      rec.work_conserving = prm_.temporal_work_conserving ? 1 : 0;
+      {
+        std::lock_guard<std::mutex> lk(log_mu_);
+        tlog_.push_back(rec);
+      }
       if (!launch_one(j, k, 0, S(), temporal_stream_, (k == 0 || k == m - 1) ? act_req[j] : -1, k == m - 1)) return;
       F = st + dur;
       last_sid = sid;
@@ -1054,6 +1133,10 @@ void Engine::loop_temporal() {
         act_next[j] = 0;
       }
     } else {
+      // T-wc: a kernel that does not fit ends the turn at once (the next
+      // tenant with work takes over; des.run_temporal); T-cap idles to the
+      // end of the fixed slice
+      if (prm_.temporal_work_conserving) turn_end = host;
       cpu_relax();
     }
   }

@@ -121,6 +121,10 @@ class Engine {
   bl_status launches(size_t first, bl_launch_rec* buf, size_t cap, size_t* n);
   bl_status decide_pure(int64_t now, int n, const int32_t* ten, const int64_t* arr, const int32_t* nxt,
                         bl_decision* out, std::string& err);
+  bl_status temporal_log(size_t first, bl_temporal_rec* buf, size_t cap, size_t* n);
+  bl_status time_decide(const bl_decision* recs, size_t n, int reps, int64_t* total_ns, int64_t* picks,
+                        std::string& err);
+  bool virtual_clock() const { return prm_.clock == BL_CLOCK_VIRTUAL; }
 
  private:
   void thread_main();
@@ -195,6 +199,7 @@ class Engine {
   std::mutex log_mu_;
   std::vector<bl_decision> dlog_;
   std::vector<bl_launch_rec> llog_;
+  std::vector<bl_temporal_rec> tlog_;
 };
 
 }  // namespace bless

@@ -134,8 +134,18 @@ def test_c1_bless_wall_replay_bit_exact(lib_built, dtype, ablate, tmp_path):
     for r in ctx.launches():
         bits = mask_bits(r)
         assert all(r.lo <= b < r.hi for b in bits) and r.fallback == 0
-    # end-to-end numerics of the last request of each tenant (buffers hold it)
+    # numerics of the last request of each tenant (buffers hold it): every
+    # layer on its own GPU input at the north-star tolerance (R24: 1e-4 fp32,
+    # 1e-2 bf16), and for fp32 the whole model end to end at 1e-4 (no
+    # per-layer rounding to compound).  bf16 has no end-to-end bound: each
+    # layer rounds its output to bf16 (2^-9 relative) and SURVEY §8(c) C-4
+    # compares bf16 per layer only.
     for m in ms:
+        for k, layer in enumerate(m.layers):
+            err, tol = check_layer(layer, dtype)
+            assert err <= tol, (m.name, k, err)
+        if dtype != "fp32":
+            continue
         x = np64(m.input)
         for layer in m.layers:
             if layer.kind == "gemm":
@@ -143,7 +153,7 @@ def test_c1_bless_wall_replay_bit_exact(lib_built, dtype, ablate, tmp_path):
             else:
                 x = L.conv2d_nhwc(x, np64(layer.w), None, np64(layer.shift), 1, 1, 1, layer.act)
         err = L.max_rel_err(np64(m.output).reshape(x.shape), x)
-        assert err < (1e-4 if dtype == "fp32" else 5e-2), (m.name, err)
+        assert err < 1e-4, (m.name, err)
     ctx.close()
 
 
