@@ -2,15 +2,22 @@
 """BLESS hot-path benchmark (BASELINE.json metric: avg/p99 request latency per
 tenant at fixed quotas vs time-slice / static-split, and quota attainment %).
 
-A "step" is one pass of the whole hot path over one synthetic trace: the C++
-scheduler forms kernel squads from the tenants' Poisson arrivals and the
-SM-gated sm_100a kernels execute them (all of SURVEY.md §8(a)).  Workload at
-N=1: config C2 (VGG11 quota 1/3 + ResNet50 quota 2/3, bf16, batch 1, 224x224).
+A "step" is one pass of the whole hot path over one synthetic trace: the
+native dispatcher (bl_dispatch) hands each request to its GPU's context at its
+arrival time, the C++ scheduler forms kernel squads from the tenants' active
+requests and the SM-gated sm_100a kernels execute them (all of SURVEY.md
+§8(a)).  Workload at N=1: config C2 (VGG11 quota 1/3 + ResNet50 quota 2/3,
+bf16, batch 1, 224x224; BASELINE.json configs[1], the paper's Fig. 1 setup).
 `value` = mean request latency (ms) under BLESS over the K timed steps; the
-in-run baselines (ISO, STATIC, TEMPORAL T-cap and T-wc, UNBOUND) run on the
-same trace and executor.  Under torchrun every rank is an independent replica
-(no data-path collective; torch.distributed is used only for the barrier and
-the max-over-ranks of the step time).
+in-run baselines (ISO, STATIC, TEMPORAL T-cap and T-wc, UNBOUND) replay the
+same traces on the same executor.  C3 and C4 are reported beside it
+(`other_configs`, a load sweep each).
+
+Multi-GPU (replicas only, no NCCL): under torchrun every rank
+owns one GPU's context and dispatches its slice of one box-wide trace; without
+torchrun, `--gpus N` runs one process with N contexts and one dispatcher
+thread.  The ranks meet only on the host (gloo) for the barrier, the max of
+the step time and the whole-job sums.
 
 --impl reference times the oracle (oracle/: fp64 layer reference + the
 discrete-event model of the policy) on the host cores instead.
@@ -22,7 +29,6 @@ import json
 import os
 import subprocess
 import sys
-import tempfile
 import threading
 import time
 
@@ -40,7 +46,7 @@ CONFIG_NAMES = {"C1": "tiny MLP (1/3) + tiny CNN (2/3), fp32",
                 "C3": "ResNet50 (0.4) + VGG16 (0.3) + BERT-base s128 (0.2) + MobileNetV2 (0.1), bf16 batch 1",
                 "C4": "BERT-large s384 (1/2) + ResNet152 (1/4) + DenseNet121 (1/4), bf16 batch 1, bursty",
                 "C5": "per-GPU mix of C2/C3/C4 (GPU g hosts C[2 + g mod 3])"}
-
+SQUAD_MAX = {"C1": 4, "C2": 20, "C3": 10, "C4": 10}
 
 # tenant (name, quota) per config -- data only, so the reference arm imports
 # nothing from the product package
@@ -62,12 +68,11 @@ def parse():
     ap.add_argument("--rho", type=float, default=0.5, help="per-tenant load relative to its ISO latency")
     ap.add_argument("--rhos", default="", help="comma list: per-tenant rho (PAPER.md L298 workload E, biased load)")
     ap.add_argument("--quotas", default="", help="comma list: per-tenant quota override (PAPER.md Table 2 quota sets)")
-    ap.add_argument("--requests", type=int, default=60, help="requests per tenant per step")
-    # B200 operating point chosen by the c% x S_max sweep (DESIGN.md §9.3), the
+    ap.add_argument("--requests", type=int, default=100, help="requests per tenant per step (20 steps -> 2000)")
+    # B200 operating point chosen by the c% x S_max sweep (DESIGN.md §13), the
     # way the paper picks its own empirically (§6.7).
     ap.add_argument("--squad-max", type=int, default=None,
-                    help="S_max (L406-L408); default per config from the B200 sweeps in "
-                         "profiles/round1/param_sweep: C1 4, C2 20, C3 10, C4 10")
+                    help="S_max (L406-L408); default per config from the B200 sweeps: C1 4, C2 20, C3 10, C4 10")
     ap.add_argument("--split-pct", type=int, default=25)
     ap.add_argument("--ablate", type=int, default=0,
                     help="PAPER.md §6.8 ablation (R32): 1 = no multi-task scheduler, 2 = no determiner, 3 = both")
@@ -77,32 +82,30 @@ def parse():
     ap.add_argument("--no-baselines", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-slo", action="store_true", help="skip the SLO-mode experiment (§6.5)")
+    ap.add_argument("--also", default="C3,C4", help="other configs reported beside the headline (N=1 only)")
+    ap.add_argument("--also-rhos", default="0.3,0.5")
+    ap.add_argument("--also-requests", type=int, default=40)
     ap.add_argument("--load-profile", default="", help="reuse a saved profile table instead of profiling")
     ap.add_argument("--light", action="store_true", help="timed steps only (for ncu launch lists)")
     ap.add_argument("--out-dir", default=os.path.join(ROOT, "gpurun_out"))
-    return ap.parse_args()
-
-
-def default_squad_max(args):
-    """S_max per config unless given (B200 sweeps, profiles/round1/param_sweep)."""
-    if args.squad_max is None:
-        args.squad_max = {"C1": 4, "C2": 20, "C3": 10, "C4": 10}.get(args.config, 20)
+    a = ap.parse_args()
+    return a
 
 
 # ---------------------------------------------------------------------------- clocks
 class ClockSampler:
     """nvidia-smi clocks / throttle reasons sampled during the timed region."""
 
-    def __init__(self, gpu: int):
-        self.gpu, self.proc, self.lines = gpu, None, []
+    def __init__(self, gpus):
+        self.gpus, self.proc, self.lines = list(gpus), None, []
 
     def __enter__(self):
         q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
              "clocks_event_reasons.sw_power_cap")
         try:
-            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={q}",
-                                          "--format=csv,noheader,nounits", "-lms", "200"],
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", ",".join(str(g) for g in self.gpus),
+                                          f"--query-gpu={q}", "--format=csv,noheader,nounits", "-lms", "200"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.th = threading.Thread(target=self._read, daemon=True)
             self.th.start()
@@ -141,41 +144,40 @@ class ClockSampler:
 
 
 # ---------------------------------------------------------------------------- helpers
-def stats(xs):
-    xs = sorted(xs)
-    if not xs:
-        return {}
-    rank = lambda p: xs[max(0, int(np.ceil(p / 100 * len(xs))) - 1)]  # noqa: E731
-    return {"mean_ms": float(np.mean(xs)) / 1e6, "p50_ms": rank(50) / 1e6, "p99_ms": rank(99) / 1e6, "n": len(xs)}
-
-
 def squad_timeline(decisions, launches):
     """Map each BLESS decision to its launches (logged in pick order) and
     measure: squad makespan vs the predicted t_hat (Eq. 1 for SP, Eq. 2 for
     NSP; PAPER.md L214/L227 report 6.7%/7.1% error on A100) and the GPU idle
-    gap between consecutive squads (L432: 20 us squad switch on A100)."""
+    gap between consecutive squads (L432: 20 us squad switch on A100).  Gaps
+    are signed: a negative gap would be an overlap of squad s+1 with squad s
+    (a broken barrier); tests/test_gpu_concurrent.py asserts there is none
+    across tenants."""
     i = 0
     spans = []
     for d in decisions:
         ls = launches[i:i + d.n_picks]
         i += d.n_picks
-        if len(ls) != d.n_picks or any(r.end_ns <= 0 for r in ls):
+        if len(ls) != d.n_picks or any(r.end_ns <= 0 or r.nsm <= 0 for r in ls):
             continue
         spans.append((min(r.start_ns for r in ls), max(r.end_ns for r in ls), d.t_hat, bool(d.config_sp)))
     if not spans:
         return {}
     err = {True: [], False: []}
-    gaps = []
-    for a, b in zip(spans, spans[1:]):
-        gaps.append(max(0, b[0] - a[1]))
+    sgn = {True: [], False: []}
+    gaps = [b[0] - a[1] for a, b in zip(spans, spans[1:])]
     for s, e, th, sp in spans:
         err[sp].append(abs((e - s) - th) / max(1, e - s))
+        sgn[sp].append(((e - s) - th) / max(1, e - s))
+    med = lambda x: float(np.median(x)) / 1e3 if x else None  # noqa: E731
     return {"squads": len(spans),
             "pred_err_sp_pct": 100 * float(np.mean(err[True])) if err[True] else None,
             "pred_err_nsp_pct": 100 * float(np.mean(err[False])) if err[False] else None,
-            "gap_us_median": float(np.median(gaps)) / 1e3 if gaps else None,
-            "gap_us_mean": float(np.mean(gaps)) / 1e3 if gaps else None,
-            "makespan_us_median": float(np.median([e - s for s, e, _, _ in spans])) / 1e3}
+            "pred_bias_sp_pct": 100 * float(np.mean(sgn[True])) if sgn[True] else None,
+            "pred_bias_nsp_pct": 100 * float(np.mean(sgn[False])) if sgn[False] else None,
+            "gap_us_median": med(gaps), "gap_us_mean": float(np.mean(gaps)) / 1e3 if gaps else None,
+            "gap_us_min_signed": float(min(gaps)) / 1e3 if gaps else None,
+            "overlapping_squad_pairs": int(sum(1 for g in gaps if g < 0)),
+            "makespan_us_median": med([e - s for s, e, _, _ in spans])}
 
 
 def make_trace(T_iso, rho, n, seed, bursty=False):
@@ -189,38 +191,85 @@ def make_trace(T_iso, rho, n, seed, bursty=False):
     return syntrace.poisson(gaps, n, seed)
 
 
-def run_policy(ctx, capi, params, trace, tenants_filter=None):
-    """Replay a trace through the engine on the wall clock; returns per-tenant
-    latency lists (ns), launch records, decision records, and wall span."""
-    ctx.reset(params)
-    ctx.start()
+# ---------------------------------------------------------------------------- replicas
+class Replica:
+    """One GPU's sharing domain: ctx, tenant models, profile (L171)."""
+
+    def __init__(self, gpu, device, cfg, args, capi, models):
+        import torch
+        self.gpu, self.device, self.cfg = gpu, device, cfg
+        self.dtype = "fp32" if cfg == "C1" else "bf16"
+        self.squad_max = args.squad_max or SQUAD_MAX.get(cfg, 20)
+        with torch.cuda.device(device):
+            self.ctx = capi.Ctx(device, capi.default_params(squad_max=self.squad_max))
+            quotas = [float(x) for x in args.quotas.split(",")] if args.quotas and cfg == args.config else None
+            self.tms = models.build_config(self.ctx, cfg, self.dtype, quotas, device=device)
+        self.names = [m.name for m in self.tms]
+        self.info = self.ctx.device_info()
+        self.S = self.info.sm_count
+
+    def profile(self, args, out_dir, tag):
+        t0 = time.perf_counter()
+        if args.load_profile and self.cfg == args.config:
+            self.ctx.load_profile(args.load_profile)
+        else:
+            for m in self.tms:
+                self.ctx.profile_tenant(m.tenant, reps=args.profile_reps)
+        self.profile_s = time.perf_counter() - t0
+        self.prof_path = os.path.join(out_dir, f"profile_{self.cfg}_{tag}.txt")
+        self.ctx.save_profile(self.prof_path)
+        self.T_iso = [self.ctx.tenant_info(m.tenant)[2] for m in self.tms]
+        self.quota_sms = [self.ctx.tenant_info(m.tenant)[0] for m in self.tms]
+
+    def params(self, capi, args, pol="BLESS", extra=None):
+        return capi.default_params(squad_max=self.squad_max, policy=pol, split_pct=args.split_pct,
+                                   ablate=args.ablate, lookahead_ns=int(args.lookahead_us * 1000),
+                                   max_inflight_squads=args.max_inflight, **(extra or {}))
+
+
+def run_box(reps, capi, params_of, box, gpu_to_ctx, tenants_filter=None):
+    """Replay a box trace through the replicas this process owns, on the wall
+    clock: start every ctx, dispatch each request to its GPU's ctx at its
+    arrival time (native dispatcher thread, bl_dispatch), drain, stop.
+    Returns per replica: per-tenant latency lists (ns), launches, decisions."""
+    ctxs = [r.ctx for r in reps]
+    for r in reps:
+        r.ctx.reset(params_of(r))
+        r.ctx.start()
+    ents = [e for e in syntrace_entries(box, gpu_to_ctx)
+            if tenants_filter is None or e[1] in tenants_filter]
     base = capi.now_ns() + 3_000_000
-    ids = []
-    for a in trace:
-        if tenants_filter is not None and a.tenant not in tenants_filter:
-            continue
-        ids.append((a.tenant, ctx.submit(a.tenant, base + a.arrival_ns)))
-    ctx.drain(int(120e9))
-    ctx.stop()
-    lat = {}
-    first, last = None, 0
-    for t, r in ids:
-        st, info = ctx.poll(r)
-        assert st == capi.BL_OK
-        lat.setdefault(t, []).append(info.finish_ns - info.arrival_ns)
-        first = info.arrival_ns if first is None else min(first, info.arrival_ns)
-        last = max(last, info.finish_ns)
-    return lat, ctx.launches(), ctx.decisions(), (last - first)
+    ids = capi.dispatch(ctxs, ents, base)
+    for r in reps:
+        r.ctx.drain(int(300e9))
+        r.ctx.stop()
+    out = []
+    for i, r in enumerate(reps):
+        lat = {}
+        for (ci, t, _), q in zip(ents, ids):
+            if ci != i:
+                continue
+            st, info = r.ctx.poll(q)
+            assert st == capi.BL_OK
+            lat.setdefault(t, []).append(info.finish_ns - info.arrival_ns)
+        out.append((lat, r.ctx.launches(), r.ctx.decisions()))
+    return out
+
+
+def syntrace_entries(box, gpu_to_ctx):
+    return [(gpu_to_ctx[a.gpu], a.tenant, a.arrival_ns) for a in box if a.gpu in gpu_to_ctx]
 
 
 # ---------------------------------------------------------------------------- cpu baseline (oracle)
-def oracle_timing(cfg_models, decisions, prof, requests_per_tenant_seen, squads_per_req, params):
+def oracle_timing(cfg_models, decisions, prof, params, req_seen, squads_seen):
     """Time the oracle as it stands: one fp64 forward per tenant (all host
-    cores, numpy BLAS) plus decide_ref on a sample of decision records."""
+    cores, numpy BLAS) plus decide_ref on a sample of decision records (1
+    core); per request = forward + decide_ref x the squads that request took
+    part in (from the decision log, per tenant)."""
     from threadpoolctl import threadpool_info
 
     from oracle import models_ref
-    from oracle.sched_ref import Active, Params, decide_ref
+    from oracle.sched_ref import Active, decide_ref
     from paper_conf_eurosys_zhangcc0xz0g25_b200 import capi as _c
 
     fwd = {}
@@ -235,219 +284,48 @@ def oracle_timing(cfg_models, decisions, prof, requests_per_tenant_seen, squads_
         decide_ref(got["now"], [Active(*a) for a in got["active"]], prof, params)
         dec_t.append(time.perf_counter() - t0)
     mean_dec = float(np.mean(dec_t)) if dec_t else 0.0
-    per_req = [fwd[n] + mean_dec * squads_per_req for n in cfg_models]
-    weights = requests_per_tenant_seen
-    val = float(np.average(per_req, weights=weights)) * 1e3
+    per_req = [fwd[n] + mean_dec * squads_seen[j] / max(1, req_seen[j]) for j, n in enumerate(cfg_models)]
+    val = float(np.average(per_req, weights=[max(1, x) for x in req_seen])) * 1e3
     cores = max([x.get("num_threads", 1) for x in threadpool_info()] or [1])
     return {"value": val, "unit": "ms", "cores": int(cores), "kind": "oracle",
             "sample": f"1 fp64 forward per tenant ({', '.join(f'{k} {v:.2f}s' for k, v in fwd.items())}) + "
                       f"decide_ref on {len(dec_t)} logged decisions ({mean_dec * 1e6:.0f} us each, 1 core) x "
-                      f"{squads_per_req:.1f} squads/request",
+                      "the squads each tenant's request joined",
             "decide_ref_us_per_decision": mean_dec * 1e6}
 
 
-# ---------------------------------------------------------------------------- native arm
-def native(args):
-    import torch
+def replay_all(decisions, prof_path, params):
+    """Every logged decision through the oracle's decide_ref (bit-exact)."""
+    from oracle.sched_ref import Active, Prof, decide_ref
+    from paper_conf_eurosys_zhangcc0xz0g25_b200 import capi as _c
+    prof = Prof(synprof.load(prof_path))
+    ok = 0
+    for rec in decisions:
+        got = _c.decision_to_tuple(rec)
+        ref = decide_ref(got["now"], [Active(*a) for a in got["active"]], prof, params)
+        ok += int(got["picks"] == [tuple(p) for p in ref.picks] and got["config"] == ref.config
+                  and got["t_hat"] == ref.t_hat)
+    return f"{ok}/{len(decisions)}"
 
-    from paper_conf_eurosys_zhangcc0xz0g25_b200 import build as bld
-    bld.build(verbose=False)
-    from paper_conf_eurosys_zhangcc0xz0g25_b200 import capi, models, replicas
 
-    rank = int(os.environ.get("RANK", 0))
-    world = int(os.environ.get("WORLD_SIZE", 1))
-    local = int(os.environ.get("LOCAL_RANK", 0))
-    torch.cuda.set_device(local)
-    dist = None
-    if world > 1:
-        import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    plan = replicas.plan(rank, world, local, args.config, sorted(models.CONFIGS))
-    args.config = plan.config
-    default_squad_max(args)
-
-    dtype = "fp32" if args.config == "C1" else "bf16"
-    # tcgen05 tile configurations are autotuned at registration; a saved profile
-    # is only valid with the configurations it was measured with (tctune file)
-    os.makedirs(args.out_dir, exist_ok=True)
-    if args.load_profile:
-        tune = args.load_profile.replace("profile_", "tctune_")
-        if not os.path.exists(tune):
-            raise SystemExit(f"--load-profile needs its tuning file {tune}")
-    else:
-        tune = os.path.join(args.out_dir, f"tctune_{args.config}_rank{rank}.txt")
-        if os.path.exists(tune):
-            os.remove(tune)
-    os.environ["BLESS_TC_TUNE_FILE"] = tune
-    params = capi.default_params(squad_max=args.squad_max)
-    ctx = capi.Ctx(local, params)
-    info = ctx.device_info()
-    S = info.sm_count
-    quotas = [float(x) for x in args.quotas.split(",")] if args.quotas else None
-    tms = models.build_config(ctx, args.config, dtype, quotas)
-    rho = [float(x) for x in args.rhos.split(",")] if args.rhos else args.rho
-    names = [m.name for m in tms]
-    t_prof = time.perf_counter()
-    if args.load_profile:
-        ctx.load_profile(args.load_profile)
-    else:
-        for m in tms:
-            ctx.profile_tenant(m.tenant, reps=args.profile_reps)
-    t_prof = time.perf_counter() - t_prof
-    os.makedirs(args.out_dir, exist_ok=True)
-    prof_path = os.path.join(args.out_dir, f"profile_{args.config}_rank{rank}.txt")
-    ctx.save_profile(prof_path)
-    T_iso = [ctx.tenant_info(m.tenant)[2] for m in tms]
-    quota_sms = [ctx.tenant_info(m.tenant)[0] for m in tms]
-
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
-
-    def step(seed, pol="BLESS", filt=None, extra=None):
-        p = capi.default_params(squad_max=args.squad_max, policy=pol, split_pct=args.split_pct, ablate=args.ablate,
-                                lookahead_ns=int(args.lookahead_us * 1000), max_inflight_squads=args.max_inflight,
-                                **(extra or {}))
-        return run_policy(ctx, capi, p, make_trace(T_iso, rho, args.requests, seed + plan.trace_seed_offset,
-                                                   args.config == "C4"), filt)
-
-    for w in range(args.warmup):
-        flush.zero_()
-        step(100 + w)
-
-    # ---------------- timed region: K BLESS steps
-    lat_all = {j: [] for j in range(len(tms))}
-    launches_all, decisions_all = [], []
-    timelines = []
-    if dist:
-        dist.barrier()
-    torch.cuda.synchronize()
-    with ClockSampler(local) as clk:
-        t0 = time.perf_counter()
-        for k in range(args.steps):
-            flush.zero_()
-            lat, launches, decisions, span = step(1 + k % 3)
-            for j, v in lat.items():
-                lat_all[j].extend(v)
-            launches_all.extend(launches)
-            decisions_all.extend(decisions)
-            timelines.append((decisions, launches))
-        torch.cuda.synchronize()
-        t1 = time.perf_counter()
-    step_ms = replicas.max_over_ranks((t1 - t0) * 1e3 / args.steps, dist, device="cuda")
-    if dist:
-        dist.barrier()
-    n_local = sum(len(v) for v in lat_all.values())
-    agg = replicas.sum_over_ranks({"n": n_local, "lat_sum": float(sum(x for v in lat_all.values() for x in v))},
-                                  dist, device="cuda")
-    n_req = int(agg["n"])                          # whole job (all ranks)
-    mean_ms = agg["lat_sum"] / max(1.0, agg["n"]) / 1e6
-    if args.light:
-        if rank == 0:
-            print(json.dumps({"metric": METRIC, "value": mean_ms, "unit": "ms", "light": True,
-                              "gpu_launches": len(launches_all), "ms_per_step": step_ms}))
-        ctx.close()
-        return
-
-    # ---------------- in-run baselines on the SAME traces as the timed steps
-    # (each distinct seed once, weighted by how often the timed steps used it),
-    # so attainment and the BLESS-vs-baseline ratios compare like with like
-    per_tenant = {}
-    base = {}
-    iso_means = {}
-    seeds = [1 + k % 3 for k in range(args.steps)]
-    mult = {sd: seeds.count(sd) for sd in sorted(set(seeds))}
-
-    def run_seeds(pol, filt=None, extra=None):
-        out = {}
-        for sd, n in mult.items():
-            l, *_ = step(sd, pol, filt, extra)
-            for j, v in l.items():
-                out.setdefault(j, []).extend(v * n)
-        return out
-
-    if not args.no_baselines:
-        iso = {}
-        for j in range(len(tms)):
-            iso[j] = run_seeds("ISO", {j})[j]
-            iso_means[j] = float(np.mean(iso[j]))
-        base["ISO"] = {names[j]: stats(iso[j]) for j in iso}
-        base["ISO"]["all_mean_ms"] = float(np.mean([x for v in iso.values() for x in v])) / 1e6
-        runs = {"STATIC": ("STATIC", {}), "TEMPORAL_Tcap": ("TEMPORAL", {}),
-                "TEMPORAL_Twc": ("TEMPORAL", {"temporal_work_conserving": 1}), "UNBOUND": ("UNBOUND", {})}
-        base_lat = {}
-        for label, (pol, extra) in runs.items():
-            l = run_seeds(pol, None, extra)
-            base_lat[label] = l
-            base[label] = {names[j]: stats(v) for j, v in l.items()}
-            base[label]["all_mean_ms"] = float(np.mean([x for v in l.values() for x in v])) / 1e6
-        base["seeds"] = mult
-    for j in range(len(tms)):
-        s = stats(lat_all[j])
-        if iso_means:
-            s["attainment_pct"] = 100.0 * iso_means[j] / float(np.mean(lat_all[j]))
-        s["quota_sms"] = quota_sms[j]
-        s["T_iso_profile_ms"] = T_iso[j] / 1e6
-        per_tenant[names[j]] = s
-
-    # ---------------- SLO mode (§6.5): QoS target replaces T[n%] in
-    # the progress order; violation rate = share of requests over the target,
-    # for BLESS with the targets, default BLESS, and the baselines (same traces)
-    slo = None
-    if not args.no_baselines and not args.no_slo:
-        slo = {}
-        for label, fac in (("tight", (1.2, 2.0)), ("loose", (1.5, 3.0))):
-            tgt = [int(fac[j % 2] * T_iso[j]) for j in range(len(tms))]
-            for m, q in zip(tms, tgt):
-                ctx.set_slo(m.tenant, q)
-            ls = run_seeds("BLESS")
-            for m in tms:
-                ctx.set_slo(m.tenant, 0)
-
-            def viol(l):
-                n = sum(len(v) for v in l.values())
-                return 100.0 * sum(sum(1 for x in v if x > tgt[j]) for j, v in l.items()) / max(1, n)
-            row = {"targets_ms": {names[j]: tgt[j] / 1e6 for j in range(len(tms))},
-                   "factors_x_T_iso": list(fac), "violation_pct": {"BLESS_SLO": viol(ls), "BLESS": viol(lat_all)}}
-            row["violation_pct"].update({k: viol(v) for k, v in base_lat.items()})
-            row["BLESS_SLO_mean_ms"] = {names[j]: float(np.mean(v)) / 1e6 for j, v in ls.items()}
-            slo[label] = row
-
-    # ---------------- e2e: same metric with host buffers (H2D input, D2H output per request)
-    e2e = None
-    pinned = []
-    for m in tms:
-        hin = torch.empty(m.input.shape, dtype=m.input.dtype).pin_memory()
-        hin.copy_(m.input.cpu())
-        hout = torch.empty(m.output.shape, dtype=m.output.dtype).pin_memory()
-        pinned += [hin, hout]
-        ctx.set_tenant_io(m.tenant, hin.data_ptr(), m.input.data_ptr(), hin.numel() * hin.element_size(),
-                          m.output.data_ptr(), hout.data_ptr(), hout.numel() * hout.element_size())
-    le, *_ = step(1)
-    n_e = sum(len(v) for v in le.values())
-    h2d = sum(tms[j].input.numel() * tms[j].input.element_size() * len(v) for j, v in le.items())
-    d2h = sum(tms[j].output.numel() * tms[j].output.element_size() * len(v) for j, v in le.items())
-    e2e = {"value": float(np.mean([x for v in le.values() for x in v])) / 1e6, "unit": "ms",
-           "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h), "requests": n_e}
-    for m in tms:
-        ctx.set_tenant_io(m.tenant, 0, 0, 0, 0, 0, 0)
-
-    # ---------------- roofline of the dominant kernel (largest share of step time)
-    # "Kernel" = one kernel function (family, e.g. the tcgen05 GEMM/conv kernel):
-    # its launches' share of the step's device-busy time comes from the in-step
-    # stamps; achieved = sum of algorithmic work / sum of CUDA-event launch times
-    # (each layer of the family timed alone on its tenant stream, full GPU,
-    # weighted by its launch count in the timed steps).
-    peaks = {}
-    try:
-        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
-    except Exception:
-        pass
+# ---------------------------------------------------------------------------- roofline
+def roofline_of(rep, launches_all, peaks, args):
+    """Roofline of the dominant kernel (largest share of the step's device
+    time).  "Kernel" = one kernel function (family, e.g. the tcgen05 conv):
+    achieved = its algorithmic work / its CUDA-event launch time, each layer of
+    the family timed on its tenant stream over all S SMs (bl_profile_kernel,
+    back to back with PDL as inside a request), weighted by its launch count in
+    the timed steps.  Also per tenant the SM-share roofline fraction (SURVEY
+    §8(d)): sum_k t_roof(k, s) / sum_k t_meas(k) over the BLESS launches, with
+    t_roof = max(F / (P_tc * s/S), B / (BW * s/S))."""
+    ctx, S, names = rep.ctx, rep.S, rep.names
     hbm_peak = float(peaks.get("hbm_gbs", 6650.0))
     tc_peak = float(peaks.get("bf16_tflops", 1590.0))
     ridge = tc_peak * 1e12 / (hbm_peak * 1e9)
-    peak_src = "MEASURED_PEAKS.json" if peaks else "fallback (B200_PROFILING.md)"
+    peak_src = "MEASURED_PEAKS.json (burst)" if peaks else "fallback (B200_PROFILING.md)"
     busy, nlaunch = {}, {}
     for r in launches_all:
-        if r.end_ns > r.start_ns:
+        if r.end_ns > r.start_ns and r.nsm > 0:
             busy[(r.tenant, r.kernel)] = busy.get((r.tenant, r.kernel), 0) + (r.end_ns - r.start_ns)
             nlaunch[(r.tenant, r.kernel)] = nlaunch.get((r.tenant, r.kernel), 0) + 1
     total_busy = sum(busy.values())
@@ -475,46 +353,39 @@ def native(args):
     else:
         bound, unit, achieved, peak = "hbm", "GB/s", B / T, hbm_peak
     per_layer.sort(reverse=True)
-    # traffic: ncu dram bytes per launch of the same layers (committed capture,
-    # tools/traffic.py: each kernel alone on all SMs, cold L2), launch-weighted
+    nl = sum(nlaunch[tk] for tk in busy if fam_of[tk] == fam)
     traffic = None
-    tpath = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
+    tpath = os.path.join(ROOT, "profiles", f"traffic_{rep.cfg}.json")
     if os.path.exists(tpath):
         tl = json.load(open(tpath))["layers"]
         keys = [(tk, f"{names[tk[0]]}[{tk[1]}]") for tk in busy if fam_of[tk] == fam]
         if all(k in tl and tl[k]["dram_read"] is not None for _, k in keys):
-            nl = sum(nlaunch[tk] for tk, _ in keys)
             traffic = sum(nlaunch[tk] * (tl[k]["dram_read"] + tl[k]["dram_write"]) for tk, k in keys) / max(1, nl)
-    roofline = {"bound": bound, "achieved": achieved, "peak": peak, "unit": unit, "frac": achieved / peak,
-                "traffic": traffic, "traffic_source": f"profiles/traffic_{args.config}.json" if traffic else None,
-                "kernel": fam, "layers": len(per_layer),
-                "algorithmic_flops_per_launch": F / max(1, sum(nlaunch[tk] for tk in busy if fam_of[tk] == fam)),
-                "algorithmic_bytes_per_launch": B / max(1, sum(nlaunch[tk] for tk in busy if fam_of[tk] == fam)),
-                "event_avg_ns_per_launch": T / max(1, sum(nlaunch[tk] for tk in busy if fam_of[tk] == fam)),
-                "roofline_time_frac": TR / T, "instep_share": fam_busy[fam] / max(total_busy, 1),
-                "top_layers": [{"layer": nm, "event_ns": round(ev), "roofline_time_frac": round(fr, 3)}
-                               for _, nm, ev, fr in per_layer[:5]],
-                "peak_source": peak_src}
-    # the largest single HBM-bound launch (e.g. VGG FC1 weight stream), for reference
+    roof = {"bound": bound, "achieved": achieved, "peak": peak, "unit": unit, "frac": achieved / peak,
+            "traffic": traffic, "traffic_source": f"profiles/traffic_{rep.cfg}.json" if traffic else None,
+            "kernel": fam, "layers": len(per_layer),
+            "algorithmic_flops_per_launch": F / max(1, nl), "algorithmic_bytes_per_launch": B / max(1, nl),
+            "event_avg_ns_per_launch": T / max(1, nl), "roofline_time_frac": TR / T,
+            "instep_share": fam_busy[fam] / max(total_busy, 1),
+            "top_layers": [{"layer": nm, "event_ns": round(ev), "roofline_time_frac": round(fr, 3)}
+                           for _, nm, ev, fr in per_layer[:5]],
+            "peak_source": peak_src}
     hb = [tk for tk in busy if (lambda k: k.flops / max(k.bytes, 1.0) < ridge)(ctx.kernel_info(*tk))]
     if hb:
         tk = max(hb, key=lambda x: busy[x] / nlaunch[x])
         ki = ctx.kernel_info(*tk)
         ev, _ = ctx.profile_kernel(tk[0], tk[1], S, reps=20)
-        roofline["hbm_kernel"] = {"kernel": f"{names[tk[0]]}[{tk[1]}] {ki.family.decode()}", "bound": "hbm",
-                                  "achieved": ki.bytes / ev, "peak": hbm_peak, "unit": "GB/s",
-                                  "frac": ki.bytes / ev / hbm_peak, "algorithmic_bytes": ki.bytes,
-                                  "event_ns": ev}
+        roof["hbm_kernel"] = {"kernel": f"{names[tk[0]]}[{tk[1]}] {ki.family.decode()}", "bound": "hbm",
+                              "achieved": ki.bytes / ev, "peak": hbm_peak, "unit": "GB/s",
+                              "frac": ki.bytes / ev / hbm_peak, "algorithmic_bytes": ki.bytes, "event_ns": ev}
         if os.path.exists(tpath):
             rec = json.load(open(tpath))["layers"].get(f"{names[tk[0]]}[{tk[1]}]")
             if rec and rec["dram_read"] is not None:
-                roofline["hbm_kernel"]["traffic"] = rec["dram_read"] + rec["dram_write"]
-
-    # SM-share roofline per tenant: sum t_roof / sum t_meas over BLESS launches
-    kinfo = {(m.tenant, k): ctx.kernel_info(m.tenant, k) for m in tms for k in range(len(m.layers))}
+                roof["hbm_kernel"]["traffic"] = rec["dram_read"] + rec["dram_write"]
+    kinfo = {(m.tenant, k): ctx.kernel_info(m.tenant, k) for m in rep.tms for k in range(len(m.layers))}
     share = {}
     for r in launches_all:
-        if r.end_ns <= r.start_ns:
+        if r.end_ns <= r.start_ns or r.nsm <= 0:
             continue
         ki2 = kinfo[(r.tenant, r.kernel)]
         s_used = max(1, r.hi - r.lo)
@@ -522,56 +393,367 @@ def native(args):
         a = share.setdefault(names[r.tenant], [0.0, 0.0])
         a[0] += t_roof
         a[1] += r.end_ns - r.start_ns
-    for nm, (tr_, tm_) in share.items():
-        per_tenant[nm]["sm_share_roofline_frac"] = tr_ / tm_
+    return roof, {nm: tr_ / tm_ for nm, (tr_, tm_) in share.items()}
 
-    # ---------------- cpu baseline (oracle), rank 0 at N=1 only
+
+# ---------------------------------------------------------------------------- other configs (N=1)
+def other_config(cfg, args, capi, models, metrics, out_dir):
+    """A compact run of another config beside the headline: profile, then per
+    load rho BLESS / STATIC / TEMPORAL T-wc / ISO on seeds 1-3 (same traces):
+    mean latency per policy, attainment per tenant, deviation (L320)."""
+    rep = Replica(0, 0, cfg, args, capi, models)
+    rep.squad_max = args.squad_max or SQUAD_MAX[cfg]
+    rep.profile(argparse.Namespace(**{**vars(args), "load_profile": ""}), out_dir, "also")
+    res = {"workload": f"{cfg}: {CONFIG_NAMES[cfg]}", "squad_max": rep.squad_max, "T_iso_profile_ms":
+           {n: t / 1e6 for n, t in zip(rep.names, rep.T_iso)}, "rho": {}}
+    nt = len(rep.tms)
+    for rho in [float(x) for x in args.also_rhos.split(",") if x]:
+        lat = {}
+        for pol, extra in (("BLESS", None), ("STATIC", None), ("TEMPORAL_Twc", {"temporal_work_conserving": 1}),
+                           ("ISO", None)):
+            acc = {j: [] for j in range(nt)}
+            for seed in (1, 2, 3):
+                tr = make_trace(rep.T_iso, rho, args.also_requests, seed, cfg == "C4")
+                box = [syntrace.BoxArrival(a.arrival_ns, 0, a.tenant) for a in tr]
+                name = pol.split("_")[0]
+                if pol == "ISO":
+                    for j in range(nt):
+                        (l, _, _), = run_box([rep], capi, lambda r: r.params(capi, args, "ISO"), box, {0: 0}, {j})
+                        acc[j].extend(l.get(j, []))
+                else:
+                    (l, _, _), = run_box([rep], capi, lambda r: r.params(capi, args, name, extra), box, {0: 0})
+                    for j, v in l.items():
+                        acc[j].extend(v)
+            lat[pol] = acc
+        means = {p: {j: float(np.mean(v)) for j, v in acc.items()} for p, acc in lat.items()}
+        allm = {p: float(np.mean([x for v in acc.values() for x in v])) / 1e6 for p, acc in lat.items()}
+        att = {rep.names[j]: metrics.attainment_pct(means["ISO"][j], means["BLESS"][j]) for j in range(nt)}
+        res["rho"][str(rho)] = {
+            "mean_ms": allm,
+            "attainment_pct": att, "min_attainment_pct": min(att.values()),
+            "deviation_ms": {p: metrics.latency_deviation(means[p], means["ISO"]) / 1e6 for p in means if p != "ISO"},
+            "bless_beats_static": allm["BLESS"] < allm["STATIC"], "bless_beats_twc": allm["BLESS"] < allm["TEMPORAL_Twc"],
+            "time_domain_demand_D": float(rho * sum(_full_over_quota(rep)))}
+    rep.ctx.close()
+    return res
+
+
+def _full_over_quota(rep):
+    """T_j(S) / T_j(quota SMs) from the profile: the time-domain demand factor
+    per tenant (D = sum_j rho_j T_j(S)/T_j(q_j))."""
+    out = []
+    for m, Tq in zip(rep.tms, rep.T_iso):
+        TS = sum(rep.ctx.get_profile_row(m.tenant, k, rep.S)[0][rep.S - 1] for k in range(len(m.layers)))
+        out.append(TS / max(1, Tq))
+    return out
+
+
+# ---------------------------------------------------------------------------- native arm
+def native(args):
+    import torch
+
+    from paper_conf_eurosys_zhangcc0xz0g25_b200 import build as bld
+    bld.build(verbose=False)
+    from paper_conf_eurosys_zhangcc0xz0g25_b200 import capi, metrics, models, replicas
+
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("gloo")   # host-side barrier and reductions only (no NCCL: nothing shards)
+        gpus = [(rank, local)]
+    else:
+        gpus = [(g, g) for g in range(max(1, args.gpus))]
+    n_box = world if world > 1 else len(gpus)
+    os.makedirs(args.out_dir, exist_ok=True)
+    # tcgen05 tile configurations are autotuned at registration; a saved profile
+    # is only valid with the configurations it was measured with (tctune file)
+    if args.load_profile:
+        tune = args.load_profile.replace("profile_", "tctune_")
+        if not os.path.exists(tune):
+            raise SystemExit(f"--load-profile needs its tuning file {tune}")
+    else:
+        tune = os.path.join(args.out_dir, f"tctune_{args.config}_rank{rank}.txt")
+        if os.path.exists(tune):
+            os.remove(tune)
+    os.environ["BLESS_TC_TUNE_FILE"] = tune
+
+    reps = []
+    for g, dev in gpus:
+        torch.cuda.set_device(dev)
+        reps.append(Replica(g, dev, replicas.plan(g, args.config).config, args, capi, models))
+    for r in reps:
+        r.profile(args, args.out_dir, f"gpu{r.gpu}")
+    gpu_to_ctx = {r.gpu: i for i, r in enumerate(reps)}
+    # box-wide per-GPU T_iso -> the same box trace on every rank
+    tiso = {}
+    for part in replicas.gather({r.gpu: (r.T_iso, r.cfg) for r in reps}, dist):
+        tiso.update(part)
+    rho_t = [float(x) for x in args.rhos.split(",")] if args.rhos else None
+
+    def box_of(seed):
+        gaps, bursty = [], []
+        for g in range(n_box):
+            T, cfg = tiso[g]
+            rr = rho_t if (rho_t and cfg == args.config) else [args.rho] * len(T)
+            gaps.append([t / x for t, x in zip(T, rr)])
+            bursty.append(cfg == "C4")
+        return syntrace.box_trace(gaps, args.requests, seed, bursty)
+
+    def step(seed, pol="BLESS", filt=None, extra=None):
+        return run_box(reps, capi, lambda r: r.params(capi, args, pol, extra), box_of(seed), gpu_to_ctx, filt)
+
+    flush = [torch.empty(256 << 20, dtype=torch.uint8, device=f"cuda:{r.device}") for r in reps]
+
+    def flush_l2():
+        for f in flush:
+            f.zero_()
+
+    for w in range(args.warmup):
+        flush_l2()
+        step(100 + w)
+
+    # ---------------- timed region: K BLESS steps
+    nrep = len(reps)
+    lat_all = [{j: [] for j in range(len(r.tms))} for r in reps]
+    seed_lat = {}
+    launches_all = [[] for _ in reps]
+    decisions_all = [[] for _ in reps]
+    timelines = []
+    replicas.barrier(dist)
+    for r in reps:
+        torch.cuda.synchronize(r.device)
+    with ClockSampler([r.device for r in reps]) as clk:
+        t0 = time.perf_counter()
+        for k in range(args.steps):
+            flush_l2()
+            sd = 1 + k % 3
+            out = step(sd)
+            for i, (lat, launches, decisions) in enumerate(out):
+                for j, v in lat.items():
+                    lat_all[i][j].extend(v)
+                    seed_lat.setdefault(sd, []).extend(v)
+                launches_all[i].extend(launches)
+                decisions_all[i].extend(decisions)
+                if i == 0:
+                    timelines.append((decisions, launches))
+        for r in reps:
+            torch.cuda.synchronize(r.device)
+        t1 = time.perf_counter()
+    step_ms = replicas.max_over_ranks((t1 - t0) * 1e3 / args.steps, dist)
+    replicas.barrier(dist)
+    n_local = sum(len(v) for la in lat_all for v in la.values())
+    agg = replicas.sum_over_ranks({"n": n_local, "lat_sum": float(sum(x for la in lat_all for v in la.values()
+                                                                     for x in v))}, dist)
+    n_req = int(agg["n"])
+    mean_ms = agg["lat_sum"] / max(1.0, agg["n"]) / 1e6
+    gpu_launches = int(replicas.sum_over_ranks({"l": sum(len(x) for x in launches_all)}, dist)["l"])
+    if args.light:
+        if rank == 0:
+            print(json.dumps({"metric": METRIC, "value": mean_ms, "unit": "ms", "light": True,
+                              "gpu_launches": gpu_launches, "ms_per_step": step_ms}))
+        for r in reps:
+            r.ctx.close()
+        return
+
+    # ---------------- in-run baselines on the SAME traces as the timed steps
+    # (each distinct seed once, weighted by how often the timed steps used it)
+    seeds = [1 + k % 3 for k in range(args.steps)]
+    mult = {sd: seeds.count(sd) for sd in sorted(set(seeds))}
+
+    def run_seeds(pol, filt_of=None, extra=None):
+        out = [{} for _ in reps]
+        for sd, n in mult.items():
+            if filt_of is None:
+                res = step(sd, pol, None, extra)
+                for i, (l, _, _) in enumerate(res):
+                    for j, v in l.items():
+                        out[i].setdefault(j, []).extend(v * n)
+            else:
+                for filt in filt_of:
+                    res = step(sd, pol, filt, extra)
+                    for i, (l, _, _) in enumerate(res):
+                        for j, v in l.items():
+                            out[i].setdefault(j, []).extend(v * n)
+        return out
+
+    def key(i, j):
+        return reps[i].names[j] if nrep == 1 else f"gpu{reps[i].gpu}:{reps[i].names[j]}"
+
+    per_tenant, base, iso_means, base_lat, deviation = {}, {}, {}, {}, {}
+    bless_means = {(i, j): float(np.mean(v)) for i in range(nrep) for j, v in lat_all[i].items() if v}
+    if not args.no_baselines:
+        maxt = max(len(r.tms) for r in reps)
+        iso = run_seeds("ISO", [{j} for j in range(maxt)])
+        iso_means = {(i, j): float(np.mean(v)) for i in range(nrep) for j, v in iso[i].items()}
+        base["ISO"] = {key(i, j): metrics.summary_ms(v) for i in range(nrep) for j, v in iso[i].items()}
+        base["ISO"]["all_mean_ms"] = float(np.mean([x for d in iso for v in d.values() for x in v])) / 1e6
+        runs = {"STATIC": ("STATIC", {}), "TEMPORAL_Tcap": ("TEMPORAL", {}),
+                "TEMPORAL_Twc": ("TEMPORAL", {"temporal_work_conserving": 1}), "UNBOUND": ("UNBOUND", {})}
+        for label, (pol, extra) in runs.items():
+            lsb = run_seeds(pol, None, extra)
+            base_lat[label] = lsb
+            base[label] = {key(i, j): metrics.summary_ms(v) for i in range(nrep) for j, v in lsb[i].items()}
+            base[label]["all_mean_ms"] = float(np.mean([x for d in lsb for v in d.values() for x in v])) / 1e6
+            means = {(i, j): float(np.mean(v)) for i in range(nrep) for j, v in lsb[i].items()}
+            deviation[label] = metrics.latency_deviation(means, iso_means) / 1e6
+        base["seeds"] = mult
+        deviation["BLESS"] = metrics.latency_deviation(bless_means, iso_means) / 1e6
+    for i in range(nrep):
+        for j in range(len(reps[i].tms)):
+            s = metrics.summary_ms(lat_all[i][j])
+            if iso_means:
+                s["attainment_pct"] = metrics.attainment_pct(iso_means[(i, j)], bless_means[(i, j)])
+            s["quota_sms"] = reps[i].quota_sms[j]
+            s["T_iso_profile_ms"] = reps[i].T_iso[j] / 1e6
+            per_tenant[key(i, j)] = s
+    atts = [s["attainment_pct"] for s in per_tenant.values() if "attainment_pct" in s]
+
+    # ---------------- SLO mode (§6.5, L364-L366): QoS target replaces T[n%] in
+    # the progress order; violation rate = share of requests over the target
+    slo = None
+    if not args.no_baselines and not args.no_slo:
+        slo = {}
+        for label, fac in (("tight", (1.2, 2.0)), ("loose", (1.5, 3.0))):
+            tgt = {(i, j): int(fac[j % 2] * iso_means[(i, j)]) for i in range(nrep) for j in range(len(reps[i].tms))}
+            for i, r in enumerate(reps):
+                for m in r.tms:
+                    r.ctx.set_slo(m.tenant, tgt[(i, m.tenant)])
+            ls = run_seeds("BLESS")
+            for r in reps:
+                for m in r.tms:
+                    r.ctx.set_slo(m.tenant, 0)
+
+            def viol(l):
+                n = sum(len(v) for d in l for v in d.values())
+                return 100.0 * sum(sum(1 for x in v if x > tgt[(i, j)]) for i, d in enumerate(l)
+                                   for j, v in d.items()) / max(1, n)
+            row = {"targets_ms": {key(i, j): v / 1e6 for (i, j), v in tgt.items()},
+                   "factors_x_measured_ISO_mean": list(fac),
+                   "violation_pct": {"BLESS_SLO": viol(ls), "BLESS": viol(lat_all)}}
+            row["violation_pct"].update({k: viol(v) for k, v in base_lat.items()})
+            row["BLESS_SLO_mean_ms"] = {key(i, j): float(np.mean(v)) / 1e6 for i, d in enumerate(ls)
+                                        for j, v in d.items()}
+            slo[label] = row
+
+    # ---------------- e2e: same metric with host buffers (H2D input, D2H output per request)
+    pinned = []
+    for r in reps:
+        for m in r.tms:
+            hin = torch.empty(m.input.shape, dtype=m.input.dtype).pin_memory()
+            hin.copy_(m.input.cpu())
+            hout = torch.empty(m.output.shape, dtype=m.output.dtype).pin_memory()
+            pinned += [hin, hout]
+            r.ctx.set_tenant_io(m.tenant, hin.data_ptr(), m.input.data_ptr(), hin.numel() * hin.element_size(),
+                                m.output.data_ptr(), hout.data_ptr(), hout.numel() * hout.element_size())
+    le = step(1)
+    h2d = sum(r.tms[j].input.numel() * r.tms[j].input.element_size() * len(v)
+              for r, (l, _, _) in zip(reps, le) for j, v in l.items())
+    d2h = sum(r.tms[j].output.numel() * r.tms[j].output.element_size() * len(v)
+              for r, (l, _, _) in zip(reps, le) for j, v in l.items())
+    e2e_all = [x for (l, _, _) in le for v in l.values() for x in v]
+    e2e = {"value": float(np.mean(e2e_all)) / 1e6, "unit": "ms", "h2d_bytes_per_step": int(h2d),
+           "d2h_bytes_per_step": int(d2h), "requests": len(e2e_all),
+           "path": "bl_set_tenant_io: pinned host input -> device per request, output -> pinned host; a request "
+                   "completes when its output has landed in host memory"}
+    for r in reps:
+        for m in r.tms:
+            r.ctx.set_tenant_io(m.tenant, 0, 0, 0, 0, 0, 0)
+
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        pass
+    roofline, share = roofline_of(reps[0], launches_all[0], peaks, args)
+    for nm, fr in share.items():
+        per_tenant[nm if nrep == 1 else f"gpu{reps[0].gpu}:{nm}"]["sm_share_roofline_frac"] = fr
+
+    # ---------------- host cost of the C++ scheduler (L436), 1 core
+    dec = decisions_all[0]
+    decide_cost = None
+    if dec:
+        r0 = reps[0]
+        r0.ctx.reset(r0.params(capi, args))
+        ns, picks = r0.ctx.time_decide(dec, reps=3)
+        decide_cost = {"us_per_decision": ns / (3 * len(dec)) / 1e3, "us_per_kernel": ns / max(1, picks) / 1e3,
+                       "decisions": len(dec), "cores": 1,
+                       "paper_us_per_kernel": 6.7, "paper_host": "AMD EPYC 7302 (L282, L436)"}
+
+    # ---------------- cpu baseline (oracle) + full decision replay, rank 0 at N=1 only
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        from oracle.sched_ref import Params, Prof
-        prof = Prof(synprof.load(prof_path))
-        sq = len(decisions_all) / max(1, n_local)
-        cpu = oracle_timing(names, decisions_all, prof, [len(lat_all[j]) for j in range(len(tms))], sq * 2,
-                            Params(squad_max=args.squad_max, split_pct=args.split_pct, ablate=args.ablate))
-
-    # decisions replayed bit-exactly through the oracle (sample)
     replay_ok = None
     if rank == 0:
-        from oracle.sched_ref import Active, Params, Prof, decide_ref
-        prof = Prof(synprof.load(prof_path))
-        replay_ok = 0
-        for rec in decisions_all[:200]:
-            got = capi.decision_to_tuple(rec)
-            ref = decide_ref(got["now"], [Active(*a) for a in got["active"]], prof, Params(squad_max=args.squad_max, split_pct=args.split_pct, ablate=args.ablate))
-            replay_ok += int(got["picks"] == [tuple(p) for p in ref.picks] and got["config"] == ref.config
-                             and got["t_hat"] == ref.t_hat)
-        replay_ok = f"{replay_ok}/{min(200, len(decisions_all))}"
+        from oracle.sched_ref import Params, Prof
+        r0 = reps[0]
+        prm = Params(squad_max=r0.squad_max, split_pct=args.split_pct, ablate=args.ablate)
+        replay_ok = replay_all(dec, r0.prof_path, prm)
+        if world == 1 and nrep == 1 and not args.no_cpu_baseline:
+            prof = Prof(synprof.load(r0.prof_path))
+            sq_seen = [sum(1 for d in dec if j in [d.part_tenant[x] for x in range(d.n_part)])
+                       for j in range(len(r0.tms))]
+            cpu = oracle_timing(r0.names, dec, prof, prm, [len(lat_all[0][j]) for j in range(len(r0.tms))], sq_seen)
 
-    gpu_launches = len(launches_all)
-    fallbacks = sum(r.fallback for r in launches_all)
-    sp_squads = sum(1 for d in decisions_all if d.config_sp)
+    tl = [squad_timeline(d, l) for d, l in timelines]
+    tl = [t for t in tl if t]
+    timeline = {}
+    if tl:
+        timeline = {k: (float(np.mean([t[k] for t in tl if t.get(k) is not None]))
+                        if any(t.get(k) is not None for t in tl) else None)
+                    for k in tl[0] if k not in ("squads", "overlapping_squad_pairs", "gap_us_min_signed")}
+        timeline["squads"] = int(sum(t["squads"] for t in tl))
+        timeline["overlapping_squad_pairs"] = int(sum(t["overlapping_squad_pairs"] for t in tl))
+        mins = [t["gap_us_min_signed"] for t in tl if t.get("gap_us_min_signed") is not None]
+        timeline["gap_us_min_signed"] = min(mins) if mins else None
+
+    others = {}
+    if rank == 0 and world == 1 and nrep == 1 and args.also and not args.no_baselines:
+        for cfg in [c for c in args.also.split(",") if c and c != args.config]:
+            others[cfg] = other_config(cfg, args, capi, models, metrics, args.out_dir)
+
+    fallbacks = sum(r.fallback for la in launches_all for r in la)
+    seed_means = {str(sd): float(np.mean(v)) / 1e6 for sd, v in sorted(seed_lat.items())}
+    bmean = {k: v["all_mean_ms"] for k, v in base.items() if isinstance(v, dict) and "all_mean_ms" in v}
+    r0 = reps[0]
     out = {
-        "metric": METRIC, "value": mean_ms, "unit": "ms", "n_gpus": world, "steps": args.steps,
+        "metric": METRIC, "value": mean_ms, "unit": "ms", "n_gpus": n_box, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": step_ms, "higher_is_better": False, "scaling": "weak",
-        "vs_baseline": None, "dtype": "bf16" if dtype == "bf16" else "f32", "data": "synthetic",
+        "vs_baseline": None, "dtype": "bf16" if r0.dtype == "bf16" else "f32", "data": "synthetic",
         "config": {"workload": f"{args.config}: {CONFIG_NAMES[args.config]}",
+                   "per_gpu_configs": {str(g): tiso[g][1] for g in sorted(tiso)},
                    "trace": f"{'MMPP-2 bursty' if args.config == 'C4' else 'Poisson'} rho={args.rhos or args.rho} "
-                   f"per tenant, {args.requests} requests/tenant/step, seeds 1-3", "squad_max": args.squad_max,
+                   f"per tenant, {args.requests} requests/tenant/step, seeds 1-3, box-wide trace routed by the "
+                   "native dispatcher (bl_dispatch)", "squad_max": r0.squad_max,
                    "split_pct": args.split_pct, "ablate": args.ablate,
-                   "parallelism": f"replicas x{world} (no collective)",
-                   "quotas": [m.quota for m in tms],
+                   "parallelism": f"replicas x{n_box} (no collective; "
+                                  f"{'one process per GPU, gloo host barrier' if world > 1 else 'one process'})",
+                   "quotas": [m.quota for m in r0.tms],
                    "l2": "256 MiB buffer written between timed steps (> 126 MB L2); VGG11 weights 266 MB > L2"},
-        "per_tenant": per_tenant, "baselines": base, "slo": slo, "requests_per_s": n_req / (step_ms * args.steps / 1e3),
+        "min_attainment_pct": min(atts) if atts else None,
+        "vs_static": mean_ms / bmean["STATIC"] if "STATIC" in bmean else None,
+        "vs_temporal_twc": mean_ms / bmean["TEMPORAL_Twc"] if "TEMPORAL_Twc" in bmean else None,
+        "vs_temporal_tcap": mean_ms / bmean["TEMPORAL_Tcap"] if "TEMPORAL_Tcap" in bmean else None,
+        "vs_unbound": mean_ms / bmean["UNBOUND"] if "UNBOUND" in bmean else None,
+        "deviation_ms": deviation or None,
+        "seed_means_ms": seed_means,
+        "seed_std_ms": float(np.std(list(seed_means.values()))) if seed_means else None,
+        "per_tenant": per_tenant, "baselines": base, "slo": slo,
+        "requests_per_s": n_req / (step_ms * args.steps / 1e3), "requests": n_req,
         "e2e": e2e, "gpu_launches": gpu_launches, "roofline": roofline, "cpu_baseline": cpu,
         "clocks": clk.summary(),
-        "scheduler": {"decisions": len(decisions_all), "sp_squads": sp_squads, "fallback_launches": fallbacks,
-                      "oracle_replay_bit_exact": replay_ok, "profile_s": t_prof,
-                      "timeline": squad_timeline(*timelines[0]) if timelines else {}},
-        "device": {"sm_count": S, "globaltimer_res_ns": info.globaltimer_res_ns, "host_cores": os.cpu_count()},
+        "scheduler": {"decisions": sum(len(d) for d in decisions_all),
+                      "sp_squads": sum(1 for dd in decisions_all for d in dd if d.config_sp),
+                      "fallback_launches": fallbacks, "oracle_replay_bit_exact": replay_ok,
+                      "decide_cost": decide_cost, "profile_s": r0.profile_s, "timeline": timeline},
+        "other_configs": others or None,
+        "device": {"sm_count": r0.S, "globaltimer_res_ns": r0.info.globaltimer_res_ns, "host_cores": os.cpu_count()},
     }
     if rank == 0:
         print(json.dumps(out))
-    ctx.close()
+    for r in reps:
+        r.ctx.close()
     if dist:
         dist.destroy_process_group()
 
@@ -587,7 +769,7 @@ def reference(args):
 
     cfg = "C2" if args.config == "C5" else args.config
     args.config = cfg
-    default_squad_max(args)
+    squad_max = args.squad_max or SQUAD_MAX[cfg]
     tenants = REF_CONFIGS[cfg]
     names = [n for n, _ in tenants]
     # profile table: the last B200 profile committed under profiles/, else a synthetic stand-in
@@ -603,8 +785,8 @@ def reference(args):
     vals = []
     for it in range(args.warmup + args.steps):
         t0 = time.perf_counter()
-        trace = make_trace(prof.T, args.rho, max(4, args.requests // 10), 1 + it % 3, cfg == "C4")
-        res = des.run_bless(trace, prof, Params(squad_max=args.squad_max, split_pct=args.split_pct, ablate=args.ablate))
+        trace = make_trace(prof.T, args.rho, max(4, args.requests // 20), 1 + it % 3, cfg == "C4")
+        des.run_bless(trace, prof, Params(squad_max=squad_max, split_pct=args.split_pct, ablate=args.ablate))
         t_dec = time.perf_counter() - t0
         fw = {}
         for i, n in enumerate(names):
@@ -621,7 +803,7 @@ def reference(args):
            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
            "config": {"workload": f"{args.config}: {CONFIG_NAMES[args.config]}", "profile": src},
            "cpu_baseline": {"value": v, "unit": "ms", "cores": int(cores), "kind": "oracle",
-                            "sample": f"per step: DES+decide_ref over a {max(4, args.requests // 10)}-request/tenant "
+                            "sample": f"per step: DES+decide_ref over a {max(4, args.requests // 20)}-request/tenant "
                                       "trace + one fp64 forward per tenant"},
            "e2e": {"value": v, "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out))

@@ -427,9 +427,19 @@ CONFIGS = {
 }
 
 
-def build_config(ctx: capi.Ctx, cfg: str, dtype: str, quotas: Optional[Sequence[float]] = None) -> List[TenantModel]:
+def build_config(ctx: capi.Ctx, cfg: str, dtype: str, quotas: Optional[Sequence[float]] = None,
+                 device: Optional[int] = None) -> List[TenantModel]:
     """Register and build the tenants of a config; ``quotas`` overrides the
-    config's quota per tenant (Table 2's two-model quota sets, L295)."""
+    config's quota per tenant (Table 2's two-model quota sets, L295).
+    ``device``: CUDA device of the tenants' memory (default: the ctx's)."""
+    dev = ctx.device if device is None else device
+    if dev is not None and dev >= 0 and torch.cuda.is_available():
+        with torch.cuda.device(dev):
+            return _build_config(ctx, cfg, dtype, quotas)
+    return _build_config(ctx, cfg, dtype, quotas)
+
+
+def _build_config(ctx, cfg, dtype, quotas):
     models = []
     spec = CONFIGS[cfg]
     if quotas is not None:

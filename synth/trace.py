@@ -86,6 +86,35 @@ def mmpp2(mean_gap_ns: Sequence[float], n_per_tenant: int, seed: int, on_frac: f
     return _sort(out)
 
 
+@dataclass(frozen=True)
+class BoxArrival:
+    """One request of the box-wide trace: GPU, tenant, time."""
+    arrival_ns: int
+    gpu: int
+    tenant: int
+
+
+def box_trace(per_gpu_gaps: Sequence[Sequence[float]], n_per_tenant: int, seed: int,
+              bursty: Sequence[bool] = ()) -> List[BoxArrival]:
+    """Box-wide merge of per-GPU traces (config C5).  GPU g's tenants draw
+    their own Poisson (or, if bursty[g], MMPP-2) arrivals from seed
+    seed * 1000 + g, so GPU g's slice of the box trace does not depend on how
+    many GPUs the box has; the merge is sorted by (arrival, gpu, tenant)."""
+    out = []
+    for g, gaps in enumerate(per_gpu_gaps):
+        sub_seed = seed * 1000 + g
+        sub = mmpp2(gaps, n_per_tenant, sub_seed) if (g < len(bursty) and bursty[g]) else \
+            poisson(gaps, n_per_tenant, sub_seed)
+        out.extend(BoxArrival(a.arrival_ns, g, a.tenant) for a in sub)
+    out.sort(key=lambda a: (a.arrival_ns, a.gpu, a.tenant))
+    return out
+
+
+def gpu_slice(box: Sequence[BoxArrival], gpu: int) -> List[Arrival]:
+    """GPU g's requests of a box trace (the dispatcher's routing)."""
+    return [Arrival(a.arrival_ns, a.tenant) for a in box if a.gpu == gpu]
+
+
 def save(path: str, arrs: Sequence[Arrival]) -> None:
     with open(path, "w") as f:
         for a in arrs:
