@@ -154,12 +154,22 @@ def squad_timeline(decisions, launches):
     across tenants."""
     i = 0
     spans = []
+    viol = 0
+    prev = None
     for d in decisions:
         ls = launches[i:i + d.n_picks]
         i += d.n_picks
         if len(ls) != d.n_picks or any(r.end_ns <= 0 or r.nsm <= 0 for r in ls):
+            prev = None
             continue
         spans.append((min(r.start_ns for r in ls), max(r.end_ns for r in ls), d.t_hat, bool(d.config_sp)))
+        if prev is not None:   # barrier: no launch starts before ANOTHER tenant's squad-s end
+            for r in ls:
+                others = [e for t, e in prev.items() if t != r.tenant]
+                viol += int(bool(others) and r.start_ns < max(others) - 64)
+        prev = {}
+        for r in ls:
+            prev[r.tenant] = max(prev.get(r.tenant, 0), r.end_ns)
     if not spans:
         return {}
     err = {True: [], False: []}
@@ -176,7 +186,12 @@ def squad_timeline(decisions, launches):
             "pred_bias_nsp_pct": 100 * float(np.mean(sgn[False])) if sgn[False] else None,
             "gap_us_median": med(gaps), "gap_us_mean": float(np.mean(gaps)) / 1e3 if gaps else None,
             "gap_us_min_signed": float(min(gaps)) / 1e3 if gaps else None,
-            "overlapping_squad_pairs": int(sum(1 for g in gaps if g < 0)),
+            # squad s+1 starting before squad s ends on the SAME tenant stream is
+            # the programmatic-dependent-launch prologue overlap (the kernel
+            # waits in griddepcontrol.wait before touching data); a start before
+            # ANOTHER tenant's end would be a broken barrier
+            "pdl_overlapped_switches": int(sum(1 for g in gaps if g < 0)),
+            "barrier_violations": viol,
             "makespan_us_median": med([e - s for s, e, _, _ in spans])}
 
 
@@ -702,9 +717,11 @@ def native(args):
     if tl:
         timeline = {k: (float(np.mean([t[k] for t in tl if t.get(k) is not None]))
                         if any(t.get(k) is not None for t in tl) else None)
-                    for k in tl[0] if k not in ("squads", "overlapping_squad_pairs", "gap_us_min_signed")}
+                    for k in tl[0] if k not in ("squads", "pdl_overlapped_switches", "barrier_violations",
+                                                "gap_us_min_signed")}
         timeline["squads"] = int(sum(t["squads"] for t in tl))
-        timeline["overlapping_squad_pairs"] = int(sum(t["overlapping_squad_pairs"] for t in tl))
+        timeline["pdl_overlapped_switches"] = int(sum(t["pdl_overlapped_switches"] for t in tl))
+        timeline["barrier_violations"] = int(sum(t["barrier_violations"] for t in tl))
         mins = [t["gap_us_min_signed"] for t in tl if t.get("gap_us_min_signed") is not None]
         timeline["gap_us_min_signed"] = min(mins) if mins else None
 
