@@ -348,6 +348,25 @@ bl_status bl_decide(bl_ctx* ctx, int64_t now, int n_active, const int32_t* tenan
 bl_status bl_time_decide(bl_ctx* ctx, const bl_decision* recs, size_t n, int reps, int64_t* total_ns,
                          int64_t* total_picks);
 
+/* ---- predictor study -------------
+ * bl_predict: predicted duration of one squad given as n picks (tenant,
+ * kernel) in pick order: p == NULL -> Eq. 2 (NSP, L224, reading R12); else
+ * Eq. 1 (L211) for the spatial split p[0..K-1] over the K participants in
+ * tenant-id order (partitions of g SMs, each >= 1, summing to N; the last
+ * participant gets the remaining S - g*(N - p_last) SMs).  Needs a complete
+ * profile; BL_E_INVALID on a bad pick or split.
+ * bl_run_squad: executes one squad as given on the device (ctx not started):
+ * each participant's picks in pick order on its stream, SM range [lo[i],
+ * hi[i]) per pick, all chains released together by one event, every launch
+ * stamped; repeated reps times.  makespan_ns = median over reps of (last end
+ * - first start); kernel_ns[i] (may be NULL) = median duration of pick i.
+ * This is how the study measures NSP, SP, Semi-SP and SEQ squads (L197-L203,
+ * L382) against the predictions. */
+bl_status bl_predict(bl_ctx* ctx, int n_picks, const int32_t* tenants, const int32_t* kernels, const int32_t* p,
+                     int64_t* ns_out);
+bl_status bl_run_squad(bl_ctx* ctx, int n_picks, const int32_t* tenants, const int32_t* kernels, const int16_t* lo,
+                       const int16_t* hi, int reps, int64_t* makespan_ns, int64_t* kernel_ns);
+
 /* ---- box-wide trace dispatcher ("replicating
  * its runtime components for each active GPU") -----------------------------------
  * One host thread routes a merged trace of several GPUs' tenants: entry i goes

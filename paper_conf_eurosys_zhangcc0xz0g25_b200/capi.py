@@ -136,6 +136,9 @@ _SIGS = {
     "bl_time_decide": (C.c_int, [C.c_void_p, _P(bl_decision), C.c_size_t, C.c_int, _P(C.c_int64), _P(C.c_int64)]),
     "bl_dispatch": (C.c_int, [_P(C.c_void_p), C.c_int, _P(bl_dispatch_entry), C.c_size_t, C.c_int64,
                               _P(C.c_uint64)]),
+    "bl_predict": (C.c_int, [C.c_void_p, C.c_int, _P(C.c_int32), _P(C.c_int32), _P(C.c_int32), _P(C.c_int64)]),
+    "bl_run_squad": (C.c_int, [C.c_void_p, C.c_int, _P(C.c_int32), _P(C.c_int32), _P(C.c_int16), _P(C.c_int16),
+                               C.c_int, _P(C.c_int64), _P(C.c_int64)]),
     "bl_debug_overhead": (C.c_int, [C.c_void_p, C.c_int, C.c_int, _P(C.c_int64)]),
     "bl_now_ns": (C.c_int64, []),
     "bl_last_error": (C.c_char_p, []),
@@ -327,6 +330,28 @@ class Ctx:
         ns, picks = C.c_int64(), C.c_int64()
         check("bl_time_decide", lib().bl_time_decide(self.h, arr, len(recs), int(reps), C.byref(ns), C.byref(picks)))
         return ns.value, picks.value
+
+    def predict(self, picks, p=None) -> int:
+        """Eq. 2 (p None, NSP) or Eq. 1 for split p of a squad [(tenant, kernel)]."""
+        n = len(picks)
+        t = (C.c_int32 * n)(*[x[0] for x in picks])
+        k = (C.c_int32 * n)(*[x[1] for x in picks])
+        pp = (C.c_int32 * len(p))(*p) if p is not None else None
+        out = C.c_int64()
+        check("bl_predict", lib().bl_predict(self.h, n, t, k, pp, C.byref(out)))
+        return out.value
+
+    def run_squad(self, picks, reps: int = 3):
+        """Execute a squad [(tenant, kernel, lo, hi)]: (median makespan ns, per-pick ns)."""
+        n = len(picks)
+        t = (C.c_int32 * n)(*[x[0] for x in picks])
+        k = (C.c_int32 * n)(*[x[1] for x in picks])
+        lo = (C.c_int16 * n)(*[x[2] for x in picks])
+        hi = (C.c_int16 * n)(*[x[3] for x in picks])
+        ms = C.c_int64()
+        kn = (C.c_int64 * n)()
+        check("bl_run_squad", lib().bl_run_squad(self.h, n, t, k, lo, hi, int(reps), C.byref(ms), kn))
+        return ms.value, list(kn)
 
     def decide(self, now: int, active):
         """active: list of (tenant, arrival, next_kernel)."""

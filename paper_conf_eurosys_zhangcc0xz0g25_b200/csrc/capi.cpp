@@ -211,6 +211,15 @@ bl_status bl_dispatch(bl_ctx* const* ctxs, int n_ctx, const bl_dispatch_entry* e
     return BL_OK;
   });
 }
+bl_status bl_predict(bl_ctx* ctx, int n, const int32_t* ten, const int32_t* ker, const int32_t* p, int64_t* out) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->predict(n, ten, ker, p, out, e); });
+}
+bl_status bl_run_squad(bl_ctx* ctx, int n, const int32_t* ten, const int32_t* ker, const int16_t* lo,
+                       const int16_t* hi, int reps, int64_t* makespan, int64_t* kernel_ns) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->run_squad(n, ten, ker, lo, hi, reps, makespan, kernel_ns, e); });
+}
 bl_status bl_reset(bl_ctx* ctx, const bl_params* p) {
   GUARD(ctx);
   return wrap([&](std::string& e) { return ctx->eng->reset(p, e); });

@@ -577,6 +577,103 @@ bl_status Engine::decide_pure(int64_t now, int n, const int32_t* ten, const int6
   return BL_OK;
 }
 
+// Participants (tenant-id order) and their kernels in pick order, validated.
+static bool squad_of(const Profile& prof, int n, const int32_t* ten, const int32_t* ker, std::vector<int>& parts,
+                     std::vector<std::vector<int>>& ks, std::string& err) {
+  const int nt = (int)prof.ten.size();
+  if (n < 1 || !ten || !ker) { err = "empty squad"; return false; }
+  std::vector<std::vector<int>> by(nt);
+  for (int i = 0; i < n; ++i) {
+    if (ten[i] < 0 || ten[i] >= nt || ker[i] < 0 || ker[i] >= (int)prof.ten[ten[i]].k.size()) {
+      err = "bad pick " + std::to_string(i);
+      return false;
+    }
+    by[ten[i]].push_back(ker[i]);
+  }
+  parts.clear();
+  ks.clear();
+  for (int j = 0; j < nt; ++j)
+    if (!by[j].empty()) { parts.push_back(j); ks.push_back(by[j]); }
+  return true;
+}
+
+bl_status Engine::predict(int n, const int32_t* ten, const int32_t* ker, const int32_t* p, int64_t* out,
+                          std::string& err) {
+  if (!out) { err = "null out"; return BL_E_INVALID; }
+  if (!prof_.complete()) { err = "profile incomplete"; return BL_E_STATE; }
+  prof_.g = prm_.sm_unit;
+  prof_.derive();
+  std::vector<int> parts;
+  std::vector<std::vector<int>> ks;
+  if (!squad_of(prof_, n, ten, ker, parts, ks, err)) return BL_E_INVALID;
+  if (!p) {
+    *out = predict_nsp(prof_, parts, ks);
+    return BL_OK;
+  }
+  std::vector<int> pv(p, p + parts.size());
+  int sum = 0;
+  for (int x : pv) {
+    if (x < 1) { err = "every participant needs >= 1 partition"; return BL_E_INVALID; }
+    sum += x;
+  }
+  if (sum != prof_.N) { err = "partitions must sum to N"; return BL_E_INVALID; }
+  *out = predict_sp(prof_, parts, ks, pv);
+  return BL_OK;
+}
+
+// One squad as given (f1 study): each participant's picks in order on its
+// stream, every chain released by one event, every launch with the full exit
+// protocol (start/end stamps); reps times, medians.
+bl_status Engine::run_squad(int n, const int32_t* ten, const int32_t* ker, const int16_t* lo, const int16_t* hi,
+                            int reps, int64_t* makespan, int64_t* kernel_ns, std::string& err) {
+  if (!rt_) { err = "no device"; return BL_E_STATE; }
+  if (started_) { err = "run_squad while running"; return BL_E_STATE; }
+  if (n < 1 || !ten || !ker || !lo || !hi || reps < 1 || !makespan) { err = "bad args"; return BL_E_INVALID; }
+  for (int i = 0; i < n; ++i)
+    if (ten[i] < 0 || ten[i] >= nten() || ker[i] < 0 || ker[i] >= (int)ten_[ten[i]].handles.size() ||
+        lo[i] < 0 || hi[i] > S() || lo[i] >= hi[i]) {
+      err = "bad pick " + std::to_string(i);
+      return BL_E_INVALID;
+    }
+  rt_->set_device();
+  if (!temporal_stream_) temporal_stream_ = rt_->stream_create();
+  void* go = rt_->event_create();
+  std::vector<std::vector<int64_t>> kd(n);
+  std::vector<int64_t> ms;
+  std::vector<uint64_t> seqs(n);
+  for (int r = 0; r < reps; ++r) {
+    if (!rt_->device_sync()) { err = "device error"; rt_->event_destroy(go); return BL_E_CUDA; }
+    rt_->event_record(go, temporal_stream_);
+    std::vector<int> waited(nten(), 0);
+    for (int i = 0; i < n; ++i) {
+      TenantRT& t = ten_[ten[i]];
+      if (!waited[ten[i]]) { rt_->stream_wait(t.stream, go); waited[ten[i]] = 1; }
+      seqs[i] = rt_->launch(t.handles[ker[i]], lo[i], hi[i], t.stream, err, true);
+      if (!seqs[i]) { rt_->event_destroy(go); return BL_E_CUDA; }
+    }
+    if (!rt_->device_sync()) { err = "device error"; rt_->event_destroy(go); return BL_E_CUDA; }
+    rt_->refresh_sync(seqs.front(), seqs.back());
+    int64_t a = INT64_MAX, b = 0;
+    for (int i = 0; i < n; ++i) {
+      LaunchStats st{};
+      if (!rt_->poll(seqs[i], &st)) { err = "squad launch stats missing"; rt_->event_destroy(go); return BL_E_CUDA; }
+      kd[i].push_back(st.end_host - st.start_host);
+      a = std::min(a, st.start_host);
+      b = std::max(b, st.end_host);
+    }
+    ms.push_back(b - a);
+  }
+  rt_->event_destroy(go);
+  auto med = [](std::vector<int64_t> v) {
+    std::sort(v.begin(), v.end());
+    return v[v.size() / 2];
+  };
+  *makespan = med(ms);
+  if (kernel_ns)
+    for (int i = 0; i < n; ++i) kernel_ns[i] = med(kd[i]);
+  return BL_OK;
+}
+
 void Engine::log_decision(const Decision& d) {
   bl_decision r;
   to_record(d, r);

@@ -125,6 +125,9 @@ class Engine {
   bl_status time_decide(const bl_decision* recs, size_t n, int reps, int64_t* total_ns, int64_t* picks,
                         std::string& err);
   bool virtual_clock() const { return prm_.clock == BL_CLOCK_VIRTUAL; }
+  bl_status predict(int n, const int32_t* ten, const int32_t* ker, const int32_t* p, int64_t* out, std::string& err);
+  bl_status run_squad(int n, const int32_t* ten, const int32_t* ker, const int16_t* lo, const int16_t* hi, int reps,
+                      int64_t* makespan, int64_t* kernel_ns, std::string& err);
 
  private:
   void thread_main();

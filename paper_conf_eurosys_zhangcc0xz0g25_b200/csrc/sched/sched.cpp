@@ -330,4 +330,43 @@ void decide(int64_t now, const ActiveReq* act, int n_act, const Profile& prof, c
   }
 }
 
+// Eq. 2 (L224, R12) for a given squad: levels i = 0..q-1, x_i = min(S, sum of
+// d over the level), work-equivalent time t[d]*d/x past a kernel's d (same
+// arithmetic as decide()).
+int64_t predict_nsp(const Profile& prof, const std::vector<int>& parts, const std::vector<std::vector<int>>& ks) {
+  const int K = (int)parts.size(), S = prof.S;
+  int q = 0;
+  for (int i = 0; i < K; ++i) q = std::max(q, (int)ks[i].size());
+  int64_t t = 0;
+  for (int lv = 0; lv < q; ++lv) {
+    int64_t x = 0;
+    for (int i = 0; i < K; ++i)
+      if ((int)ks[i].size() > lv) x += prof.ten[parts[i]].k[ks[i][lv]].d;
+    x = std::min<int64_t>(x, S);
+    for (int i = 0; i < K; ++i) {
+      if ((int)ks[i].size() <= lv) continue;
+      const int j = parts[i], k = ks[i][lv];
+      const int dk = prof.ten[j].k[k].d;
+      t += (x <= dk) ? prof.t(j, k, (int)x) : (prof.t(j, k, dk) * dk) / x;
+      t += io_of(prof, j, k);
+    }
+  }
+  return t;
+}
+
+// Eq. 1 (L211) for a given composition p of N partitions (R9-R11): the
+// slowest participant chain on its g*p_i SMs (the last one gets the rest).
+int64_t predict_sp(const Profile& prof, const std::vector<int>& parts, const std::vector<std::vector<int>>& ks,
+                   const std::vector<int>& p) {
+  const int K = (int)parts.size(), S = prof.S, g = prof.g, N = prof.N;
+  int64_t worst = 0;
+  for (int i = 0; i < K; ++i) {
+    const int s = (i < K - 1) ? g * p[i] : S - g * (N - p[i]);
+    int64_t sum = 0;
+    for (int k : ks[i]) sum += prof.t(parts[i], k, s) + io_of(prof, parts[i], k);
+    worst = std::max(worst, sum);
+  }
+  return worst;
+}
+
 }  // namespace bless

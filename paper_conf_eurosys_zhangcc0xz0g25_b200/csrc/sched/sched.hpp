@@ -97,4 +97,11 @@ struct DecideScratch {
 void decide(int64_t now, const ActiveReq* act, int n_act, const Profile& prof, const SchedParams& prm,
             Decision& out, DecideScratch& scratch);
 
+// The two squad-duration predictors for a GIVEN squad and configuration (the
+// f1 predictor study, PAPER.md L214/L227/L237): parts = participants in
+// tenant-id order, ks[i] = participant i's kernels in pick order.
+int64_t predict_nsp(const Profile& prof, const std::vector<int>& parts, const std::vector<std::vector<int>>& ks);
+int64_t predict_sp(const Profile& prof, const std::vector<int>& parts, const std::vector<std::vector<int>>& ks,
+                   const std::vector<int>& p);
+
 }  // namespace bless

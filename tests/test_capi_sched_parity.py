@@ -227,3 +227,37 @@ def test_ablate_out_of_range_rejected():
     with pytest.raises(capi.BlessError) as e:
         capi.Ctx(capi.BL_DEVICE_NONE, clock=capi.BL_CLOCK_VIRTUAL, ablate=4)
     assert e.value.status == capi.BL_E_INVALID
+
+
+@settings(max_examples=150, deadline=None)
+@given(world(), st.integers(0, 10_000))
+def test_predict_matches_oracle_eq1_eq2(tmp_path_factory, w, pseed):
+    """bl_predict (the f1 study's predictor entry point) == the oracle's Eq. 2
+    (NSP) and Eq. 1 (any split) on the decision's own squad; the decision's
+    t_nsp / t_hat are the same numbers."""
+    from oracle.sched_ref import compositions, per_participant, predict_nsp, predict_sp
+    pf, active, now, params = w
+    path = str(tmp_path_factory.mktemp("pr") / "p.txt")
+    sp.save(path, pf)
+    ctx = capi.Ctx(capi.BL_DEVICE_NONE, clock=capi.BL_CLOCK_VIRTUAL, **{**params, "ablate": 0})
+    ctx.load_profile(path)
+    prof = Prof(pf)
+    rec = ctx.decide(now, active)
+    got = capi.decision_to_tuple(rec)
+    picks = [(t, k) for t, k, _, _ in got["picks"]]
+    ks = per_participant(picks)
+    assert ctx.predict(picks) == predict_nsp(ks, prof)[0] == got["t_nsp"]
+    K = len(ks)
+    if K >= 2:
+        comps = list(compositions(prof.N, K))
+        rng = np.random.Generator(np.random.PCG64(pseed))
+        for i in rng.choice(len(comps), size=min(8, len(comps)), replace=False):
+            p = comps[int(i)]
+            assert ctx.predict(picks, list(p)) == predict_sp(ks, p, prof)[0]
+        if got["config"] is not None:
+            assert ctx.predict(picks, list(got["config"])) == got["t_hat"]
+    with pytest.raises(capi.BlessError):
+        ctx.predict(picks, [prof.N + 1] + [1] * (K - 1))
+    ns, npk = ctx.time_decide([rec], reps=2)
+    assert ns > 0 and npk == 2 * len(picks)
+    ctx.close()

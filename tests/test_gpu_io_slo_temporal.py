@@ -157,3 +157,21 @@ def test_temporal_decisions_replay(c2, wc, tmp_path):
         assert rec.kernel == nxt.get(rec.tenant, 0), i
         nxt[rec.tenant] = (rec.kernel + 1) % prof.m[rec.tenant]
     print(f"\nTEMPORAL {'T-wc' if wc else 'T-cap'}: {len(log)} launch decisions replayed through the R22 rule")
+
+
+def test_run_squad_and_predict(c2):
+    """bl_run_squad executes a given squad (the f1 study's measurement): NSP on
+    all SMs and an SP split; every pick's duration is positive, the makespan
+    covers the longest chain; bl_predict gives Eq. 2 / Eq. 1 for the same squad."""
+    ctx, ms = c2
+    ctx.reset(capi.default_params(policy="BLESS", squad_max=20))
+    S = ctx.device_info().sm_count
+    picks = [(0, k) for k in range(3)] + [(1, k) for k in range(5)]
+    nsp, kn = ctx.run_squad([(t, k, 0, S) for t, k in picks], reps=3)
+    assert all(x > 0 for x in kn) and nsp >= max(kn)
+    split = [(0, 49), (49, S)]
+    sp, kn2 = ctx.run_squad([(t, k, *split[t]) for t, k in picks], reps=3)
+    assert all(x > 0 for x in kn2) and sp >= max(sum(kn2[:3]), max(kn2[3:])) * 0.5
+    pn, ps = ctx.predict(picks), ctx.predict(picks, [12, 25])
+    assert pn > 0 and ps > 0
+    print(f"\nsquad NSP {nsp / 1e3:.1f} us (Eq. 2 {pn / 1e3:.1f}), SP 49/99 {sp / 1e3:.1f} us (Eq. 1 {ps / 1e3:.1f})")
