@@ -102,7 +102,12 @@ typedef struct {
                                  progress order); bit 1 = no execution configuration
                                  determiner (every squad NSP on [0,S)).  BL_E_INVALID
                                  outside 0..3 at bl_create. */
-  int32_t reserved0;          /* 0 */
+  int32_t sm_limit;           /* f4 SM-count sweep (L420): 0 = all S SMs; else the whole
+                                 system (every policy, the profile columns, quota
+                                 apportionment, N = sm_limit / g) is restricted to logical
+                                 SMs [0, sm_limit) for the run, the way the paper restricts
+                                 the GPU with MIG.  BL_E_INVALID at bl_start unless
+                                 g <= sm_limit <= S. */
 } bl_params;
 
 /* Fill *p with the defaults listed above. */
@@ -366,6 +371,29 @@ bl_status bl_predict(bl_ctx* ctx, int n_picks, const int32_t* tenants, const int
                      int64_t* ns_out);
 bl_status bl_run_squad(bl_ctx* ctx, int n_picks, const int32_t* tenants, const int32_t* kernels, const int16_t* lo,
                        const int16_t* hi, int reps, int64_t* makespan_ns, int64_t* kernel_ns);
+
+/* ---- deployment (§4.2.2) --------------------
+ * Reading R33.  A tenant's average kernel duration is T_j / m_j (isolated
+ * latency at its quota over its kernel count, from the profile).  A set of
+ * tenants may share one GPU iff (a) the largest average kernel duration is at
+ * most span_x times the smallest (L163: co-locating short-kernel with
+ * extremely long-kernel applications starves the former in every squad; the
+ * paper's working range is 10 us to 300 us, i.e. span_x = 30), and (b) their
+ * memory fits the device's free memory (L169).
+ * bl_deployment_check: the ctx's registered, profiled tenants; mem_bytes[j]
+ * per tenant; free_bytes <= 0 queries the device (cudaMemGetInfo; BL_E_STATE
+ * on a device-less ctx).  *ok_out = 1 admissible, 0 not; *reason_out (may be
+ * NULL) = 0 ok, 1 kernel-duration span, 2 memory.
+ * bl_place (L171, "a central controller can leverage the memory requirement
+ * and profiled kernel information to decide which specific GPU to place
+ * applications"): apps in order of decreasing memory (ties: smaller index),
+ * each to the GPU with the most remaining free memory among those where it
+ * fits and keeps rule (a) (ties: smaller GPU index); gpu_out[i] = -1 if none.
+ * Pure host function (no ctx). */
+bl_status bl_deployment_check(bl_ctx* ctx, const int64_t* mem_bytes, int64_t free_bytes, int32_t span_x,
+                              int32_t* ok_out, int32_t* reason_out);
+bl_status bl_place(int n_apps, const int64_t* mem_bytes, const int64_t* avg_kernel_ns, int n_gpus,
+                   const int64_t* gpu_free_bytes, int32_t span_x, int32_t* gpu_out);
 
 /* ---- box-wide trace dispatcher ("replicating
  * its runtime components for each active GPU") -----------------------------------

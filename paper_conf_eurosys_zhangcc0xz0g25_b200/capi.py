@@ -41,7 +41,7 @@ class bl_params(C.Structure):
                 ("squad_overhead_ns", C.c_int64), ("temporal_period_ns", C.c_int64),
                 ("temporal_work_conserving", C.c_int32), ("max_inflight_squads", C.c_int32),
                 ("lookahead_ns", C.c_int64), ("max_requests", C.c_int64),
-                ("ablate", C.c_int32), ("reserved0", C.c_int32)]
+                ("ablate", C.c_int32), ("sm_limit", C.c_int32)]
 
 
 class bl_op(C.Structure):
@@ -139,6 +139,10 @@ _SIGS = {
     "bl_predict": (C.c_int, [C.c_void_p, C.c_int, _P(C.c_int32), _P(C.c_int32), _P(C.c_int32), _P(C.c_int64)]),
     "bl_run_squad": (C.c_int, [C.c_void_p, C.c_int, _P(C.c_int32), _P(C.c_int32), _P(C.c_int16), _P(C.c_int16),
                                C.c_int, _P(C.c_int64), _P(C.c_int64)]),
+    "bl_deployment_check": (C.c_int, [C.c_void_p, _P(C.c_int64), C.c_int64, C.c_int32, _P(C.c_int32),
+                                      _P(C.c_int32)]),
+    "bl_place": (C.c_int, [C.c_int, _P(C.c_int64), _P(C.c_int64), C.c_int, _P(C.c_int64), C.c_int32,
+                           _P(C.c_int32)]),
     "bl_debug_overhead": (C.c_int, [C.c_void_p, C.c_int, C.c_int, _P(C.c_int64)]),
     "bl_now_ns": (C.c_int64, []),
     "bl_last_error": (C.c_char_p, []),
@@ -353,6 +357,14 @@ class Ctx:
         check("bl_run_squad", lib().bl_run_squad(self.h, n, t, k, lo, hi, int(reps), C.byref(ms), kn))
         return ms.value, list(kn)
 
+    def deployment_check(self, mem_bytes, free_bytes: int = 0, span_x: int = 30):
+        """(admissible, reason): reason 0 ok, 1 kernel-duration span, 2 memory (R33)."""
+        m = (C.c_int64 * len(mem_bytes))(*[int(x) for x in mem_bytes])
+        ok, why = C.c_int32(), C.c_int32()
+        check("bl_deployment_check", lib().bl_deployment_check(self.h, m, int(free_bytes), int(span_x),
+                                                               C.byref(ok), C.byref(why)))
+        return bool(ok.value), why.value
+
     def decide(self, now: int, active):
         """active: list of (tenant, arrival, next_kernel)."""
         n = len(active)
@@ -366,6 +378,16 @@ class Ctx:
 
 def now_ns() -> int:
     return lib().bl_now_ns()
+
+
+def place(mem_bytes, avg_kernel_ns, gpu_free_bytes, span_x: int = 30):
+    """Tenant -> GPU placement (bl_place, L171, R33): list of GPU indices (-1 = none)."""
+    n, G = len(mem_bytes), len(gpu_free_bytes)
+    out = (C.c_int32 * max(1, n))()
+    check("bl_place", lib().bl_place(n, (C.c_int64 * max(1, n))(*[int(x) for x in mem_bytes]),
+                                     (C.c_int64 * max(1, n))(*[int(x) for x in avg_kernel_ns]), G,
+                                     (C.c_int64 * max(1, G))(*[int(x) for x in gpu_free_bytes]), int(span_x), out))
+    return [out[i] for i in range(n)]
 
 
 def dispatch(ctxs, entries, base_ns: int = 0):

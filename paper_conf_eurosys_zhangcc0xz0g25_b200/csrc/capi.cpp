@@ -220,6 +220,24 @@ bl_status bl_run_squad(bl_ctx* ctx, int n, const int32_t* ten, const int32_t* ke
   GUARD(ctx);
   return wrap([&](std::string& e) { return ctx->eng->run_squad(n, ten, ker, lo, hi, reps, makespan, kernel_ns, e); });
 }
+bl_status bl_deployment_check(bl_ctx* ctx, const int64_t* mem, int64_t free_b, int32_t span, int32_t* ok,
+                              int32_t* why) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->deployment_check(mem, free_b, span, ok, why, e); });
+}
+bl_status bl_place(int n, const int64_t* mem, const int64_t* avg, int G, const int64_t* gfree, int32_t span,
+                   int32_t* out) {
+  if (n < 0 || G < 1 || span < 1 || (n && (!mem || !avg || !out)) || !gfree) {
+    g_err = "bad placement args";
+    return BL_E_INVALID;
+  }
+  return wrap([&](std::string&) {
+    const std::vector<int> r = bless::place(std::vector<int64_t>(mem, mem + n), std::vector<int64_t>(avg, avg + n),
+                                            std::vector<int64_t>(gfree, gfree + G), span);
+    for (int i = 0; i < n; ++i) out[i] = r[i];
+    return BL_OK;
+  });
+}
 bl_status bl_reset(bl_ctx* ctx, const bl_params* p) {
   GUARD(ctx);
   return wrap([&](std::string& e) { return ctx->eng->reset(p, e); });

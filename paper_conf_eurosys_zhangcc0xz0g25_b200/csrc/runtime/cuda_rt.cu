@@ -619,6 +619,10 @@ int DeviceRT::event_query(void* e) {
 }
 bool DeviceRT::stream_sync(void* s) { return cudaStreamSynchronize((cudaStream_t)s) == cudaSuccess; }
 bool DeviceRT::device_sync() { return cudaDeviceSynchronize() == cudaSuccess; }
+int64_t DeviceRT::free_bytes() {
+  size_t fr = 0, tot = 0;
+  return cudaMemGetInfo(&fr, &tot) == cudaSuccess ? (int64_t)fr : -1;
+}
 
 bool DeviceRT::profile(int h, int sm_count, int reps, void* stream, int64_t* ns_out, int* d_out, std::string& err) {
   cudaStream_t s = (cudaStream_t)stream;

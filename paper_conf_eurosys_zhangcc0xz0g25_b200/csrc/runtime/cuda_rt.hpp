@@ -81,6 +81,7 @@ class DeviceRT {
   bool stream_sync(void* s);
   bool device_sync();
   bool set_device();
+  int64_t free_bytes();   // cudaMemGetInfo free, -1 on error
 
   // Offline profiler: median over 3 batches of the per-launch mean of 'reps'
   // back-to-back launches on [0, sm_count).  d_out (if non-null): distinct SMs

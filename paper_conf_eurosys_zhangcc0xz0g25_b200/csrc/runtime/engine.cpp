@@ -310,6 +310,19 @@ bl_status Engine::start(std::string& err) {
   if (nten() == 0) { err = "no tenants"; return BL_E_STATE; }
   if (!prof_.complete()) { err = "submit/start before a complete profile (PAPER.md L155: no profile, no BLESS)"; return BL_E_STATE; }
   prof_.g = prm_.sm_unit;
+  if (prm_.sm_limit) {
+    // f4 SM-count sweep (L420): the whole system runs on logical SMs
+    // [0, sm_limit) -- profile columns 1..sm_limit, d capped, N = sm_limit/g
+    if (prm_.sm_limit < prm_.sm_unit || prm_.sm_limit > prof_.S) { err = "sm_limit outside [g, S]"; return BL_E_INVALID; }
+    prof_full_ = prof_;
+    limited_ = true;
+    prof_.S = prm_.sm_limit;
+    for (auto& tn : prof_.ten)
+      for (auto& k : tn.k) {
+        k.t.resize(prof_.S);
+        k.d = std::min(k.d, prof_.S);
+      }
+  }
   prof_.derive();
   if (prof_.N < 1) { err = "sm_unit larger than S"; return BL_E_INVALID; }
   int lo = 0;
@@ -437,7 +450,36 @@ bl_status Engine::stop(std::string& err) {
     }
   }
   started_ = false;
+  if (limited_) {   // back to the whole-GPU profile
+    prof_ = prof_full_;
+    limited_ = false;
+  }
   if (failed_) { err = fail_msg_; return BL_E_CUDA; }
+  return BL_OK;
+}
+
+bl_status Engine::deployment_check(const int64_t* mem, int64_t free_b, int32_t span, int32_t* ok, int32_t* why,
+                                   std::string& err) {
+  if (!mem || !ok || span < 1) { err = "bad args"; return BL_E_INVALID; }
+  if (!prof_.complete()) { err = "profile incomplete"; return BL_E_STATE; }
+  if (free_b <= 0) {
+    if (!rt_) { err = "no device to query free memory"; return BL_E_STATE; }
+    rt_->set_device();
+    free_b = rt_->free_bytes();
+    if (free_b < 0) { err = "cudaMemGetInfo"; return BL_E_CUDA; }
+  }
+  prof_.derive();
+  std::vector<int64_t> avg;
+  int64_t need = 0;
+  for (int j = 0; j < nten(); ++j) {
+    avg.push_back(prof_.ten[j].T / std::max<int64_t>(1, (int64_t)prof_.ten[j].k.size()));
+    need += mem[j];
+  }
+  int r = 0;
+  if (!colocatable(avg, span)) r = 1;
+  else if (need > free_b) r = 2;
+  *ok = r == 0;
+  if (why) *why = r;
   return BL_OK;
 }
 

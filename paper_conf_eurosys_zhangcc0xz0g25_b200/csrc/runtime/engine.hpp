@@ -125,6 +125,8 @@ class Engine {
   bl_status time_decide(const bl_decision* recs, size_t n, int reps, int64_t* total_ns, int64_t* picks,
                         std::string& err);
   bool virtual_clock() const { return prm_.clock == BL_CLOCK_VIRTUAL; }
+  bl_status deployment_check(const int64_t* mem, int64_t free_b, int32_t span, int32_t* ok, int32_t* why,
+                             std::string& err);
   bl_status predict(int n, const int32_t* ten, const int32_t* ker, const int32_t* p, int64_t* out, std::string& err);
   bl_status run_squad(int n, const int32_t* ten, const int32_t* ker, const int16_t* lo, const int16_t* hi, int reps,
                       int64_t* makespan, int64_t* kernel_ns, std::string& err);
@@ -157,6 +159,8 @@ class Engine {
   bl_params prm_;
   std::unique_ptr<DeviceRT> rt_;
   Profile prof_;
+  Profile prof_full_;        // the whole-GPU profile while a run is restricted by sm_limit
+  bool limited_ = false;
   std::vector<TenantRT> ten_;
   double quota_sum_ = 0;
 

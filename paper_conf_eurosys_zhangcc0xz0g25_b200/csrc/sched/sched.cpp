@@ -369,4 +369,37 @@ int64_t predict_sp(const Profile& prof, const std::vector<int>& parts, const std
   return worst;
 }
 
+bool colocatable(const std::vector<int64_t>& avg, int64_t span_x) {
+  if (avg.empty()) return true;
+  const int64_t lo = *std::min_element(avg.begin(), avg.end());
+  const int64_t hi = *std::max_element(avg.begin(), avg.end());
+  return (__int128)hi <= (__int128)lo * span_x;   // exact: max <= span * min
+}
+
+std::vector<int> place(const std::vector<int64_t>& mem, const std::vector<int64_t>& avg,
+                       const std::vector<int64_t>& gpu_free, int64_t span_x) {
+  const int n = (int)mem.size(), G = (int)gpu_free.size();
+  std::vector<int> order(n), out(n, -1);
+  for (int i = 0; i < n; ++i) order[i] = i;
+  std::stable_sort(order.begin(), order.end(), [&](int a, int b) { return mem[a] > mem[b]; });
+  std::vector<int64_t> left = gpu_free;
+  std::vector<std::vector<int64_t>> on(G);
+  for (int a : order) {
+    int best = -1;
+    for (int gpu = 0; gpu < G; ++gpu) {
+      if (mem[a] > left[gpu]) continue;
+      std::vector<int64_t> v = on[gpu];
+      v.push_back(avg[a]);
+      if (!colocatable(v, span_x)) continue;
+      if (best < 0 || left[gpu] > left[best]) best = gpu;
+    }
+    if (best >= 0) {
+      out[a] = best;
+      left[best] -= mem[a];
+      on[best].push_back(avg[a]);
+    }
+  }
+  return out;
+}
+
 }  // namespace bless

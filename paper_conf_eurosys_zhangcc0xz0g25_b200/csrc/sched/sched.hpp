@@ -104,4 +104,11 @@ int64_t predict_nsp(const Profile& prof, const std::vector<int>& parts, const st
 int64_t predict_sp(const Profile& prof, const std::vector<int>& parts, const std::vector<std::vector<int>>& ks,
                    const std::vector<int>& p);
 
+// Deployment (§4.2.2; reading R33): co-location rule and
+// the central controller's tenant -> GPU placement.  avg[j] = average kernel
+// duration (ns); span_x = largest / smallest allowed (L163: 10-300 us -> 30).
+bool colocatable(const std::vector<int64_t>& avg, int64_t span_x);
+std::vector<int> place(const std::vector<int64_t>& mem, const std::vector<int64_t>& avg,
+                       const std::vector<int64_t>& gpu_free, int64_t span_x);
+
 }  // namespace bless
