@@ -49,6 +49,12 @@ struct TcParams {
   float* ws;        // [tiles][128][BN] fp32 partial sums (zero between launches)
   unsigned* sem;    // [tiles] arrival counters (zero between launches)
   int sk_tiles;     // output tiles (workspace layout)
+  // halo mode (3x3 stride-1 convs, HALO kernels): per 64-channel chunk ONE TMA
+  // box of the tile's input halo ((BH+2) x BW pixels) serves all nine taps --
+  // tap (r, s) is the same smem tile read from row r*BW + s on
+  int astages;      // halo stages in smem (1 or 2)
+  int a_stage_bytes;
+  int a_tx;         // bytes one halo box delivers
 };
 
 #ifdef __CUDACC__
@@ -159,6 +165,19 @@ __device__ __forceinline__ uint64_t smem_desc(uint32_t saddr) {
   d |= (uint64_t)1 << 46;                    // version
   d |= layout << 61;
   return d;
+}
+
+// Same descriptor for a K-major SW128 tile that starts `row` 128-byte rows
+// after a 1024-byte-aligned swizzle atom: the matrix base offset (bits 49-51)
+// is the start's row phase inside the 8-row swizzle pattern, (addr >> 7) & 7.
+// The halo conv reads each tap's A tile this way (start = halo + (r*BW + s)
+// rows).  BLESS_TC_HALO_BO=0 at build time drops the field (A/B probe).
+__device__ __forceinline__ uint64_t smem_desc_row(uint32_t saddr) {
+#if defined(BLESS_TC_HALO_BO) && BLESS_TC_HALO_BO == 0
+  return smem_desc<64>(saddr);
+#else
+  return smem_desc<64>(saddr) | ((uint64_t)((saddr >> 7) & 7) << 49);
+#endif
 }
 
 // Instruction descriptor kind::f16: A, B bf16, D f32, both K-major, M = 128.
@@ -328,26 +347,31 @@ struct TcCfg {
   static constexpr int kSmemMax = kMaxStages * kStageBytes + kFixed;
 };
 
-template <int BN, int BK>
+template <int BN, int BK, bool HALO>
 __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   using Cfg = TcCfg<BN, BK>;
-  const int ST = p.stages;
+  const int ST = p.stages;                           // B stages (A and B stages when !HALO)
+  const int NA = HALO ? p.astages : ST;              // A stages
+  const int a_bytes = HALO ? p.a_stage_bytes : Cfg::kStageA;
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   unsigned char* smem = (unsigned char*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   unsigned char* sA = smem;
-  unsigned char* sB = smem + ST * Cfg::kStageA;
-  uint64_t* bars = (uint64_t*)(smem + ST * Cfg::kStageBytes);
+  unsigned char* sB = smem + NA * a_bytes;
+  unsigned char* bar_base = sB + ST * Cfg::kStageB;
+  uint64_t* bars = (uint64_t*)bar_base;
   uint64_t* full = bars;            // [ST]
   uint64_t* empty = bars + ST;      // [ST]
   uint64_t* tfull = bars + 2 * ST;  // [2] accumulator ready
   uint64_t* tempty = tfull + 2;     // [2] accumulator drained
   uint64_t* rfull = tempty + 2;     // [2] tile ring
   uint64_t* rempty = rfull + 2;     // [2]
-  int* ring = (int*)(rempty + 2);   // [2]
+  uint64_t* fullA = rempty + 2;     // [2] halo stages (HALO)
+  uint64_t* emptyA = fullA + 2;     // [2]
+  int* ring = (int*)(emptyA + 2);   // [2]
   uint32_t* tmem_slot = (uint32_t*)(ring + 2);
   volatile int* last_flag = (volatile int*)(tmem_slot + 1);
-  float* epi_sc = (float*)(smem + ST * Cfg::kStageBytes + 256);  // [BN] tile scale
-  float* epi_sh = epi_sc + BN;                                    // [BN] tile shift
+  float* epi_sc = (float*)(bar_base + 256);  // [BN] tile scale
+  float* epi_sh = epi_sc + BN;               // [BN] tile shift
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) TR(1);   // 1: work entry
@@ -365,6 +389,8 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       mbar_init(&tempty[i], kEpiWarps);
       mbar_init(&rfull[i], 1);
       mbar_init(&rempty[i], 1 + kEpiWarps);
+      mbar_init(&fullA[i], 1);
+      mbar_init(&emptyA[i], 1);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -409,6 +435,8 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       bool dep_waited = false;
       int stage = 0;
       uint32_t phase = 0;
+      int astage = 0;
+      uint32_t aphase = 0;
       int rs = 0;
       uint32_t rph = 0;
       for (;;) {
@@ -467,6 +495,36 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
             }
           }
         };
+        if constexpr (HALO) {
+          // per 64-channel chunk: the input halo once, then the nine taps' weights
+          const int taps = p.R_ * p.S_;
+          auto load_Bt = [&](int c, int tap) {
+            mbar_wait(&empty[stage], phase ^ 1);
+            mbar_expect_tx(&full[stage], (uint32_t)Cfg::kStageB);
+            tma_load_2d(sB + stage * Cfg::kStageB, &p.tmB, &full[stage], tap * p.C + c * 64, tn * BN);
+            if (++stage == ST) { stage = 0; phase ^= 1; }
+          };
+          auto load_halo = [&](int c) {
+            mbar_wait(&emptyA[astage], aphase ^ 1);
+            mbar_expect_tx(&fullA[astage], (uint32_t)p.a_tx);
+            tma_load_4d(sA + astage * a_bytes, &p.tmA, &fullA[astage], c * 64, -p.pad, oh0 - p.pad, 0);
+            if (++astage == NA) { astage = 0; aphase ^= 1; }
+          };
+          for (int c = kb0; c < kb1; ++c) {
+            int tap0 = 0;
+            if (!dep_waited) {   // weights before the grid dependency resolves, activations after
+              tap0 = min(taps, ST);
+              for (int tap = 0; tap < tap0; ++tap) load_Bt(c, tap);
+              pdl_wait();
+              if (t == 0) gate_prev_end(g, (int64_t)ptx_globaltimer());
+              TR(4);
+              dep_waited = true;
+            }
+            load_halo(c);
+            for (int tap = tap0; tap < taps; ++tap) load_Bt(c, tap);
+          }
+          continue;
+        }
         int kb = kb0;
         if (!dep_waited) {
           // first tile: weights for up to ST stages before the grid dependency
@@ -502,6 +560,8 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
     const uint32_t idesc = instr_desc<BN>();
     int stage = 0;
     uint32_t phase = 0;
+    int astage = 0;
+    uint32_t aphase = 0;
     int rs = 0;
     uint32_t rph = 0;
     int acc = 0;
@@ -518,7 +578,34 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       mbar_wait(&tempty[acc], aph ^ 1);
       tc_fence_after();
       const uint32_t d_tmem = tmem_base + acc * BN;
-      for (int kb = kb0; kb < kb1; ++kb) {
+      if constexpr (HALO) {
+        const int taps = p.R_ * p.S_;
+        for (int c = kb0; c < kb1; ++c) {
+          mbar_wait(&fullA[astage], aphase);
+          tc_fence_after();
+          const uint32_t a_base = smem_u32(sA + astage * a_bytes);
+          for (int tap = 0; tap < taps; ++tap) {
+            mbar_wait(&full[stage], phase);
+            tc_fence_after();
+            if (lane == 0) {
+              const int r = tap / p.S_, s_ = tap - r * p.S_;
+              const uint32_t a0 = a_base + (uint32_t)(r * p.BW + s_) * 128u;
+              const uint32_t b0 = smem_u32(sB + stage * Cfg::kStageB);
+#pragma unroll
+              for (int k = 0; k < 4; ++k)
+                tc_mma(d_tmem, smem_desc_row(a0 + k * 32), smem_desc<64>(b0 + k * 32), idesc,
+                       (c != kb0 || tap || k) ? 1u : 0u);
+              tc_commit(&empty[stage]);
+            }
+            __syncwarp();
+            if (++stage == ST) { stage = 0; phase ^= 1; }
+          }
+          if (lane == 0) tc_commit(&emptyA[astage]);
+          __syncwarp();
+          if (++astage == NA) { astage = 0; aphase ^= 1; }
+        }
+      }
+      for (int kb = HALO ? kb1 : kb0; kb < kb1; ++kb) {
         mbar_wait(&full[stage], phase);
         tc_fence_after();
         if (lane == 0 && kb == kb0) TR(5);   // 5: first stage landed (last tile of this CTA)
@@ -666,10 +753,10 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   __syncthreads();
 }
 
-template <int BN, int BK>
+template <int BN, int BK, bool HALO>
 __global__ void __launch_bounds__(kTcThreads, 2) k_tc_gemm(const __grid_constant__ TcParams p, const GateArgs g) {
   if (threadIdx.x == 0) TR(0);   // 0: CTA start
-  if (gate_in_range(g) || gate_linger(g)) tc_work<BN, BK>(p, g);
+  if (gate_in_range(g) || gate_linger(g)) tc_work<BN, BK, HALO>(p, g);
   pdl_trigger();
   if (threadIdx.x == 0) TR(8);   // 8: work done, before the exit atomic
   if (!g.stamp) {                // light exit
@@ -678,26 +765,38 @@ __global__ void __launch_bounds__(kTcThreads, 2) k_tc_gemm(const __grid_constant
   }
   int last = 0;
   const bool fb = gate_leave(g, last);
-  if (fb) tc_work<BN, BK>(p, g);
+  if (fb) tc_work<BN, BK, HALO>(p, g);
   if (last) gate_finalize(g, fb);
   if (threadIdx.x == 0) TR(9);   // 9: CTA exit
 }
 #endif  // __CUDACC__
 
 // ------------------------------------------------------------------ host side
-template <int BN, int BK>
+template <int BN, int BK, bool HALO>
 static cudaError_t launch_tc(const KernelDesc& d, const GateArgs& g, cudaStream_t st) {
   void* args[2] = {(void*)d.params, (void*)&g};
-  return launch_kernel((const void*)k_tc_gemm<BN, BK>, dim3(launch_grid(d, g)), dim3(d.block), (size_t)d.smem, st, args);
+  return launch_kernel((const void*)k_tc_gemm<BN, BK, HALO>, dim3(launch_grid(d, g)), dim3(d.block), (size_t)d.smem,
+                       st, args);
 }
 
-template <int BN, int BK>
+// Halo stages: NA halo stages + ST weight stages within ~100 KB (two CTAs
+// per SM, as the other tiles): two halo stages when three weight stages still
+// fit beside them, else one.
+template <int BN>
+static void halo_stages(TcParams& p, int& na, int& nb) {
+  using Cfg = TcCfg<BN, 64>;
+  const int budget = 100 * 1024 - Cfg::kFixed;
+  na = (2 * p.a_stage_bytes + 3 * Cfg::kStageB <= budget) ? 2 : 1;
+  nb = std::max(2, std::min(kMaxStages, (budget - na * p.a_stage_bytes) / Cfg::kStageB));
+}
+
+template <int BN, int BK, bool HALO>
 static bool prep(KernelDesc& d, TcParams& p, std::string& err) {
   static std::once_flag once;
   static cudaError_t attr_err = cudaSuccess;
   std::call_once(once, [] {
-    attr_err = cudaFuncSetAttribute((const void*)k_tc_gemm<BN, BK>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    std::min(TcCfg<BN, BK>::kSmemMax, kDynSmemMax));
+    attr_err = cudaFuncSetAttribute((const void*)k_tc_gemm<BN, BK, HALO>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    HALO ? kDynSmemMax : std::min(TcCfg<BN, BK>::kSmemMax, kDynSmemMax));
   });
   if (attr_err != cudaSuccess) {
     err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(attr_err);
@@ -713,8 +812,15 @@ static bool prep(KernelDesc& d, TcParams& p, std::string& err) {
   }
   p.stages = st;
   d.smem = st * Cfg::kStageBytes + Cfg::kFixed;
-  d.launch = launch_tc<BN, BK>;
-  d.kernel_fn = (const void*)k_tc_gemm<BN, BK>;
+  if (HALO) {
+    int na = 1, nb = 2;
+    halo_stages<BN>(p, na, nb);
+    p.astages = na;
+    p.stages = nb;
+    d.smem = na * p.a_stage_bytes + nb * Cfg::kStageB + Cfg::kFixed;
+  }
+  d.launch = launch_tc<BN, BK, HALO>;
+  d.kernel_fn = (const void*)k_tc_gemm<BN, BK, HALO>;
   return true;
 }
 
@@ -871,6 +977,31 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     }
     if (p.mode != 0) p.tiles_n = 0;  // set below
     (void)tiles_h;
+    // halo mode: 3x3 "same" stride-1 conv, C % 64 == 0, and a tile row wide
+    // enough that every valid output column's taps stay inside its halo row
+    // (OW + 2 <= BW): one (64, BW, BH + 2) box per channel chunk serves all
+    // nine taps (autotuner candidate, or BLESS_TC_HALO=1 as the default)
+    const char* he = std::getenv("BLESS_TC_HALO");
+    const int halo_env = he ? std::atoi(he) : 0;
+    const bool want_halo = force ? force->halo != 0 : halo_env != 0;
+    if (want_halo && stride == 1 && R == 3 && S == 3 && pad == 1 && C % 64 == 0 && p.OW + 2 <= 128) {
+      int hw = 8;
+      while (hw < p.OW + 2) hw <<= 1;
+      p.mode = 3;
+      BK = 64;
+      p.BW = hw;
+      p.BH = 128 / hw;
+      p.tiles_w = 1;
+      p.kc_per_tap = C / 64;
+      p.num_kb = C / 64;            // K blocks = channel chunks (nine taps each)
+      const int rows = (p.BH + 2) * p.BW + 8;   // + the s-shift overrun rows (only invalid outputs read them)
+      p.a_stage_bytes = (rows * 128 + 1023) / 1024 * 1024;
+      p.a_tx = 64 * 2 * p.BW * (p.BH + 2);
+      cuuint64_t da[4] = {(cuuint64_t)C, (cuuint64_t)Wd, (cuuint64_t)H, 1};
+      cuuint64_t sa[3] = {(cuuint64_t)ldx * 2, (cuuint64_t)Wd * ldx * 2, (cuuint64_t)H * Wd * ldx * 2};
+      cuuint32_t ba[4] = {64, (cuuint32_t)p.BW, (cuuint32_t)(p.BH + 2), 1};
+      if (!encode(&p.tmA, 4, X, da, sa, ba, 64, err)) return false;
+    }
   } else {
     return false;
   }
@@ -887,7 +1018,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   int splits = 1;
   if (ntiles(BN) < caps.S) {
     const int want = (int)((caps.S + ntiles(BN) - 1) / ntiles(BN));
-    splits = std::max(1, std::min(want, p.num_kb / 3));
+    splits = std::max(1, std::min(want, p.mode == 3 ? p.num_kb : p.num_kb / 3));
   }
   if (force && force->bn) {
     fbn = force->bn;
@@ -945,14 +1076,18 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   if (const char* e = std::getenv("BLESS_TC_MAX_OCC")) d.max_occ = std::max(1, std::atoi(e));   // sweeps
   bool ok = false;
 #define TC_CASE(bn, bk) \
-  if (BN == bn && BK == bk) ok = prep<bn, bk>(d, p, err);
+  if (BN == bn && BK == bk && p.mode != 3) ok = prep<bn, bk, false>(d, p, err);
+#define TC_HALO(bn) \
+  if (BN == bn && p.mode == 3) ok = prep<bn, 64, true>(d, p, err);
   TC_CASE(16, 16) TC_CASE(16, 32) TC_CASE(16, 64)
   TC_CASE(32, 16) TC_CASE(32, 32) TC_CASE(32, 64)
   TC_CASE(64, 16) TC_CASE(64, 32) TC_CASE(64, 64)
   TC_CASE(128, 16) TC_CASE(128, 32) TC_CASE(128, 64)
   TC_CASE(256, 16) TC_CASE(256, 32) TC_CASE(256, 64)
   TC_CASE(16, 128) TC_CASE(32, 128) TC_CASE(64, 128)
+  TC_HALO(16) TC_HALO(32) TC_HALO(64) TC_HALO(128)
 #undef TC_CASE
+#undef TC_HALO
   if (!ok) {
     if (err.empty()) err = "no tc instantiation";
     return false;
@@ -962,7 +1097,9 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   d.choice_bn = BN;
   d.choice_splits = p.splits;
   d.choice_bk = BK;
+  d.choice_halo = p.mode == 3 ? 1 : 0;
   d.family = op.kind == BL_OP_GEMM ? "tc_gemm_bf16" : (p.mode == 0 ? "tc_conv1x1_bf16" : "tc_conv_bf16");
+  if (BK == 128 && BN > 64 && p.mode == 3) { err = "halo BN"; return false; }
   d.flops = 2.0 * p.M * p.N * p.K;
   double a_bytes = (op.kind == BL_OP_CONV) ? 2.0 * op.dims[1] * op.dims[2] * op.dims[3] : 2.0 * p.M * p.K;
   d.bytes = a_bytes + 2.0 * p.N * p.K + 2.0 * p.M * p.N * (p.R ? 2 : 1);
@@ -980,8 +1117,8 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
 // reduction costs several us), BK = 128 wins the 3x3 convs, BN = 128 with
 // BK = 64 wins large GEMMs; BN = 256 never won with 96 KB of stages.
 int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int max) {
-  long long M, N, num_kb, tiles_m;
-  bool bk128_ok = false;
+  long long M, N, num_kb, tiles_m, halo_tiles_m = 0, chunks = 0;
+  bool bk128_ok = false, halo_ok = false;
   if (op.kind == BL_OP_GEMM) {
     M = op.dims[0], N = op.dims[1];
     num_kb = (op.dims[2] + 63) / 64;
@@ -998,11 +1135,27 @@ int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int ma
     while (BW < OW && BW < 128) BW <<= 1;
     tiles_m = ((OW + BW - 1) / BW) * ((OH + (128 / BW) - 1) / (128 / BW));
     bk128_ok = st == 1 && (one ? C % 64 == 0 : C % 128 == 0);
+    halo_ok = st == 1 && R == 3 && S == 3 && pad == 1 && C % 64 == 0 && OW + 2 <= 128;
+    long long hw = 8;
+    while (hw < OW + 2) hw <<= 1;
+    halo_tiles_m = (OH + (128 / hw) - 1) / (128 / hw);
+    chunks = C / 64;
   } else {
     return 0;
   }
   int n = 0;
   const int nmax = N <= 16 ? 16 : (N <= 32 ? 32 : (N <= 64 ? 64 : 128));
+  if (halo_ok) {
+    // halo tiles: BH x BW with BW >= OW + 2; K blocks = 64-channel chunks
+    for (int bn = std::min(32, nmax); bn <= nmax && n < max; bn <<= 1) {
+      const long long tiles = halo_tiles_m * ((N + bn - 1) / bn);
+      out[n++] = TcChoice{bn, 1, 64, 1};
+      if (tiles < caps.S && chunks >= 2 && n < max) {
+        const long long want = std::min<long long>((caps.S + tiles - 1) / tiles, chunks);
+        if (want >= 2) out[n++] = TcChoice{bn, (int)want, 64, 1};
+      }
+    }
+  }
   for (int bn = std::min(32, nmax); bn <= nmax; bn <<= 1) {
     for (int bk = 64; bk <= 128; bk += 64) {
       if (bk == 128 && (!bk128_ok || bn > 64)) continue;

@@ -147,8 +147,9 @@ std::unique_ptr<DeviceRT> DeviceRT::create(int device, void* ws, size_t ws_bytes
     rt->tune_file_ = e;
     if (FILE* f = std::fopen(e, "r")) {
       char sig[512];
-      int bn = 0, sp = 0, bk = 0;
-      while (std::fscanf(f, "%511s %d %d %d", sig, &bn, &sp, &bk) == 4) rt->tune_cache_[sig] = TcChoice{bn, sp, bk};
+      int bn = 0, sp = 0, bk = 0, halo = 0;
+      while (std::fscanf(f, "%511s %d %d %d %d", sig, &bn, &sp, &bk, &halo) == 5)
+        rt->tune_cache_[sig] = TcChoice{bn, sp, bk, halo};
       std::fclose(f);
     }
   }
@@ -269,7 +270,7 @@ int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
     auto it = tune_cache_.find(sig);
     if (it != tune_cache_.end()) {
       if (it->second.bn != kd->choice_bn || it->second.splits != kd->choice_splits ||
-          it->second.bk != kd->choice_bk) {
+          it->second.bk != kd->choice_bk || it->second.halo != kd->choice_halo) {
         std::unique_ptr<KernelDesc> k2(new KernelDesc());
         std::string e2;
         if (build_tc_gemm(op, caps_, *k2, e2, &it->second)) {
@@ -282,10 +283,11 @@ int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
       }
     } else {
       if (!autotune_tc(op, kd, err)) return -1;
-      tune_cache_[sig] = TcChoice{kd->choice_bn, kd->choice_splits, kd->choice_bk};
+      tune_cache_[sig] = TcChoice{kd->choice_bn, kd->choice_splits, kd->choice_bk, kd->choice_halo};
       if (!tune_file_.empty()) {
         if (FILE* f = std::fopen(tune_file_.c_str(), "a")) {
-          std::fprintf(f, "%s %d %d %d\n", sig.c_str(), kd->choice_bn, kd->choice_splits, kd->choice_bk);
+          std::fprintf(f, "%s %d %d %d %d\n", sig.c_str(), kd->choice_bn, kd->choice_splits, kd->choice_bk,
+                       kd->choice_halo);
           std::fclose(f);
         }
       }
@@ -298,7 +300,7 @@ int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
 // Shape signature of a tc op for the tuning cache (pointers excluded).
 std::string DeviceRT::tc_signature(const bl_op& op) const {
   // "v2": tune files since the autotuner also picks BK (older lines never match)
-  std::string s = "v2k" + std::to_string(op.kind) + "_t" + std::to_string(op.dtype) + "_r" + (op.ptr[4] ? "1" : "0");
+  std::string s = "v3k" + std::to_string(op.kind) + "_t" + std::to_string(op.dtype) + "_r" + (op.ptr[4] ? "1" : "0");
   for (int i = 0; i < 12; ++i) s += "_" + std::to_string(op.dims[i]);
   return s;
 }
@@ -309,8 +311,8 @@ std::string DeviceRT::tc_signature(const bl_op& op) const {
 // events, all S SMs) on the layer's own buffers; the fastest wins, and within
 // 3 % of it the one with fewer tiles (smaller d leaves more SMs to co-runners).
 bool DeviceRT::autotune_tc(const bl_op& op, std::unique_ptr<KernelDesc>& best, std::string& err) {
-  TcChoice cand[16];
-  const int nc = tc_candidates(op, caps_, cand, 16);
+  TcChoice cand[24];
+  const int nc = tc_candidates(op, caps_, cand, 24);
   if (nc <= 1) return true;
   if (!tune_stream_ && cudaStreamCreateWithFlags((cudaStream_t*)&tune_stream_, cudaStreamNonBlocking) != cudaSuccess) {
     err = "autotune stream";
@@ -326,13 +328,14 @@ bool DeviceRT::autotune_tc(const bl_op& op, std::unique_ptr<KernelDesc>& best, s
     if (!ok) return false;
   }
   for (int i = 0; i < nc; ++i) {
-    if (cand[i].bn == best->choice_bn && cand[i].splits == best->choice_splits && cand[i].bk == best->choice_bk)
+    if (cand[i].bn == best->choice_bn && cand[i].splits == best->choice_splits && cand[i].bk == best->choice_bk &&
+        cand[i].halo == best->choice_halo)
       continue;
     std::unique_ptr<KernelDesc> kd(new KernelDesc());
     std::string e2;
     if (!build_tc_gemm(op, caps_, *kd, e2, &cand[i])) continue;
     if (kd->choice_bn == best->choice_bn && kd->choice_splits == best->choice_splits &&
-        kd->choice_bk == best->choice_bk) {
+        kd->choice_bk == best->choice_bk && kd->choice_halo == best->choice_halo) {
       if (kd->owned) cudaFree(kd->owned);
       continue;
     }

@@ -139,6 +139,28 @@ def test_tc_forced_configs(ctx, cfg, shape, monkeypatch):
     run_and_check(ctx, m, "bf16")
 
 
+@pytest.mark.parametrize("cfg", ["32,64,1", "64,64,1", "128,64,1", "64,64,3", "32,64,4"])
+@pytest.mark.parametrize("dims", [(56, 56, 64, 256), (28, 28, 128, 256), (14, 14, 256, 256), (7, 7, 512, 512),
+                                  (20, 27, 256, 96), (112, 112, 64, 128), (13, 11, 64, 48)])
+def test_tc_halo_conv(ctx, cfg, dims, monkeypatch):
+    """Halo implicit-GEMM 3x3 conv (mode 3): one TMA box of the tile's
+    (BH + 2) x BW input halo per 64-channel chunk, each tap's A operand read
+    from it at row offset r*BW + s (UMMA descriptor with the swizzle base
+    offset).  Exact vs the oracle for square, ragged and 112-wide maps, every
+    BN, split-K over channel chunks, with residual + ReLU epilogue."""
+    monkeypatch.setenv("BLESS_TC_HALO", "1")
+    monkeypatch.setenv("BLESS_TC_CFG", cfg)
+    H, W, C, K = dims
+
+    def mk(b):
+        x = b.input((1, H, W, C))
+        r = b.param(np.random.default_rng(2).standard_normal((1, H, W, K)).astype(np.float32))
+        b.conv(x, K, 3, 1, 1, act="relu", bn=True, res=r)
+    m = one_layer(ctx, "bf16", mk)
+    assert ctx.kernel_info(m.tenant, 0).family.decode() == "tc_conv_bf16"
+    run_and_check(ctx, m, "bf16")
+
+
 @pytest.mark.parametrize("H,W,C,k,s,p,mode", [(112, 112, 64, 3, 2, 1, "max"), (224, 224, 64, 2, 2, 0, "max"),
                                               (9, 8, 5, 3, 2, 1, "avg"), (7, 7, 2048, 0, 1, 0, "gap")])
 @pytest.mark.parametrize("dtype", ["bf16", "fp32"])
