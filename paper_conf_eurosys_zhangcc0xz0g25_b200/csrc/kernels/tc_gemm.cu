@@ -168,15 +168,17 @@ __device__ __forceinline__ uint64_t smem_desc(uint32_t saddr) {
 }
 
 // Same descriptor for a K-major SW128 tile that starts `row` 128-byte rows
-// after a 1024-byte-aligned swizzle atom: the matrix base offset (bits 49-51)
-// is the start's row phase inside the 8-row swizzle pattern, (addr >> 7) & 7.
-// The halo conv reads each tap's A tile this way (start = halo + (r*BW + s)
-// rows).  BLESS_TC_HALO_BO=0 at build time drops the field (A/B probe).
+// after a 1024-byte-aligned swizzle atom (the halo conv reads each tap's A
+// tile at halo + (r*BW + s) rows).  Measured on B200 (profiles/round2/halo/):
+// the hardware applies the 128-byte swizzle to the absolute shared-memory
+// address bits, so a row-shifted start needs NO matrix base offset -- with
+// base offset = (addr >> 7) & 7 the result is wrong, with 0 it is exact.
+// -DBLESS_TC_HALO_BO=1 builds the other variant (probe only).
 __device__ __forceinline__ uint64_t smem_desc_row(uint32_t saddr) {
-#if defined(BLESS_TC_HALO_BO) && BLESS_TC_HALO_BO == 0
-  return smem_desc<64>(saddr);
-#else
+#if defined(BLESS_TC_HALO_BO) && BLESS_TC_HALO_BO == 1
   return smem_desc<64>(saddr) | ((uint64_t)((saddr >> 7) & 7) << 49);
+#else
+  return smem_desc<64>(saddr);
 #endif
 }
 
