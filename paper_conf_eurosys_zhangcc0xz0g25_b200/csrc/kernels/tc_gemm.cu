@@ -55,6 +55,11 @@ struct TcParams {
   int astages;      // halo stages in smem (1 or 2)
   int a_stage_bytes;
   int a_tx;         // bytes one halo box delivers
+  // weights in halo mode: one TMA box per filter row (the S taps of row r,
+  // 3-D view (C, N, R*S) of the KRSC weights), so a 64-channel chunk costs
+  // 1 + R boxes instead of 2 per tap (B200: a TMA box costs >= 130-180 ns per
+  // SM whatever its size, profiles/round2/halo/tma_bench.txt)
+  int b_stage_bytes;
 };
 
 #ifdef __CUDACC__
@@ -357,9 +362,10 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   const int a_bytes = HALO ? p.a_stage_bytes : Cfg::kStageA;
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   unsigned char* smem = (unsigned char*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  const int b_bytes = HALO ? p.b_stage_bytes : Cfg::kStageB;
   unsigned char* sA = smem;
   unsigned char* sB = smem + NA * a_bytes;
-  unsigned char* bar_base = sB + ST * Cfg::kStageB;
+  unsigned char* bar_base = sB + ST * b_bytes;
   uint64_t* bars = (uint64_t*)bar_base;
   uint64_t* full = bars;            // [ST]
   uint64_t* empty = bars + ST;      // [ST]
@@ -498,12 +504,12 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           }
         };
         if constexpr (HALO) {
-          // per 64-channel chunk: the input halo once, then the nine taps' weights
-          const int taps = p.R_ * p.S_;
-          auto load_Bt = [&](int c, int tap) {
+          // per 64-channel chunk: the input halo once, then one weight box per filter row
+          const int taps = p.R_;
+          auto load_Bt = [&](int c, int r) {
             mbar_wait(&empty[stage], phase ^ 1);
-            mbar_expect_tx(&full[stage], (uint32_t)Cfg::kStageB);
-            tma_load_2d(sB + stage * Cfg::kStageB, &p.tmB, &full[stage], tap * p.C + c * 64, tn * BN);
+            mbar_expect_tx(&full[stage], (uint32_t)b_bytes);
+            tma_load_3d(sB + stage * b_bytes, &p.tmB, &full[stage], c * 64, tn * BN, r * p.S_);
             if (++stage == ST) { stage = 0; phase ^= 1; }
           };
           auto load_halo = [&](int c) {
@@ -581,22 +587,23 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       tc_fence_after();
       const uint32_t d_tmem = tmem_base + acc * BN;
       if constexpr (HALO) {
-        const int taps = p.R_ * p.S_;
         for (int c = kb0; c < kb1; ++c) {
           mbar_wait(&fullA[astage], aphase);
           tc_fence_after();
           const uint32_t a_base = smem_u32(sA + astage * a_bytes);
-          for (int tap = 0; tap < taps; ++tap) {
+          for (int r = 0; r < p.R_; ++r) {   // one weight stage = filter row r (S taps)
             mbar_wait(&full[stage], phase);
             tc_fence_after();
             if (lane == 0) {
-              const int r = tap / p.S_, s_ = tap - r * p.S_;
-              const uint32_t a0 = a_base + (uint32_t)(r * p.BW + s_) * 128u;
-              const uint32_t b0 = smem_u32(sB + stage * Cfg::kStageB);
+              const uint32_t b_row = smem_u32(sB + stage * b_bytes);
+              for (int s_ = 0; s_ < p.S_; ++s_) {
+                const uint32_t a0 = a_base + (uint32_t)(r * p.BW + s_) * 128u;
+                const uint32_t b0 = b_row + (uint32_t)s_ * (BN * 128u);
 #pragma unroll
-              for (int k = 0; k < 4; ++k)
-                tc_mma(d_tmem, smem_desc_row(a0 + k * 32), smem_desc<64>(b0 + k * 32), idesc,
-                       (c != kb0 || tap || k) ? 1u : 0u);
+                for (int k = 0; k < 4; ++k)
+                  tc_mma(d_tmem, smem_desc_row(a0 + k * 32), smem_desc<64>(b0 + k * 32), idesc,
+                         (c != kb0 || r || s_ || k) ? 1u : 0u);
+              }
               tc_commit(&empty[stage]);
             }
             __syncwarp();
@@ -781,15 +788,17 @@ static cudaError_t launch_tc(const KernelDesc& d, const GateArgs& g, cudaStream_
                        st, args);
 }
 
-// Halo stages: NA halo stages + ST weight stages within ~100 KB (two CTAs
-// per SM, as the other tiles): two halo stages when three weight stages still
-// fit beside them, else one.
+// Halo stages: NA halo stages + NB weight stages (one filter row each) within
+// ~113 KB, so that two halo convs (or a halo conv and any other tile) still
+// share an SM's 228 KB: two halo stages when two weight stages fit beside
+// them, else one halo stage.  Returns false if not even 1 + 2 fit.
 template <int BN>
-static void halo_stages(TcParams& p, int& na, int& nb) {
+static bool halo_stages(const TcParams& p, int& na, int& nb) {
   using Cfg = TcCfg<BN, 64>;
-  const int budget = 100 * 1024 - Cfg::kFixed;
-  na = (2 * p.a_stage_bytes + 3 * Cfg::kStageB <= budget) ? 2 : 1;
-  nb = std::max(2, std::min(kMaxStages, (budget - na * p.a_stage_bytes) / Cfg::kStageB));
+  const int budget = 113 * 1024 - Cfg::kFixed;
+  na = (2 * p.a_stage_bytes + 2 * p.b_stage_bytes <= budget) ? 2 : 1;
+  nb = std::min(4, (budget - na * p.a_stage_bytes) / p.b_stage_bytes);
+  return nb >= 2;
 }
 
 template <int BN, int BK, bool HALO>
@@ -816,10 +825,13 @@ static bool prep(KernelDesc& d, TcParams& p, std::string& err) {
   d.smem = st * Cfg::kStageBytes + Cfg::kFixed;
   if (HALO) {
     int na = 1, nb = 2;
-    halo_stages<BN>(p, na, nb);
+    if (!halo_stages<BN>(p, na, nb)) {
+      err = "halo stages do not fit";
+      return false;
+    }
     p.astages = na;
     p.stages = nb;
-    d.smem = na * p.a_stage_bytes + nb * Cfg::kStageB + Cfg::kFixed;
+    d.smem = na * p.a_stage_bytes + nb * p.b_stage_bytes + Cfg::kFixed;
   }
   d.launch = launch_tc<BN, BK, HALO>;
   d.kernel_fn = (const void*)k_tc_gemm<BN, BK, HALO>;
@@ -1057,7 +1069,13 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     p.sem = (unsigned*)((char*)buf + wsb);
     d.owned = buf;
   }
-  if (BK == 128) {
+  if (p.mode == 3) {
+    p.b_stage_bytes = p.S_ * BN * 128;
+    cuuint64_t db[3] = {(cuuint64_t)p.C, (cuuint64_t)p.N, (cuuint64_t)(p.R_ * p.S_)};
+    cuuint64_t sb[2] = {(cuuint64_t)p.K * 2, (cuuint64_t)p.C * 2};
+    cuuint32_t bb[3] = {64, (cuuint32_t)BN, (cuuint32_t)p.S_};
+    if (!encode(&p.tmB, 3, W, db, sb, bb, 64, err)) return false;
+  } else if (BK == 128) {
     if (p.K % 64) { err = "BK 128 needs K % 64 == 0"; return false; }
     cuuint64_t db[3] = {64, (cuuint64_t)p.N, (cuuint64_t)(p.K / 64)}, sb[2] = {(cuuint64_t)p.K * 2, 128};
     cuuint32_t bb[3] = {64, (cuuint32_t)BN, 2};

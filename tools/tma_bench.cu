@@ -1,0 +1,166 @@
+// tma_bench.cu -- per-SM TMA load throughput on B200 for the box shapes the
+// tcgen05 GEMM/conv kernels use (cost model of the operand feed).
+//
+// One CTA per SM, one thread issues TMA loads of a given box into a ring of
+// ST shared-memory stages (no consumer work: a stage is re-armed as soon as its
+// previous load has landed), N boxes per CTA, coordinates walking over an
+// L2-resident tensor.  Reports ns per box and bytes per SM clock.
+//
+//   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o tma_bench tools/tma_bench.cu -lcuda && ./tma_bench
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdio>
+#include <vector>
+
+struct __align__(64) Maps {
+  CUtensorMap m;
+};
+
+__device__ __forceinline__ uint32_t su32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+template <int RANK>
+__global__ void k_tma(const __grid_constant__ Maps mp, int ST, int nbox, int box_bytes, int d1, int d2, int d3,
+                      int m1, int m2, int m3, unsigned long long* out) {
+  extern __shared__ __align__(1024) unsigned char sm_raw[];
+  unsigned char* sm = (unsigned char*)(((uintptr_t)sm_raw + 1023) & ~(uintptr_t)1023);
+  __shared__ uint64_t bar[16];
+  if (threadIdx.x != 0) return;
+  for (int i = 0; i < ST; ++i) asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&bar[i])));
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  asm volatile("prefetch.tensormap [%0];" ::"l"(&mp.m) : "memory");
+  unsigned long long t0;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  uint32_t ph[16] = {0};
+  for (int i = 0; i < nbox; ++i) {
+    const int s = i % ST;
+    if (i >= ST) {
+      asm volatile(
+          "{\n\t.reg .pred p;\n\tW_%=:\n\t"
+          "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t@!p bra W_%=;\n\t}" ::"r"(su32(&bar[s])),
+          "r"(ph[s])
+          : "memory");
+      ph[s] ^= 1;
+    }
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(su32(&bar[s])), "r"(box_bytes)
+                 : "memory");
+    const int c1 = ((blockIdx.x * 7 + i) % d1) * m1, c2 = ((blockIdx.x * 3 + i / d1) % d2) * m2,
+              c3 = ((i / (d1 * d2)) % d3) * m3;
+    void* dst = sm + (size_t)s * box_bytes;
+    if (RANK == 2)
+      asm volatile(
+          "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];"
+          ::"r"(su32(dst)), "l"(&mp.m), "r"(su32(&bar[s])), "r"(0), "r"(c1) : "memory");
+    else if (RANK == 3)
+      asm volatile(
+          "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5}], "
+          "[%2];" ::"r"(su32(dst)), "l"(&mp.m), "r"(su32(&bar[s])), "r"(0), "r"(c1), "r"(c2) : "memory");
+    else
+      asm volatile(
+          "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6}], "
+          "[%2];" ::"r"(su32(dst)), "l"(&mp.m), "r"(su32(&bar[s])), "r"(0), "r"(c1 - 1), "r"(c2 - 1), "r"(c3)
+          : "memory");
+  }
+  for (int i = nbox; i < nbox + ST; ++i) {
+    const int s = i % ST;
+    if (i >= ST) {
+      asm volatile(
+          "{\n\t.reg .pred p;\n\tW_%=:\n\t"
+          "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t@!p bra W_%=;\n\t}" ::"r"(su32(&bar[s])),
+          "r"(ph[s])
+          : "memory");
+      ph[s] ^= 1;
+    }
+  }
+  unsigned long long t1;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
+  out[blockIdx.x] = t1 - t0;
+}
+
+typedef CUresult (*Enc)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*, const cuuint64_t*,
+                        const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                        CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+int main() {
+  void* fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q);
+  Enc enc = (Enc)fn;
+  int S = 0;
+  cudaDeviceGetAttribute(&S, cudaDevAttrMultiProcessorCount, 0);
+  int clk_khz = 0;
+  cudaDeviceGetAttribute(&clk_khz, cudaDevAttrClockRate, 0);
+  // NHWC 56 x 64 x 512 bf16 (3.7 MB) and a [8192, 512] matrix: L2 resident
+  const int H = 56, W = 64, C = 512;
+  void* X = nullptr;
+  cudaMalloc(&X, (size_t)64 << 20);
+  cudaMemset(X, 0, (size_t)64 << 20);
+  unsigned long long* d_out;
+  cudaMalloc(&d_out, S * sizeof(unsigned long long));
+  std::vector<unsigned long long> h(S);
+  struct Case {
+    const char* name;
+    int rank;
+    cuuint64_t dims[4];
+    cuuint64_t strides[3];
+    cuuint32_t box[4];
+    int d1, d2, d3;
+  };
+  std::vector<Case> cases = {
+      {"2D (64ch, 64 rows) 8KB", 2, {64, 8192}, {(cuuint64_t)C * 2}, {64, 64}, 8192 / 64, 1, 1},
+      {"2D (64ch, 128 rows) 16KB", 2, {64, 8192}, {(cuuint64_t)C * 2}, {64, 128}, 8192 / 128, 1, 1},
+      {"2D (64ch, 256 rows) 32KB", 2, {64, 8192}, {(cuuint64_t)C * 2}, {64, 256}, 8192 / 256, 1, 1},
+      {"3D (64, 128 rows, 2 slabs) 32KB", 3, {64, 8192, 8}, {(cuuint64_t)C * 2, 128}, {64, 128, 2}, 8192 / 128, 4, 1},
+      {"3D (64, 64 rows, 2 slabs) 16KB", 3, {64, 8192, 8}, {(cuuint64_t)C * 2, 128}, {64, 64, 2}, 8192 / 64, 4, 1},
+      {"4D conv (64ch, 64w, 2h, 1) 16KB", 4, {64, (cuuint64_t)W, (cuuint64_t)H, 8},
+       {(cuuint64_t)C * 2, (cuuint64_t)W * C * 2, 128}, {64, 64, 2, 1}, 1, H / 2, 8},
+      {"4D conv (64ch, 64w, 2h, 2 slabs) 32KB", 4, {64, (cuuint64_t)W, (cuuint64_t)H, 8},
+       {(cuuint64_t)C * 2, (cuuint64_t)W * C * 2, 128}, {64, 64, 2, 2}, 1, H / 2, 4},
+      {"4D halo (64ch, 64w, 4h, 1) 32KB", 4, {64, (cuuint64_t)W, (cuuint64_t)H, 8},
+       {(cuuint64_t)C * 2, (cuuint64_t)W * C * 2, 128}, {64, 64, 4, 1}, 1, H / 4, 8},
+      {"4D conv (16ch, 64w, 2h, 1) 4KB", 4, {64, (cuuint64_t)W, (cuuint64_t)H, 8},
+       {(cuuint64_t)C * 2, (cuuint64_t)W * C * 2, 128}, {16, 64, 2, 1}, 1, H / 2, 8},
+  };
+  printf("S=%d sm_clock=%d MHz\n", S, clk_khz / 1000);
+  for (auto& c : cases) {
+    Maps mp;
+    const CUtensorMapSwizzle sw = c.box[0] * 2 >= 128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_32B;
+    cuuint32_t es[4] = {1, 1, 1, 1};
+    CUresult r = enc(&mp.m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, c.rank, X, c.dims, c.strides, c.box, es,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) {
+      printf("%s: encode failed %d\n", c.name, (int)r);
+      continue;
+    }
+    int bytes = 2;
+    for (int i = 0; i < c.rank; ++i) bytes *= c.box[i];
+    for (int ST : {1, 2, 4, 8}) {
+      const size_t smem = (size_t)ST * bytes + 1024;
+      if (smem > 220 * 1024) continue;
+      const void* kf = c.rank == 2 ? (const void*)k_tma<2> : (c.rank == 3 ? (const void*)k_tma<3> : (const void*)k_tma<4>);
+      cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024);
+      const int nbox = 400;
+      for (int rep = 0; rep < 2; ++rep) {
+        const int m1 = c.rank == 4 ? 0 : c.box[1], m2 = c.rank == 4 ? c.box[2] : (c.rank == 3 ? c.box[2] : 0),
+                  m3 = c.rank == 4 ? c.box[3] : 0;
+        if (c.rank == 2) k_tma<2><<<S, 32, smem>>>(mp, ST, nbox, bytes, c.d1, c.d2, c.d3, m1, m2, m3, d_out);
+        else if (c.rank == 3) k_tma<3><<<S, 32, smem>>>(mp, ST, nbox, bytes, c.d1, c.d2, c.d3, m1, m2, m3, d_out);
+        else k_tma<4><<<S, 32, smem>>>(mp, ST, nbox, bytes, c.d1, c.d2, c.d3, m1, m2, m3, d_out);
+      }
+      cudaError_t e = cudaDeviceSynchronize();
+      if (e != cudaSuccess) {
+        printf("%s ST=%d: %s\n", c.name, ST, cudaGetErrorString(e));
+        return 1;
+      }
+      cudaMemcpy(h.data(), d_out, S * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
+      double avg = 0;
+      for (int i = 0; i < S; ++i) avg += (double)h[i] / S;
+      const double ns_box = avg / nbox;
+      printf("%-40s ST=%d  %7.1f ns/box  %6.1f B/clk/SM  %7.1f GB/s/SM  chip %6.2f TB/s\n", c.name, ST, ns_box,
+             bytes / (ns_box * clk_khz / 1e6), bytes / ns_box, bytes / ns_box * S / 1e3);
+    }
+  }
+  return 0;
+}
