@@ -143,6 +143,34 @@ __device__ __forceinline__ void tc_mma(uint32_t d_tmem, uint64_t adesc, uint64_t
       "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc)
       : "memory");
 }
+// Warp-uniform issue: the whole MMA warp runs the loop, so descriptors and
+// TMEM addresses live in uniform registers, and ONE elected lane issues.
+// (Issuing from `if (lane == 0)` made ptxas wrap every tcgen05.mma in an
+// ELECT + R2UR.BROADCAST waterfall loop: ~150 cycles per MMA instead of the
+// 32-64 cycle tensor floor -- B200 phase traces, profiles/round2/mma_issue/.)
+__device__ __forceinline__ void tc_mma_e(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                         uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p, e;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc)
+      : "memory");
+}
+__device__ __forceinline__ void tc_commit_e(uint64_t* bar) {
+  asm volatile(
+      "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_e(uint64_t* bar) {
+  asm volatile(
+      "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+      "@e mbarrier.arrive.shared::cta.b64 _, [%0];\n\t}" ::"r"(smem_u32(bar))
+      : "memory");
+}
+
 // 32 lanes x 32 bit, 16 consecutive columns per thread
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
   asm volatile(
@@ -381,7 +409,9 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   float* epi_sc = (float*)(bar_base + 256);  // [BN] tile scale
   float* epi_sh = epi_sc + BN;               // [BN] tile shift
 
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  // warp index through a shuffle: provably warp-uniform, so role branches and
+  // the MMA warp's loop stay on the uniform datapath
+  const int warp = __shfl_sync(0xffffffffu, (int)(threadIdx.x >> 5), 0), lane = threadIdx.x & 31;
   if (threadIdx.x == 0) TR(1);   // 1: work entry
   // the first tile claim (an L2 atomic round trip) overlaps the barrier/TMEM setup
   bool marked = false;
@@ -564,8 +594,9 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       }
     }
   } else if (warp == 1) {
-    // ---------------- MMA issuer
+    // ---------------- MMA issuer (warp-uniform loop, elected issue)
     const uint32_t idesc = instr_desc<BN>();
+    const uint32_t tmem_u = __shfl_sync(0xffffffffu, tmem_base, 0);
     int stage = 0;
     uint32_t phase = 0;
     int astage = 0;
@@ -576,16 +607,16 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
     uint32_t aph = 0;
     for (;;) {
       mbar_wait(&rfull[rs], rph);
-      const int t = ring[rs];
+      const int t = __shfl_sync(0xffffffffu, ring[rs], 0);
       __syncwarp();
-      if (lane == 0) mbar_arrive(&rempty[rs]);
+      mbar_arrive_e(&rempty[rs]);
       if (++rs == 2) { rs = 0; rph ^= 1; }
       if (t < 0) break;
       const int ks = t % p.splits;
       const int kb0 = ks * p.kbs, kb1 = min(p.num_kb, kb0 + p.kbs);
       mbar_wait(&tempty[acc], aph ^ 1);
       tc_fence_after();
-      const uint32_t d_tmem = tmem_base + acc * BN;
+      const uint32_t d_tmem = tmem_u + acc * BN;
       if constexpr (HALO) {
         for (int c = kb0; c < kb1; ++c) {
           mbar_wait(&fullA[astage], aphase);
@@ -594,22 +625,20 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           for (int r = 0; r < p.R_; ++r) {   // one weight stage = filter row r (S taps)
             mbar_wait(&full[stage], phase);
             tc_fence_after();
-            if (lane == 0) {
-              const uint32_t b_row = smem_u32(sB + stage * b_bytes);
-              for (int s_ = 0; s_ < p.S_; ++s_) {
-                const uint32_t a0 = a_base + (uint32_t)(r * p.BW + s_) * 128u;
-                const uint32_t b0 = b_row + (uint32_t)s_ * (BN * 128u);
+            const uint32_t b_row = smem_u32(sB + stage * b_bytes);
+            for (int s_ = 0; s_ < p.S_; ++s_) {
+              const uint32_t a0 = a_base + (uint32_t)(r * p.BW + s_) * 128u;
+              const uint32_t b0 = b_row + (uint32_t)s_ * (BN * 128u);
 #pragma unroll
-                for (int k = 0; k < 4; ++k)
-                  tc_mma(d_tmem, smem_desc_row(a0 + k * 32), smem_desc<64>(b0 + k * 32), idesc,
+              for (int k = 0; k < 4; ++k)
+                tc_mma_e(d_tmem, smem_desc_row(a0 + k * 32), smem_desc<64>(b0 + k * 32), idesc,
                          (c != kb0 || r || s_ || k) ? 1u : 0u);
-              }
-              tc_commit(&empty[stage]);
             }
+            tc_commit_e(&empty[stage]);
             __syncwarp();
             if (++stage == ST) { stage = 0; phase ^= 1; }
           }
-          if (lane == 0) tc_commit(&emptyA[astage]);
+          tc_commit_e(&emptyA[astage]);
           __syncwarp();
           if (++astage == NA) { astage = 0; aphase ^= 1; }
         }
@@ -618,30 +647,25 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         mbar_wait(&full[stage], phase);
         tc_fence_after();
         if (lane == 0 && kb == kb0) TR(5);   // 5: first stage landed (last tile of this CTA)
-        if (lane == 0) {
-          const uint32_t a0 = smem_u32(sA + stage * Cfg::kStageA);
-          const uint32_t b0 = smem_u32(sB + stage * Cfg::kStageB);
-          if (kSkipMma) {
-            mbar_arrive(&empty[stage]);
-          } else {
+        const uint32_t a0 = smem_u32(sA + stage * Cfg::kStageA);
+        const uint32_t b0 = smem_u32(sB + stage * Cfg::kStageB);
+        if (kSkipMma) {
+          mbar_arrive_e(&empty[stage]);
+        } else {
 #pragma unroll
-            for (int k = 0; k < BK / 16; ++k) {
-              // BK = 128: slab k / 4 (128 x 64 of A, BN x 64 of B), K step k % 4
-              const uint32_t ao = BK > 64 ? (k >> 2) * (128 * 128) + (k & 3) * 32 : k * 32;
-              const uint32_t bo = BK > 64 ? (k >> 2) * (BN * 128) + (k & 3) * 32 : k * 32;
-              tc_mma(d_tmem, smem_desc<BK>(a0 + ao), smem_desc<BK>(b0 + bo), idesc,
-                     (kb != kb0 || k) ? 1u : 0u);
-            }
-            tc_commit(&empty[stage]);
+          for (int k = 0; k < BK / 16; ++k) {
+            // BK = 128: slab k / 4 (128 x 64 of A, BN x 64 of B), K step k % 4
+            const uint32_t ao = BK > 64 ? (k >> 2) * (128 * 128) + (k & 3) * 32 : k * 32;
+            const uint32_t bo = BK > 64 ? (k >> 2) * (BN * 128) + (k & 3) * 32 : k * 32;
+            tc_mma_e(d_tmem, smem_desc<BK>(a0 + ao), smem_desc<BK>(b0 + bo), idesc, (kb != kb0 || k) ? 1u : 0u);
           }
+          tc_commit_e(&empty[stage]);
         }
         __syncwarp();
         if (++stage == ST) { stage = 0; phase ^= 1; }
       }
-      if (lane == 0) {
-        if (kSkipMma) mbar_arrive(&tfull[acc]);
-        else tc_commit(&tfull[acc]);
-      }
+      if (kSkipMma) mbar_arrive_e(&tfull[acc]);
+      else tc_commit_e(&tfull[acc]);
       __syncwarp();
       if (++acc == Cfg::kAcc) { acc = 0; aph ^= 1; }
     }
@@ -1050,6 +1074,14 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     BN = 64;
     p.tiles_n = (p.N + BN - 1) / BN;
   }
+  if (p.mode == 3) {   // halo: the widest BN whose 1 halo + 2 filter-row stages fit (halo_stages)
+    auto fits = [&](int bn) {
+      const int fixed = 1024 + 256 + 2 * bn * 4;
+      return p.a_stage_bytes + 2 * p.S_ * bn * 128 <= 113 * 1024 - fixed;
+    };
+    while (BN > 16 && !fits(BN)) BN >>= 1;
+    p.tiles_n = (p.N + BN - 1) / BN;
+  }
   if (fs >= 1) splits = std::min(fs, p.num_kb);
   p.kbs = (p.num_kb + splits - 1) / splits;
   p.splits = (p.num_kb + p.kbs - 1) / p.kbs;
@@ -1137,7 +1169,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
 // reduction costs several us), BK = 128 wins the 3x3 convs, BN = 128 with
 // BK = 64 wins large GEMMs; BN = 256 never won with 96 KB of stages.
 int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int max) {
-  long long M, N, num_kb, tiles_m, halo_tiles_m = 0, chunks = 0;
+  long long M, N, num_kb, tiles_m, halo_tiles_m = 0, chunks = 0, halo_bw = 8;
   bool bk128_ok = false, halo_ok = false;
   if (op.kind == BL_OP_GEMM) {
     M = op.dims[0], N = op.dims[1];
@@ -1159,6 +1191,7 @@ int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int ma
     long long hw = 8;
     while (hw < OW + 2) hw <<= 1;
     halo_tiles_m = (OH + (128 / hw) - 1) / (128 / hw);
+    halo_bw = hw;
     chunks = C / 64;
   } else {
     return 0;
@@ -1167,7 +1200,9 @@ int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int ma
   const int nmax = N <= 16 ? 16 : (N <= 32 ? 32 : (N <= 64 ? 64 : 128));
   if (halo_ok) {
     // halo tiles: BH x BW with BW >= OW + 2; K blocks = 64-channel chunks
+    const long long a_stage = (((128 / halo_bw) + 2) * halo_bw + 8) * 128;
     for (int bn = std::min(32, nmax); bn <= nmax && n < max; bn <<= 1) {
+      if ((a_stage + 1023) / 1024 * 1024 + 2 * 3 * bn * 128 > 113 * 1024 - (1024 + 256 + 2 * bn * 4)) break;
       const long long tiles = halo_tiles_m * ((N + bn - 1) / bn);
       out[n++] = TcChoice{bn, 1, 64, 1};
       if (tiles < caps.S && chunks >= 2 && n < max) {
