@@ -77,8 +77,21 @@ __device__ __forceinline__ void tr_mark(int i) {
   if (blockIdx.x < kTrMax) g_tc_trace[blockIdx.x][i] = t;
 }
 #define TR(i) tr_mark(i)
+// wait accounting per CTA: [0] MMA warp waiting for operands (ns), [1] count,
+// [2] producer waiting for free stages (ns), [3] count
+__device__ unsigned long long g_tc_wait[kTrMax][4];
+__device__ __forceinline__ unsigned long long tr_now() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define TW_BEGIN() const unsigned long long tw0_ = tr_now()
+#define TW_END(slot) \
+  if ((threadIdx.x & 31) == 0 && blockIdx.x < kTrMax) { g_tc_wait[blockIdx.x][slot] += tr_now() - tw0_; g_tc_wait[blockIdx.x][slot + 1] += 1; }
 #else
 #define TR(i) ((void)0)
+#define TW_BEGIN() ((void)0)
+#define TW_END(slot) ((void)0)
 #endif
 
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
@@ -537,13 +550,13 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           // per 64-channel chunk: the input halo once, then one weight box per filter row
           const int taps = p.R_;
           auto load_Bt = [&](int c, int r) {
-            mbar_wait(&empty[stage], phase ^ 1);
+            { TW_BEGIN(); mbar_wait(&empty[stage], phase ^ 1); TW_END(2); }
             mbar_expect_tx(&full[stage], (uint32_t)b_bytes);
             tma_load_3d(sB + stage * b_bytes, &p.tmB, &full[stage], c * 64, tn * BN, r * p.S_);
             if (++stage == ST) { stage = 0; phase ^= 1; }
           };
           auto load_halo = [&](int c) {
-            mbar_wait(&emptyA[astage], aphase ^ 1);
+            { TW_BEGIN(); mbar_wait(&emptyA[astage], aphase ^ 1); TW_END(2); }
             mbar_expect_tx(&fullA[astage], (uint32_t)p.a_tx);
             tma_load_4d(sA + astage * a_bytes, &p.tmA, &fullA[astage], c * 64, -p.pad, oh0 - p.pad, 0);
             if (++astage == NA) { astage = 0; aphase ^= 1; }
@@ -585,7 +598,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           kb = kb0 + npre;
         }
         for (; kb < kb1; ++kb) {
-          mbar_wait(&empty[stage], phase ^ 1);
+          { TW_BEGIN(); mbar_wait(&empty[stage], phase ^ 1); TW_END(2); }
           mbar_expect_tx(&full[stage], kTxBytes);
           if (!kSkipB) load_B(kb, stage);
           if (!kSkipA) load_A(kb, stage);
@@ -619,11 +632,11 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       const uint32_t d_tmem = tmem_u + acc * BN;
       if constexpr (HALO) {
         for (int c = kb0; c < kb1; ++c) {
-          mbar_wait(&fullA[astage], aphase);
+          { TW_BEGIN(); mbar_wait(&fullA[astage], aphase); TW_END(0); }
           tc_fence_after();
           const uint32_t a_base = smem_u32(sA + astage * a_bytes);
           for (int r = 0; r < p.R_; ++r) {   // one weight stage = filter row r (S taps)
-            mbar_wait(&full[stage], phase);
+            { TW_BEGIN(); mbar_wait(&full[stage], phase); TW_END(0); }
             tc_fence_after();
             const uint32_t b_row = smem_u32(sB + stage * b_bytes);
             for (int s_ = 0; s_ < p.S_; ++s_) {
@@ -644,7 +657,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         }
       }
       for (int kb = HALO ? kb1 : kb0; kb < kb1; ++kb) {
-        mbar_wait(&full[stage], phase);
+        { TW_BEGIN(); mbar_wait(&full[stage], phase); TW_END(0); }
         tc_fence_after();
         if (lane == 0 && kb == kb0) TR(5);   // 5: first stage landed (last tile of this CTA)
         const uint32_t a0 = smem_u32(sA + stage * Cfg::kStageA);
@@ -1235,8 +1248,14 @@ extern "C" int bl_debug_tc_trace(unsigned long long* host, int n_cta) {
   const size_t n = (size_t)std::min(n_cta, bless::kTrMax) * bless::kTrN * sizeof(unsigned long long);
   return (int)cudaMemcpyFromSymbol(host, bless::g_tc_trace, n);
 }
+extern "C" int bl_debug_tc_wait(unsigned long long* host, int n_cta) {
+  const size_t n = (size_t)std::min(n_cta, bless::kTrMax) * 4 * sizeof(unsigned long long);
+  return (int)cudaMemcpyFromSymbol(host, bless::g_tc_wait, n);
+}
 extern "C" int bl_debug_tc_trace_clear() {
   static unsigned long long z[bless::kTrMax][bless::kTrN];
+  static unsigned long long zw[bless::kTrMax][4];
+  cudaMemcpyToSymbol(bless::g_tc_wait, zw, sizeof(zw));
   return (int)cudaMemcpyToSymbol(bless::g_tc_trace, z, sizeof(z));
 }
 #endif

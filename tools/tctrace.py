@@ -63,6 +63,16 @@ def main():
                 print(f"  {i} {nm:10s} {col.min() / 1e3:8.2f} {np.median(col) / 1e3:8.2f} {col.max() / 1e3:8.2f}")
         allx = v[v[:, 9] > 0, 9] - t0
         print(f"  last CTA exit (all CTAs) {allx.max() / 1e3:.2f} us")
+        if reps == 1:   # wait accounting of that single launch (counters accumulate over launches)
+            wb = np.zeros((2048, 4), dtype=np.uint64)
+            L.bl_debug_tc_wait.argtypes = [C.c_void_p, C.c_int]
+            L.bl_debug_tc_wait(wb.ctypes.data, 2048)
+            wb = wb.astype(np.int64)
+            act = wb[:, 1] > 0
+            if act.any():
+                print(f"  MMA warp waiting for operands: {wb[act, 0].mean() / 1e3:.2f} us over "
+                      f"{wb[act, 1].mean():.1f} waits; producer waiting for free stages: "
+                      f"{wb[act, 2].mean() / 1e3:.2f} us over {wb[act, 3].mean():.1f} waits (per working CTA)")
     ctx.close()
 
 

@@ -78,6 +78,135 @@ __global__ void k_tma(const __grid_constant__ Maps mp, int ST, int nbox, int box
   out[blockIdx.x] = t1 - t0;
 }
 
+// Same ring with the engine's handoff: warp 0 (one thread) issues loads into
+// stage s after waiting on empty[s]; warp 1 waits on full[s] and arrives on
+// empty[s] (what the MMA warp does after its MMAs).  Measures the cost of the
+// two mbarrier handoffs per stage on top of the TMA time.
+template <int RANK>
+__global__ void k_tma_pc(const __grid_constant__ Maps mp, int ST, int nbox, int box_bytes, int d1, int d2, int d3,
+                         int m1, int m2, int m3, unsigned long long* out) {
+  extern __shared__ __align__(1024) unsigned char sm_raw[];
+  unsigned char* sm = (unsigned char*)(((uintptr_t)sm_raw + 1023) & ~(uintptr_t)1023);
+  __shared__ uint64_t full[16], empty[16];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < ST; ++i) {
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&full[i])));
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&empty[i])));
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  unsigned long long t0;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  if (warp == 0 && lane == 0) {
+    for (int i = 0; i < nbox; ++i) {
+      const int s = i % ST;
+      const uint32_t ph = ((i / ST) & 1) ^ 1;
+      asm volatile(
+          "{\n\t.reg .pred p;\n\tW_%=:\n\t"
+          "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t@!p bra W_%=;\n\t}" ::"r"(su32(&empty[s])),
+          "r"(ph)
+          : "memory");
+      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(su32(&full[s])), "r"(box_bytes)
+                   : "memory");
+      const int c1 = ((blockIdx.x * 7 + i) % d1) * m1, c2 = ((blockIdx.x * 3 + i / d1) % d2) * m2,
+                c3 = ((i / (d1 * d2)) % d3) * m3;
+      void* dst = sm + (size_t)s * box_bytes;
+      if (RANK == 2)
+        asm volatile(
+            "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];"
+            ::"r"(su32(dst)), "l"(&mp.m), "r"(su32(&full[s])), "r"(0), "r"(c1) : "memory");
+      else
+        asm volatile(
+            "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6}], "
+            "[%2];" ::"r"(su32(dst)), "l"(&mp.m), "r"(su32(&full[s])), "r"(0), "r"(c1 - 1), "r"(c2 - 1), "r"(c3)
+            : "memory");
+    }
+  } else if (warp == 1) {
+    for (int i = 0; i < nbox; ++i) {
+      const int s = i % ST;
+      const uint32_t ph = (i / ST) & 1;
+      asm volatile(
+          "{\n\t.reg .pred p;\n\tW_%=:\n\t"
+          "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t@!p bra W_%=;\n\t}" ::"r"(su32(&full[s])),
+          "r"(ph)
+          : "memory");
+      if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(su32(&empty[s])) : "memory");
+      __syncwarp();
+    }
+    unsigned long long t1;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
+    if (lane == 0) out[blockIdx.x] = t1 - t0;
+  }
+}
+
+// tcgen05.mma issue rate: one warp issues n MMAs (M = 128, N = BN, K = 16,
+// bf16, A/B from zeroed shared memory, D in TMEM) and waits for their commit;
+// 'elect' = warp-uniform loop with elect.sync, else `if (lane == 0)`.
+template <int BN>
+__global__ void k_mma_rate(int n, int elect, unsigned long long* out) {
+  extern __shared__ __align__(1024) unsigned char sm_raw[];
+  unsigned char* sm = (unsigned char*)(((uintptr_t)sm_raw + 1023) & ~(uintptr_t)1023);
+  __shared__ uint64_t bar;
+  __shared__ uint32_t tslot;
+  const int lane = threadIdx.x & 31;
+  for (int i = threadIdx.x; i < (128 + BN) * 128 / 4; i += 32) ((uint32_t*)sm)[i] = 0;
+  if (lane == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&bar)));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 256;" ::"r"(su32(&tslot)));
+  asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncwarp();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tm = __shfl_sync(0xffffffffu, tslot, 0);
+  const uint32_t a = su32(sm), b = su32(sm + 128 * 128);
+  auto desc = [](uint32_t addr) {
+    uint64_t d = (uint64_t)((addr >> 4) & 0x3FFF) | ((uint64_t)1 << 16) | ((uint64_t)(1024 >> 4) << 32) |
+                 ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
+    return d;
+  };
+  const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+  unsigned long long t0, t1;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  if (elect) {
+    for (int i = 0; i < n; ++i) {
+      const uint32_t k = (i & 3) * 32;
+      asm volatile(
+          "{\n\t.reg .pred p, e;\n\telect.sync _|e, 0xffffffff;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+          "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tm),
+          "l"(desc(a + k)), "l"(desc(b + k)), "r"(idesc), "r"(i)
+          : "memory");
+    }
+    asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+                 "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(su32(&bar))
+                 : "memory");
+  } else if (lane == 0) {
+    for (int i = 0; i < n; ++i) {
+      const uint32_t k = (i & 3) * 32;
+      asm volatile(
+          "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+          "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tm),
+          "l"(desc(a + k)), "l"(desc(b + k)), "r"(idesc), "r"(i)
+          : "memory");
+    }
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(su32(&bar))
+                 : "memory");
+  }
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tW_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], 0;\n\t@!p bra W_%=;\n\t}" ::"r"(su32(&bar))
+      : "memory");
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
+  if (lane == 0) out[blockIdx.x] = t1 - t0;
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncwarp();
+  asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 256;" ::"r"(tm));
+}
+
 typedef CUresult (*Enc)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*, const cuuint64_t*,
                         const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
                         CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
@@ -123,6 +252,29 @@ int main() {
        {(cuuint64_t)C * 2, (cuuint64_t)W * C * 2, 128}, {16, 64, 2, 1}, 1, H / 2, 8},
   };
   printf("S=%d sm_clock=%d MHz\n", S, clk_khz / 1000);
+  // MMA issue rate
+  for (int elect = 0; elect < 2; ++elect) {
+    for (int bn : {64, 128, 256}) {
+      const void* kf = bn == 64 ? (const void*)k_mma_rate<64> : (bn == 128 ? (const void*)k_mma_rate<128>
+                                                                           : (const void*)k_mma_rate<256>);
+      cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024);
+      const int n = 2048;
+      for (int rep = 0; rep < 2; ++rep) {
+        if (bn == 64) k_mma_rate<64><<<S, 32, 96 * 1024>>>(n, elect, d_out);
+        else if (bn == 128) k_mma_rate<128><<<S, 32, 96 * 1024>>>(n, elect, d_out);
+        else k_mma_rate<256><<<S, 32, 96 * 1024>>>(n, elect, d_out);
+      }
+      cudaError_t e = cudaDeviceSynchronize();
+      if (e != cudaSuccess) { printf("mma: %s\n", cudaGetErrorString(e)); return 1; }
+      cudaMemcpy(h.data(), d_out, S * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
+      double avg = 0;
+      for (int i = 0; i < S; ++i) avg += (double)h[i] / S;
+      const double cyc = avg / n * clk_khz / 1e6;
+      printf("MMA 128x%dx16 %s: %.1f ns/mma = %.1f cycles (floor %d)  -> %.0f TF/s chip\n", bn,
+             elect ? "elect.sync uniform loop" : "if (lane == 0)      ", avg / n, cyc, 128 * bn / 256,
+             2.0 * 128 * bn * 16 / (avg / n) * S / 1e3);
+    }
+  }
   for (auto& c : cases) {
     Maps mp;
     const CUtensorMapSwizzle sw = c.box[0] * 2 >= 128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_32B;
@@ -160,6 +312,21 @@ int main() {
       const double ns_box = avg / nbox;
       printf("%-40s ST=%d  %7.1f ns/box  %6.1f B/clk/SM  %7.1f GB/s/SM  chip %6.2f TB/s\n", c.name, ST, ns_box,
              bytes / (ns_box * clk_khz / 1e6), bytes / ns_box, bytes / ns_box * S / 1e3);
+      if (c.rank == 3) continue;
+      {   // producer/consumer handoff variant
+        const int m1 = c.rank == 4 ? 0 : c.box[1], m2 = c.rank == 4 ? c.box[2] : 0, m3 = c.rank == 4 ? c.box[3] : 0;
+        const void* kp = c.rank == 2 ? (const void*)k_tma_pc<2> : (const void*)k_tma_pc<4>;
+        cudaFuncSetAttribute(kp, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024);
+        for (int rep = 0; rep < 2; ++rep) {
+          if (c.rank == 2) k_tma_pc<2><<<S, 64, smem>>>(mp, ST, nbox, bytes, c.d1, c.d2, c.d3, m1, m2, m3, d_out);
+          else k_tma_pc<4><<<S, 64, smem>>>(mp, ST, nbox, bytes, c.d1, c.d2, c.d3, m1, m2, m3, d_out);
+        }
+        cudaDeviceSynchronize();
+        cudaMemcpy(h.data(), d_out, S * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
+        double a2 = 0;
+        for (int i = 0; i < S; ++i) a2 += (double)h[i] / S;
+        printf("%-40s ST=%d  %7.1f ns/box  (producer/consumer mbarrier handoff)\n", c.name, ST, a2 / nbox);
+      }
     }
   }
   return 0;
