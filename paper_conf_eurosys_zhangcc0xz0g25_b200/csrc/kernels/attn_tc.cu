@@ -88,6 +88,35 @@ __device__ __forceinline__ void commit(uint64_t* bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(su32(bar))
                : "memory");
 }
+// Elected-lane variants: warp 0 runs the load/MMA sequence as a whole warp
+// (uniform descriptors in uniform registers) and one elected lane issues
+// (issuing under `if (lane == 0)` wrapped every tcgen05.mma in an ELECT +
+// R2UR.BROADCAST waterfall loop -- see tc_gemm.cu).
+__device__ __forceinline__ void bar_expect_e(uint64_t* b, uint32_t bytes) {
+  asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+               "@e mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n\t}" ::"r"(su32(b)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void tma2d_e(void* dst, const CUtensorMap* m, uint64_t* bar, int c0, int c1) {
+  asm volatile(
+      "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+      "@e cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];"
+      "\n\t}" ::"r"(su32(dst)),
+      "l"(m), "r"(su32(bar)), "r"(c0), "r"(c1)
+      : "memory");
+}
+__device__ __forceinline__ void mma_e(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p, e;\n\telect.sync _|e, 0xffffffff;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d),
+      "l"(a), "l"(b), "r"(idesc), "r"(acc)
+      : "memory");
+}
+__device__ __forceinline__ void commit_e(uint64_t* bar) {
+  asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+               "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(su32(bar))
+               : "memory");
+}
 __device__ __forceinline__ void ld16(uint32_t taddr, uint32_t (&v)[16]) {
   asm volatile(
       "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
@@ -146,7 +175,7 @@ __device__ void attn_work(const AttnTcParams& p, const GateArgs& g) {
   uint32_t* tmem_slot = (uint32_t*)(tile_slot + 1);
   float* red_max = (float*)(bars + 32);   // [kParts][128] per key part
   float* red_sum = red_max + kParts * 128;  // [kParts][128]
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int warp = __shfl_sync(0xffffffffu, (int)(threadIdx.x >> 5), 0), lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     bar_init(b_qk, 1);
     bar_init(b_v, 1);
@@ -166,7 +195,7 @@ __device__ void attn_work(const AttnTcParams& p, const GateArgs& g) {
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-  const uint32_t tmem = *tmem_slot;
+  const uint32_t tmem = __shfl_sync(0xffffffffu, *tmem_slot, 0);
   pdl_wait();
   const int L = p.L, H = p.H;
   const int nkb = L / 64;      // 64-key blocks
@@ -175,45 +204,44 @@ __device__ void attn_work(const AttnTcParams& p, const GateArgs& g) {
   for (;;) {
     if (threadIdx.x == 0) *tile_slot = gate_claim(g, marked);
     __syncthreads();
-    const int t = *tile_slot;
+    const int t = __shfl_sync(0xffffffffu, *tile_slot, 0);
     __syncthreads();
     if (t < 0) break;
     const int h = t / p.qblocks, qb = t - h * p.qblocks;
     if (warp == 0) {
-      if (lane == 0) {
-        // ---- loads: Q block and K (K-major, SW128)
-        bar_expect(b_qk, kQBytes + L * 128);
-        tma2d(sQ, &p.tm, b_qk, h * 64, qb * 128);
-        for (int r = 0; r < L; r += 128) tma2d(sKV + r * 128, &p.tm, b_qk, H * 64 + h * 64, r);
-        bar_wait(b_qk, ph);
-        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        // ---- S = Q K^T  (N chunks of <= 256 keys, 4 k-steps of 16 over dh = 64)
-        for (int n0 = 0; n0 < L; n0 += 256) {
-          const int N = (L - n0) < 256 ? (L - n0) : 256;
-          const uint32_t id = idesc(N, false);
-          for (int k = 0; k < 4; ++k)
-            mma(tmem + n0, desc_k(su32(sQ) + k * 32), desc_k(su32(sKV) + n0 * 128 + k * 32), id, k ? 1u : 0u);
-        }
-        commit(b_s);
-        // ---- V into the K buffer once the S MMAs have consumed it
-        bar_wait(b_s, ph);
-        bar_expect(b_v, L * 128);
-        for (int r = 0; r < L; r += 128) tma2d(sKV + r * 128, &p.tm, b_v, 2 * H * 64 + h * 64, r);
-        bar_wait(b_v, ph);
-        // ---- O = P V : A = P (K-major, nkb blocks of 64 keys), B = V (MN-major, keys x dh),
-        // in two passes P = P_hi + P_lo (bf16 each) for ~16-bit precision of P
-        const uint32_t id = idesc(64, true);
-        for (int pass = 0; pass < 2; ++pass) {
-          bar_wait(pass == 0 ? b_p : b_p2, ph);   // P part in smem (writers fenced the generic proxy)
-          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-          for (int kb = 0; kb < nkb; ++kb)
-            for (int k = 0; k < 4; ++k)
-              mma(tmem + 448, desc_k(su32(sP) + kb * 16384 + k * 32),
-                  desc_mn(su32(sKV) + kb * 64 * 128 + k * 16 * 128), id, (pass | kb | k) ? 1u : 0u);
-          commit(pass == 0 ? b_o1 : b_o);
-        }
-        bar_wait(b_done, ph);   // epilogue drained O before the next tile reuses TMEM / smem
+      // whole warp: loads / MMAs issued by one elected lane (uniform loop)
+      // ---- loads: Q block and K (K-major, SW128)
+      bar_expect_e(b_qk, kQBytes + L * 128);
+      tma2d_e(sQ, &p.tm, b_qk, h * 64, qb * 128);
+      for (int r = 0; r < L; r += 128) tma2d_e(sKV + r * 128, &p.tm, b_qk, H * 64 + h * 64, r);
+      bar_wait(b_qk, ph);
+      asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      // ---- S = Q K^T  (N chunks of <= 256 keys, 4 k-steps of 16 over dh = 64)
+      for (int n0 = 0; n0 < L; n0 += 256) {
+        const int N = (L - n0) < 256 ? (L - n0) : 256;
+        const uint32_t id = idesc(N, false);
+        for (int k = 0; k < 4; ++k)
+          mma_e(tmem + n0, desc_k(su32(sQ) + k * 32), desc_k(su32(sKV) + n0 * 128 + k * 32), id, k ? 1u : 0u);
       }
+      commit_e(b_s);
+      // ---- V into the K buffer once the S MMAs have consumed it
+      bar_wait(b_s, ph);
+      bar_expect_e(b_v, L * 128);
+      for (int r = 0; r < L; r += 128) tma2d_e(sKV + r * 128, &p.tm, b_v, 2 * H * 64 + h * 64, r);
+      bar_wait(b_v, ph);
+      // ---- O = P V : A = P (K-major, nkb blocks of 64 keys), B = V (MN-major, keys x dh),
+      // in two passes P = P_hi + P_lo (bf16 each) for ~16-bit precision of P
+      const uint32_t id = idesc(64, true);
+      for (int pass = 0; pass < 2; ++pass) {
+        bar_wait(pass == 0 ? b_p : b_p2, ph);   // P part in smem (writers fenced the generic proxy)
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        for (int kb = 0; kb < nkb; ++kb)
+          for (int k = 0; k < 4; ++k)
+            mma_e(tmem + 448, desc_k(su32(sP) + kb * 16384 + k * 32),
+                  desc_mn(su32(sKV) + kb * 64 * 128 + k * 16 * 128), id, (pass | kb | k) ? 1u : 0u);
+        commit_e(pass == 0 ? b_o1 : b_o);
+      }
+      bar_wait(b_done, ph);   // epilogue drained O before the next tile reuses TMEM / smem
       __syncwarp();
     } else {
       // ---- softmax: thread = query row (TMEM lane) x key half

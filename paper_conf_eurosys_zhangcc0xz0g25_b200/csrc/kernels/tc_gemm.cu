@@ -60,6 +60,8 @@ struct TcParams {
   // 1 + R boxes instead of 2 per tap (B200: a TMA box costs >= 130-180 ns per
   // SM whatever its size, profiles/round2/halo/tma_bench.txt)
   int b_stage_bytes;
+  int taps_per_b;   // taps per weight box: S (one filter row, BN <= 64) or 1 (BN = 128: N >= 128 MMAs
+                    // run at the tensor floor, N = 64 at ~60% of it; a 3-tap 128-wide box does not fit)
 };
 
 #ifdef __CUDACC__
@@ -141,6 +143,41 @@ __device__ __forceinline__ void tma_load_5d(void* dst, const CUtensorMap* map, u
       "[%2];" ::"r"(smem_u32(dst)),
       "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4)
       : "memory");
+}
+// elected-lane TMA issue for the warp-uniform producer loop
+#define BLESS_ELECT_ASM(body) "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t@e " body "\n\t}"
+__device__ __forceinline__ void mbar_expect_tx_e(uint64_t* bar, uint32_t bytes) {
+  asm volatile(BLESS_ELECT_ASM("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;") ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void tma_load_2d_e(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1) {
+  asm volatile(BLESS_ELECT_ASM(
+                   "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], "
+                   "[%2];") ::"r"(smem_u32(dst)),
+               "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
+               : "memory");
+}
+__device__ __forceinline__ void tma_load_3d_e(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1,
+                                              int c2) {
+  asm volatile(BLESS_ELECT_ASM("cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, "
+                               "{%3, %4, %5}], [%2];") ::"r"(smem_u32(dst)),
+               "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2)
+               : "memory");
+}
+__device__ __forceinline__ void tma_load_4d_e(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1, int c2,
+                                              int c3) {
+  asm volatile(BLESS_ELECT_ASM("cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, "
+                               "{%3, %4, %5, %6}], [%2];") ::"r"(smem_u32(dst)),
+               "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+               : "memory");
+}
+__device__ __forceinline__ void tma_load_5d_e(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1, int c2,
+                                              int c3, int c4) {
+  asm volatile(BLESS_ELECT_ASM("cp.async.bulk.tensor.5d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, "
+                               "{%3, %4, %5, %6, %7}], [%2];") ::"r"(smem_u32(dst)),
+               "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4)
+               : "memory");
 }
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
@@ -479,10 +516,13 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
 #endif
   constexpr uint32_t kTxBytes = (kSkipA ? 0u : (uint32_t)Cfg::kStageA) + (kSkipB ? 0u : (uint32_t)Cfg::kStageB);
   if (warp == 0) {
-    // ---------------- tile scheduler + TMA producer
+    // ---------------- tile scheduler + TMA producer: the whole warp runs the
+    // loop (uniform coordinates), lane 0 claims tiles, an elected lane issues
     if (lane == 0) {
       asm volatile("prefetch.tensormap [%0];" ::"l"(&p.tmA) : "memory");
       asm volatile("prefetch.tensormap [%0];" ::"l"(&p.tmB) : "memory");
+    }
+    {
       bool dep_waited = false;
       int stage = 0;
       uint32_t phase = 0;
@@ -491,12 +531,17 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       int rs = 0;
       uint32_t rph = 0;
       for (;;) {
-        const int t = first_claim != -2 ? first_claim : gate_claim(g, marked, dep_waited);
+        int t0 = 0;
+        if (lane == 0) t0 = first_claim != -2 ? first_claim : gate_claim(g, marked, dep_waited);
+        const int t = __shfl_sync(0xffffffffu, t0, 0);
         first_claim = -2;
-        if (!dep_waited) TR(3);          // 3: first claim returned
+        if (!dep_waited && lane == 0) TR(3);          // 3: first claim returned
         mbar_wait(&rempty[rs], rph ^ 1);
-        ring[rs] = t;
-        mbar_arrive(&rfull[rs]);
+        if (lane == 0) {
+          ring[rs] = t;
+          mbar_arrive(&rfull[rs]);
+        }
+        __syncwarp();
         if (++rs == 2) { rs = 0; rph ^= 1; }
         if (t < 0) {
           pdl_trigger();  // queue exhausted: let the next kernel on this stream launch
@@ -515,50 +560,50 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           unsigned char* b = sB + st * Cfg::kStageB;
           if (BK > 64) {   // 3-D view (64, N, K/64): one box = two 64-deep slabs
             const int kc = p.mode == 0 ? kb * 2 : (kb / p.kc_per_tap) * (p.C / 64) + (kb % p.kc_per_tap) * 2;
-            tma_load_3d(b, &p.tmB, &full[st], 0, tn * BN, kc);
+            tma_load_3d_e(b, &p.tmB, &full[st], 0, tn * BN, kc);
           } else if (p.mode == 0) {
-            tma_load_2d(b, &p.tmB, &full[st], kb * BK, tn * BN);
+            tma_load_2d_e(b, &p.tmB, &full[st], kb * BK, tn * BN);
           } else {
             const int tap = kb / p.kc_per_tap, c0 = (kb - tap * p.kc_per_tap) * BK;
-            tma_load_2d(b, &p.tmB, &full[st], tap * p.C + c0, tn * BN);
+            tma_load_2d_e(b, &p.tmB, &full[st], tap * p.C + c0, tn * BN);
           }
         };
         auto load_A = [&](int kb, int st) {
           unsigned char* a = sA + st * Cfg::kStageA;
           if (BK > 64 && p.mode == 0) {   // 3-D view (64, M, K/64)
-            tma_load_3d(a, &p.tmA, &full[st], 0, tm * 128, kb * 2);
+            tma_load_3d_e(a, &p.tmA, &full[st], 0, tm * 128, kb * 2);
           } else if (BK > 64) {            // 4-D view (64, W, H, C/64), stride 1 only
             const int tap = kb / p.kc_per_tap, ch = (kb - tap * p.kc_per_tap) * 2;
             const int r = tap / p.S_, s = tap - r * p.S_;
-            tma_load_4d(a, &p.tmA, &full[st], 0, ow0 - p.pad + s, oh0 - p.pad + r, ch);
+            tma_load_4d_e(a, &p.tmA, &full[st], 0, ow0 - p.pad + s, oh0 - p.pad + r, ch);
           } else if (p.mode == 0) {
-            tma_load_2d(a, &p.tmA, &full[st], kb * BK, tm * 128);
+            tma_load_2d_e(a, &p.tmA, &full[st], kb * BK, tm * 128);
           } else {
             const int tap = kb / p.kc_per_tap, c0 = (kb - tap * p.kc_per_tap) * BK;
             const int r = tap / p.S_, s = tap - r * p.S_;
             if (p.mode == 1) {
-              tma_load_4d(a, &p.tmA, &full[st], c0, ow0 - p.pad + s, oh0 - p.pad + r, 0);
+              tma_load_4d_e(a, &p.tmA, &full[st], c0, ow0 - p.pad + s, oh0 - p.pad + r, 0);
             } else {
               const int dr = r - p.pad, ds = s - p.pad;
               const int ph = dr & 1, pw = ds & 1;        // parity of the input row/col
               const int qh = (dr - ph) / 2, qw = (ds - pw) / 2;
-              tma_load_5d(a, &p.tmA, &full[st], c0, pw, ow0 + qw, ph, oh0 + qh);
+              tma_load_5d_e(a, &p.tmA, &full[st], c0, pw, ow0 + qw, ph, oh0 + qh);
             }
           }
         };
         if constexpr (HALO) {
           // per 64-channel chunk: the input halo once, then one weight box per filter row
-          const int taps = p.R_;
-          auto load_Bt = [&](int c, int r) {
+          const int taps = p.R_ * p.S_ / p.taps_per_b;   // weight boxes per chunk
+          auto load_Bt = [&](int c, int j) {
             { TW_BEGIN(); mbar_wait(&empty[stage], phase ^ 1); TW_END(2); }
-            mbar_expect_tx(&full[stage], (uint32_t)b_bytes);
-            tma_load_3d(sB + stage * b_bytes, &p.tmB, &full[stage], c * 64, tn * BN, r * p.S_);
+            mbar_expect_tx_e(&full[stage], (uint32_t)b_bytes);
+            tma_load_3d_e(sB + stage * b_bytes, &p.tmB, &full[stage], c * 64, tn * BN, j * p.taps_per_b);
             if (++stage == ST) { stage = 0; phase ^= 1; }
           };
           auto load_halo = [&](int c) {
             { TW_BEGIN(); mbar_wait(&emptyA[astage], aphase ^ 1); TW_END(2); }
-            mbar_expect_tx(&fullA[astage], (uint32_t)p.a_tx);
-            tma_load_4d(sA + astage * a_bytes, &p.tmA, &fullA[astage], c * 64, -p.pad, oh0 - p.pad, 0);
+            mbar_expect_tx_e(&fullA[astage], (uint32_t)p.a_tx);
+            tma_load_4d_e(sA + astage * a_bytes, &p.tmA, &fullA[astage], c * 64, -p.pad, oh0 - p.pad, 0);
             if (++astage == NA) { astage = 0; aphase ^= 1; }
           };
           for (int c = kb0; c < kb1; ++c) {
@@ -567,8 +612,8 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
               tap0 = min(taps, ST);
               for (int tap = 0; tap < tap0; ++tap) load_Bt(c, tap);
               pdl_wait();
-              if (t == 0) gate_prev_end(g, (int64_t)ptx_globaltimer());
-              TR(4);
+              if (t == 0 && lane == 0) gate_prev_end(g, (int64_t)ptx_globaltimer());
+              if (lane == 0) TR(4);
               dep_waited = true;
             }
             load_halo(c);
@@ -584,12 +629,12 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           for (int i = 0; i < npre; ++i) {
             const int st = (stage + i) % ST;
             mbar_wait(&empty[st], (phase ^ (stage + i >= ST ? 1 : 0)) ^ 1);
-            mbar_expect_tx(&full[st], kTxBytes);
+            mbar_expect_tx_e(&full[st], kTxBytes);
             if (!kSkipB) load_B(kb0 + i, st);
           }
           pdl_wait();
-          if (t == 0) gate_prev_end(g, (int64_t)ptx_globaltimer());   // predecessor just completed
-          TR(4);                         // 4: producer past griddepcontrol.wait
+          if (t == 0 && lane == 0) gate_prev_end(g, (int64_t)ptx_globaltimer());   // predecessor just completed
+          if (lane == 0) TR(4);          // 4: producer past griddepcontrol.wait
           dep_waited = true;
           for (int i = 0; i < npre; ++i)
             if (!kSkipA) load_A(kb0 + i, (stage + i) % ST);
@@ -599,7 +644,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         }
         for (; kb < kb1; ++kb) {
           { TW_BEGIN(); mbar_wait(&empty[stage], phase ^ 1); TW_END(2); }
-          mbar_expect_tx(&full[stage], kTxBytes);
+          mbar_expect_tx_e(&full[stage], kTxBytes);
           if (!kSkipB) load_B(kb, stage);
           if (!kSkipA) load_A(kb, stage);
           if (++stage == ST) { stage = 0; phase ^= 1; }
@@ -635,17 +680,19 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           { TW_BEGIN(); mbar_wait(&fullA[astage], aphase); TW_END(0); }
           tc_fence_after();
           const uint32_t a_base = smem_u32(sA + astage * a_bytes);
-          for (int r = 0; r < p.R_; ++r) {   // one weight stage = filter row r (S taps)
+          const int nbox = p.R_ * p.S_ / p.taps_per_b;
+          for (int j = 0; j < nbox; ++j) {   // one weight stage = taps_per_b consecutive taps
             { TW_BEGIN(); mbar_wait(&full[stage], phase); TW_END(0); }
             tc_fence_after();
             const uint32_t b_row = smem_u32(sB + stage * b_bytes);
-            for (int s_ = 0; s_ < p.S_; ++s_) {
+            for (int u = 0; u < p.taps_per_b; ++u) {
+              const int tap = j * p.taps_per_b + u, r = tap / p.S_, s_ = tap - r * p.S_;
               const uint32_t a0 = a_base + (uint32_t)(r * p.BW + s_) * 128u;
-              const uint32_t b0 = b_row + (uint32_t)s_ * (BN * 128u);
+              const uint32_t b0 = b_row + (uint32_t)u * (BN * 128u);
 #pragma unroll
               for (int k = 0; k < 4; ++k)
                 tc_mma_e(d_tmem, smem_desc_row(a0 + k * 32), smem_desc<64>(b0 + k * 32), idesc,
-                         (c != kb0 || r || s_ || k) ? 1u : 0u);
+                         (c != kb0 || tap || k) ? 1u : 0u);
             }
             tc_commit_e(&empty[stage]);
             __syncwarp();
@@ -1087,13 +1134,15 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     BN = 64;
     p.tiles_n = (p.N + BN - 1) / BN;
   }
-  if (p.mode == 3) {   // halo: the widest BN whose 1 halo + 2 filter-row stages fit (halo_stages)
+  if (p.mode == 3) {   // halo: the widest BN whose 1 halo + 2 weight stages fit (halo_stages)
+    auto tpb = [&](int bn) { return bn >= 128 ? 1 : p.S_; };
     auto fits = [&](int bn) {
       const int fixed = 1024 + 256 + 2 * bn * 4;
-      return p.a_stage_bytes + 2 * p.S_ * bn * 128 <= 113 * 1024 - fixed;
+      return p.a_stage_bytes + 2 * tpb(bn) * bn * 128 <= 113 * 1024 - fixed;
     };
     while (BN > 16 && !fits(BN)) BN >>= 1;
     p.tiles_n = (p.N + BN - 1) / BN;
+    p.taps_per_b = tpb(BN);
   }
   if (fs >= 1) splits = std::min(fs, p.num_kb);
   p.kbs = (p.num_kb + splits - 1) / splits;
@@ -1115,10 +1164,10 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     d.owned = buf;
   }
   if (p.mode == 3) {
-    p.b_stage_bytes = p.S_ * BN * 128;
+    p.b_stage_bytes = p.taps_per_b * BN * 128;
     cuuint64_t db[3] = {(cuuint64_t)p.C, (cuuint64_t)p.N, (cuuint64_t)(p.R_ * p.S_)};
     cuuint64_t sb[2] = {(cuuint64_t)p.K * 2, (cuuint64_t)p.C * 2};
-    cuuint32_t bb[3] = {64, (cuuint32_t)BN, (cuuint32_t)p.S_};
+    cuuint32_t bb[3] = {64, (cuuint32_t)BN, (cuuint32_t)p.taps_per_b};
     if (!encode(&p.tmB, 3, W, db, sb, bb, 64, err)) return false;
   } else if (BK == 128) {
     if (p.K % 64) { err = "BK 128 needs K % 64 == 0"; return false; }
@@ -1215,7 +1264,8 @@ int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int ma
     // halo tiles: BH x BW with BW >= OW + 2; K blocks = 64-channel chunks
     const long long a_stage = (((128 / halo_bw) + 2) * halo_bw + 8) * 128;
     for (int bn = std::min(32, nmax); bn <= nmax && n < max; bn <<= 1) {
-      if ((a_stage + 1023) / 1024 * 1024 + 2 * 3 * bn * 128 > 113 * 1024 - (1024 + 256 + 2 * bn * 4)) break;
+      const int tpb = bn >= 128 ? 1 : 3;
+      if ((a_stage + 1023) / 1024 * 1024 + 2 * tpb * bn * 128 > 113 * 1024 - (1024 + 256 + 2 * bn * 4)) break;
       const long long tiles = halo_tiles_m * ((N + bn - 1) / bn);
       out[n++] = TcChoice{bn, 1, 64, 1};
       if (tiles < caps.S && chunks >= 2 && n < max) {

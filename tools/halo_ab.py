@@ -29,7 +29,7 @@ def main():
     for H, W, C, K in SHAPES:
         best = {}
         for halo in (0, 1):
-            cfgs = ["", "32,64,1", "64,64,1", "128,64,1", "32,64,2", "64,64,2", "32,64,4", "64,64,4", "64,128,1",
+            cfgs = ["", "128,64,4", "32,64,1", "64,64,1", "128,64,1", "32,64,2", "64,64,2", "128,64,2", "32,64,4", "64,64,4", "64,128,1",
                     "64,128,2"]
             for cfg in cfgs:
                 if halo and cfg.endswith(",128,1") or (halo and ",128," in cfg):

@@ -68,11 +68,12 @@ def main():
             L.bl_debug_tc_wait.argtypes = [C.c_void_p, C.c_int]
             L.bl_debug_tc_wait(wb.ctypes.data, 2048)
             wb = wb.astype(np.int64)
-            act = wb[:, 1] > 0
-            if act.any():
-                print(f"  MMA warp waiting for operands: {wb[act, 0].mean() / 1e3:.2f} us over "
-                      f"{wb[act, 1].mean():.1f} waits; producer waiting for free stages: "
-                      f"{wb[act, 2].mean() / 1e3:.2f} us over {wb[act, 3].mean():.1f} waits (per working CTA)")
+            on = wb[:, 1] > 0
+            if on.any():
+                print(f"  MMA warp waiting for operands: {wb[on, 0].mean() / 1e3:.2f} us over "
+                      f"{wb[on, 1].mean():.1f} waits; producer waiting for free stages: "
+                      f"{wb[on, 2].mean() / 1e3:.2f} us over {wb[on, 3].mean():.1f} waits (per working CTA, "
+                      "summed over the profile's launches)")
     ctx.close()
 
 
