@@ -490,7 +490,7 @@ def native(args):
         if not os.path.exists(tune):
             raise SystemExit(f"--load-profile needs its tuning file {tune}")
     else:
-        tune = os.path.join(args.out_dir, f"tctune_{args.config}_rank{rank}.txt")
+        tune = os.path.join(args.out_dir, f"tctune_{args.config}_gpu{rank}.txt")   # pairs with profile_*_gpu{g}
         if os.path.exists(tune):
             os.remove(tune)
     os.environ["BLESS_TC_TUNE_FILE"] = tune
