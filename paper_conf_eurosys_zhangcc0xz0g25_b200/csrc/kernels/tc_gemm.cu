@@ -1250,10 +1250,12 @@ int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int ma
     tiles_m = ((OW + BW - 1) / BW) * ((OH + (128 / BW) - 1) / (128 / BW));
     bk128_ok = st == 1 && (one ? C % 64 == 0 : C % 128 == 0);
     halo_ok = st == 1 && R == 3 && S == 3 && pad == 1 && C % 64 == 0 && OW + 2 <= 128;
-    long long hw = 8;
-    while (hw < OW + 2) hw <<= 1;
-    halo_tiles_m = (OH + (128 / hw) - 1) / (128 / hw);
-    halo_bw = hw;
+    if (halo_ok) {
+      long long hw = 8;
+      while (hw < OW + 2) hw <<= 1;
+      halo_tiles_m = (OH + (128 / hw) - 1) / (128 / hw);
+      halo_bw = hw;
+    }
     chunks = C / 64;
   } else {
     return 0;

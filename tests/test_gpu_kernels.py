@@ -97,6 +97,7 @@ CONVS = [  # H, W, C, K, k, stride, pad, act, residual
     (224, 224, 3, 64, 7, 2, 3, "relu", False),   # ResNet stem -> generic path
     (37, 37, 3, 24, 5, 2, 2, "relu", False),     # im2col: odd sizes, 5x5 stride 2, ragged pixel runs
     (17, 23, 4, 16, 3, 1, 1, "none", False),     # im2col: C = 4, non-square
+    (224, 224, 64, 64, 3, 1, 1, "relu", False),  # VGG16 conv1_2: too wide for a halo tile (OW + 2 > 128)
 ]
 
 
