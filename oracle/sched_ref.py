@@ -58,9 +58,12 @@ def static_ranges(quota_sms: Sequence[int]) -> List[Tuple[int, int]]:
 class Prof:
     """t[j][k][s] for s = 1..S, d[j][k], quota_sms, tau, T.
 
-    tau[j][k] = sum_{i<=k} t[j][i][quota_sms_j]  ("the duration from the
-    beginning of the application to the end of k" with n% SMs, L157);
-    T[j] = tau[j][m_j - 1] ("isolated latency T[n%]", L157).
+    tau[j][k] = "the duration from the beginning of the application to the
+    end of k" with n% SMs (L157): measured along an isolated run of the
+    request when the profile carries it for the tenant's quota SMs (reading
+    R35: a "tau <sms> ..." line with sms == quota_sms), else
+    sum_{i<=k} t[j][i][quota_sms_j};  T[j] = tau[j][m_j - 1] ("isolated
+    latency T[n%]", L157).
     """
 
     def __init__(self, pf: ProfileFile):
@@ -74,7 +77,11 @@ class Prof:
         self.d = [[k.d for k in tn.kernels] for tn in pf.tenants]
         self._t = [[list(k.t) for k in tn.kernels] for tn in pf.tenants]
         self.tau: List[List[int]] = []
-        for j in range(self.ntenants):
+        for j, tn in enumerate(pf.tenants):
+            measured = list(getattr(tn, "tau", []) or [])
+            if measured and len(measured) == self.m[j] and getattr(tn, "tau_sms", 0) == self.quota_sms[j]:
+                self.tau.append(measured)          # R35: measured along an isolated run
+                continue
             acc, row = 0, []
             for k in range(self.m[j]):
                 acc += self.t(j, k, self.quota_sms[j])

@@ -217,6 +217,49 @@ bl_status Engine::profile_tenant(int t, int reps, std::string& err) {
     }
   }
   prof_.derive();
+  // tau[n%][k] and T[n%] (L157, reading R35): "the duration from the
+  // beginning of the application to the end of k", measured along isolated
+  // runs of the whole request on the tenant's quota SMs, launched exactly as
+  // the engine launches a request (programmatic dependent launch, light exits
+  // for the middle kernels); element-wise median over the runs
+  TenantProfile& tp = prof_.ten[t];
+  const int q = tp.quota_sms;
+  const int m = (int)ten_[t].handles.size();
+  if (q >= 1 && m > 0) {
+    rt_->set_device();
+    const int runs = std::max(3, reps);
+    std::vector<std::vector<int64_t>> tau(m);
+    for (int r = 0; r < runs + 1; ++r) {   // run 0 warms up
+      if (!rt_->device_sync()) { err = "device error before the tau run"; return BL_E_CUDA; }
+      std::vector<uint64_t> seqs(m);
+      uint64_t prev_light = 0;
+      for (int k = 0; k < m; ++k) {
+        const bool stamp = k == 0 || k == m - 1;
+        seqs[k] = rt_->alloc_seq();
+        if (!rt_->launch_seq(ten_[t].handles[k], seqs[k], 0, q, ten_[t].stream, err, stamp, prev_light))
+          return BL_E_CUDA;
+        prev_light = stamp ? 0 : seqs[k];
+      }
+      if (!rt_->device_sync()) { err = "device error in the tau run"; return BL_E_CUDA; }
+      if (r == 0) continue;
+      rt_->refresh_sync(seqs.front(), seqs.back());
+      LaunchStats s0{};
+      rt_->peek(seqs[0], &s0);
+      for (int k = 0; k < m; ++k) {
+        LaunchStats st{};
+        rt_->peek(seqs[k], &st);
+        tau[k].push_back(std::max<int64_t>(1, st.end_host - s0.start_host));
+      }
+    }
+    tp.tau_meas.assign(m, 0);
+    for (int k = 0; k < m; ++k) {
+      std::sort(tau[k].begin(), tau[k].end());
+      tp.tau_meas[k] = tau[k][tau[k].size() / 2];
+      if (k && tp.tau_meas[k] < tp.tau_meas[k - 1]) tp.tau_meas[k] = tp.tau_meas[k - 1];   // medians of a monotone chain
+    }
+    tp.tau_sms = q;
+    prof_.derive();
+  }
   return BL_OK;
 }
 
@@ -277,6 +320,8 @@ bl_status Engine::load_profile(const char* path, std::string& err) {
       prof_.ten[j].io_in = p.ten[j].io_in;
       prof_.ten[j].io_out = p.ten[j].io_out;
     }
+    prof_.ten[j].tau_sms = p.ten[j].tau_sms;
+    prof_.ten[j].tau_meas = p.ten[j].tau_meas;
     for (size_t k = 0; k < p.ten[j].k.size(); ++k) {
       prof_.ten[j].k[k].t = p.ten[j].k[k].t;
       prof_.ten[j].k[k].d = p.ten[j].k[k].d;

@@ -47,6 +47,10 @@ void Profile::derive() {
       if ((int)tn.k[k].t.size() == S && tn.quota_sms >= 1) acc += tn.k[k].t[tn.quota_sms - 1];
       tn.tau[k] = acc;
     }
+    if (!tn.tau_meas.empty() && tn.tau_meas.size() == tn.k.size() && tn.tau_sms == tn.quota_sms) {
+      tn.tau = tn.tau_meas;   // R35: measured along an isolated run at the quota
+      acc = tn.tau.back();
+    }
     tn.T = acc;
     tn.tau_prog = tn.tau;
     if (tn.slo_ns > 0 && tn.T > 0)
@@ -89,6 +93,13 @@ bool load_profile_text(const std::string& path, Profile& out, std::string& err) 
       } else if (a == "io") {
         f >> tn.io_in >> tn.io_out;
         if (!f || tn.io_in < 0 || tn.io_out < 0) { err = "bad io line"; return false; }
+      } else if (a == "tau") {   // measured progress (R35): tau <sms> <tau_0> .. <tau_{m-1}>
+        f >> tn.tau_sms;
+        tn.tau_meas.resize(m);
+        for (int k = 0; k < m; ++k) f >> tn.tau_meas[k];
+        if (!f || tn.tau_sms < 1) { err = "bad tau line"; return false; }
+        for (int k = 0; k < m; ++k)
+          if (tn.tau_meas[k] < 0 || (k && tn.tau_meas[k] < tn.tau_meas[k - 1])) { err = "tau not monotone"; return false; }
       } else {
         f.seekg(pos);
         break;
@@ -118,6 +129,11 @@ bool save_profile_text(const std::string& path, const Profile& p, std::string& e
     f << "tenant " << tn.name << " " << tn.quota_ppm << " " << tn.k.size() << "\n";
     if (tn.slo_ns > 0) f << "slo " << tn.slo_ns << "\n";
     if (tn.io_in > 0 || tn.io_out > 0) f << "io " << tn.io_in << " " << tn.io_out << "\n";
+    if (!tn.tau_meas.empty()) {
+      f << "tau " << tn.tau_sms;
+      for (int64_t v : tn.tau_meas) f << " " << v;
+      f << "\n";
+    }
     for (auto& k : tn.k) {
       f << "kernel " << k.name << " " << k.d;
       for (int64_t v : k.t) f << " " << v;

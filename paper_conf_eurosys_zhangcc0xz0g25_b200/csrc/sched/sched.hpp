@@ -45,6 +45,14 @@ struct TenantProfile {
   // picks include kernel 0 / the last kernel; Eq. 2 adds them to the level of
   // that kernel.  0 = no per-request host I/O.
   int64_t io_in = 0, io_out = 0;
+  // Measured progress (reading R35): tau[n%][k] is "the
+  // duration from the beginning of the application to the end of k" and
+  // T[n%] its "isolated latency" -- measured along an isolated run of the
+  // whole request on tau_sms SMs.  When tau_sms equals the tenant's quota
+  // SMs, derive() takes tau (and T = tau.back()) from here instead of the
+  // prefix sums of the per-kernel t[k][quota_sms].  Empty = not measured.
+  int tau_sms = 0;
+  std::vector<int64_t> tau_meas;
 };
 
 struct Profile {

@@ -9,6 +9,7 @@ both the C++ runtime ``bl_load_profile`` and the Python oracle)::
     tenant <name> <quota_ppm> <m>
     slo <ns>                                     (optional: SLO mode target)
     io <in_ns> <out_ns>                          (optional: per-request H2D / D2H copy time)
+    tau <sms> <tau_0> ... <tau_{m-1}>            (optional: measured progress, reading R35)
     kernel <name> <d> <t_1> <t_2> ... <t_S>      (m lines per tenant)
 
 ``t_s`` is the kernel's duration in integer ns when confined to s SMs
@@ -46,6 +47,8 @@ class TenantRows:
     slo_ns: int = 0   # optional "slo <ns>" line (SLO mode); 0 = none
     io_in: int = 0    # optional "io <in_ns> <out_ns>" line: per-request H2D / D2H copy durations
     io_out: int = 0
+    tau_sms: int = 0  # optional "tau <sms> <tau_0..tau_{m-1}>" line: time from the start of an isolated
+    tau: List[int] = field(default_factory=list)   # run on tau_sms SMs to the end of kernel k (R35)
 
 
 @dataclass
@@ -63,6 +66,8 @@ def save(path: str, pf: ProfileFile) -> None:
             lines.append(f"slo {int(tn.slo_ns)}")
         if tn.io_in or tn.io_out:
             lines.append(f"io {int(tn.io_in)} {int(tn.io_out)}")
+        if tn.tau:
+            lines.append("tau %d %s" % (int(tn.tau_sms), " ".join(str(int(v)) for v in tn.tau)))
         for k in tn.kernels:
             assert len(k.t) == pf.S, (len(k.t), pf.S)
             lines.append("kernel %s %d %s" % (k.name, int(k.d), " ".join(str(int(v)) for v in k.t)))
@@ -82,11 +87,14 @@ def load(path: str) -> ProfileFile:
         _, name, ppm, m = toks[i]
         i += 1
         tn = TenantRows(name, int(ppm))
-        while i < len(toks) and toks[i][0] in ("slo", "io"):
+        while i < len(toks) and toks[i][0] in ("slo", "io", "tau"):
             if toks[i][0] == "slo":
                 tn.slo_ns = int(toks[i][1])
-            else:
+            elif toks[i][0] == "io":
                 tn.io_in, tn.io_out = int(toks[i][1]), int(toks[i][2])
+            else:
+                tn.tau_sms = int(toks[i][1])
+                tn.tau = [int(v) for v in toks[i][2:2 + int(m)]]
             i += 1
         for _ in range(int(m)):
             row = toks[i]

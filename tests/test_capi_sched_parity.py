@@ -261,3 +261,40 @@ def test_predict_matches_oracle_eq1_eq2(tmp_path_factory, w, pseed):
     ns, npk = ctx.time_decide([rec], reps=2)
     assert ns > 0 and npk == 2 * len(picks)
     ctx.close()
+
+
+@settings(max_examples=120, deadline=None)
+@given(world(), st.integers(0, 10_000), st.booleans())
+def test_measured_tau_bit_exact(tmp_path_factory, w, seed, match):
+    """Reading R35 (tau[n%][k] is "the duration from the
+    beginning of the application to the end of k", T[n%] its isolated
+    latency): a profile carrying a measured "tau" line per tenant.  With
+    tau_sms == quota SMs both sides use it for the progress order and T;
+    with another SM count both fall back to the prefix sums.  Decisions stay
+    bit-exact, the C++ writer round-trips the line."""
+    from synth.profile import load, save
+    pf, active, now, params = w
+    prof0 = Prof(pf)
+    rng = np.random.Generator(np.random.PCG64(seed))
+    for j, tn in enumerate(pf.tenants):
+        steps = rng.integers(1, 500, size=len(tn.kernels))
+        tn.tau = [int(v) for v in np.cumsum(steps)]
+        tn.tau_sms = prof0.quota_sms[j] if match else prof0.quota_sms[j] + 1
+    d = tmp_path_factory.mktemp("tau")
+    path = str(d / "p.txt")
+    save(path, pf)
+    prof = Prof(load(path))
+    for j, tn in enumerate(pf.tenants):
+        want = tn.tau if match else prof0.tau[j]
+        assert prof.tau[j] == want and prof.T[j] == want[-1]
+    ctx = capi.Ctx(capi.BL_DEVICE_NONE, clock=capi.BL_CLOCK_VIRTUAL, **params)
+    ctx.load_profile(path)
+    for j in range(len(pf.tenants)):
+        assert ctx.tenant_info(j)[2] == prof.T[j]
+    got = _cpp_tuple(ctx.decide(now, active))
+    ref = decide_ref(now, [Active(*a) for a in active], prof, Params(**params))
+    assert got == _ref_tuple(ref)
+    out = str(d / "rt.txt")
+    ctx.save_profile(out)
+    assert open(out).read() == open(path).read()
+    ctx.close()
