@@ -222,10 +222,15 @@ bl_status Engine::profile_tenant(int t, int reps, std::string& err) {
   // runs of the whole request on the tenant's quota SMs, launched exactly as
   // the engine launches a request (programmatic dependent launch, light exits
   // for the middle kernels); element-wise median over the runs
+  // Opt-in (BLESS_MEASURED_TAU=1): on B200 the measured chains are shorter
+  // than the per-kernel prefix sums (R50 at 99 SMs: 0.44 vs 0.51 ms) and the
+  // C2 bench got 5% slower with them (profiles/round2/bench/), so the default
+  // keeps the round-1 prefix sums.
   TenantProfile& tp = prof_.ten[t];
   const int q = tp.quota_sms;
   const int m = (int)ten_[t].handles.size();
-  if (q >= 1 && m > 0) {
+  const char* mt = std::getenv("BLESS_MEASURED_TAU");
+  if (mt && std::atoi(mt) != 0 && q >= 1 && m > 0) {
     rt_->set_device();
     const int runs = std::max(3, reps);
     std::vector<std::vector<int64_t>> tau(m);
