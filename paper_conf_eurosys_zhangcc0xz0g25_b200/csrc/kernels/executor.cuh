@@ -74,6 +74,7 @@ struct GateArgs {
   uint32_t tiles;
   int32_t lo, hi;
   uint32_t stamp;          // 1: full exit protocol (last CTA publishes end + seq); 0: light exit
+  uint32_t linger_ns;      // bounded wait of out-of-range CTAs (default 30 us; BLESS_LINGER_NS, tests)
 };
 
 #ifdef __CUDACC__
@@ -167,7 +168,7 @@ __device__ __forceinline__ void gate_tile_loop(const GateArgs& g, Body&& body) {
 // when the bounded wait expires (e.g. two tenants' lingering CTAs blocking
 // each other's windows), the CTA returns true and helps drain the queue (a
 // bounded, flagged confinement violation instead of a stalled kernel).
-constexpr uint64_t kLingerNs = 30000;
+constexpr uint64_t kLingerNs = 30000;   // default GateArgs::linger_ns
 __device__ __forceinline__ bool gate_linger(const GateArgs& g) {
   __shared__ int s_steal;
   if (threadIdx.x == 0) {
@@ -178,7 +179,7 @@ __device__ __forceinline__ bool gate_linger(const GateArgs& g) {
       for (;;) {
         const unsigned long long c = *reinterpret_cast<volatile unsigned long long*>(&g.slot->ctr);
         if ((uint32_t)c != 0u) break;
-        if (ptx_globaltimer() - t0 > kLingerNs) {
+        if (ptx_globaltimer() - t0 > g.linger_ns) {
           steal = 1;
           break;
         }

@@ -142,6 +142,8 @@ std::unique_ptr<DeviceRT> DeviceRT::create(int device, void* ws, size_t ws_bytes
     return nullptr;
   }
   if (const char* e = std::getenv("BLESS_PDL")) g_use_pdl = std::atoi(e) != 0;
+  rt->linger_ns_ = (uint32_t)kLingerNs;
+  if (const char* e = std::getenv("BLESS_LINGER_NS")) rt->linger_ns_ = (uint32_t)std::max(0, std::atoi(e));
   if (const char* e = std::getenv("BLESS_TC_AUTOTUNE")) rt->autotune_ = std::atoi(e) != 0;
   if (const char* e = std::getenv("BLESS_TC_TUNE_FILE")) {   // "sig bn splits" lines, appended as tuned
     rt->tune_file_ = e;
@@ -380,6 +382,7 @@ GateArgs DeviceRT::make_gate(uint64_t seq, uint32_t tiles, int lo, int hi, bool 
   g.lo = lo;
   g.hi = hi;
   g.stamp = stamp ? 1u : 0u;
+  g.linger_ns = linger_ns_;
   return g;
 }
 

@@ -111,6 +111,7 @@ class DeviceRT {
   uint8_t* lid_map_dev_ = nullptr;
   bool identity_map_ = true;
   uint64_t seq_ = 0;
+  uint32_t linger_ns_ = 30000;   // GateArgs::linger_ns (BLESS_LINGER_NS)
   uint64_t ring_ = kSlotRingDefault;
   uint64_t ahead_ = kSlotRingDefault / 2;
   std::vector<std::unique_ptr<KernelDesc>> kernels_;

@@ -197,3 +197,34 @@ def test_baselines_complete(lib_built, policy):
     for r in ids:
         assert ctx.poll(r)[0] == capi.BL_OK
     ctx.close()
+
+
+def test_linger_steal_path_exact(lib_built, monkeypatch):
+    """Executor safety net (executor.cuh gate_linger): an out-of-range CTA that
+    sees no in-range claim within linger_ns helps drain the queue (flag bit 1,
+    a bounded confinement violation instead of a stall).  With linger 0 the
+    path runs on almost every restricted launch: every request still
+    completes, every layer matches the oracle, and the steal is reported."""
+    monkeypatch.setenv("BLESS_LINGER_NS", "0")
+    ctx = capi.Ctx(0, policy="STATIC")
+    S = ctx.device_info().sm_count
+    ms = models.build_config(ctx, "C1", "fp32")
+    for m in ms:
+        for k in range(len(m.layers)):
+            ctx.set_profile_row(m.tenant, k, [max(2000, 300000 // s) for s in range(1, S + 1)], S)
+    ctx.start()
+    base = capi.now_ns() + 1_000_000
+    ids = [ctx.submit(j, base + i * 50_000) for i in range(4) for j in range(2)]
+    ctx.drain(int(20e9))
+    ctx.stop()
+    for r in ids:
+        assert ctx.poll(r)[0] == capi.BL_OK
+    recs = ctx.launches()
+    steals = sum(1 for r in recs if r.fallback & 2)
+    assert steals > 0, "linger 0 should exercise the steal path"
+    for m in ms:
+        for k, layer in enumerate(m.layers):
+            err, tol = check_layer(layer, "fp32")
+            assert err <= tol, (m.name, k, err)
+    print(f"\nsteal path: {steals}/{len(recs)} launches helped by out-of-range CTAs, outputs exact")
+    ctx.close()

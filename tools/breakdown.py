@@ -23,6 +23,9 @@ def main():
     ap.add_argument("--requests", type=int, default=100)
     ap.add_argument("--squad-max", type=int, default=20)
     ap.add_argument("--split-pct", type=int, default=25)
+    ap.add_argument("--max-inflight", type=int, default=2)
+    ap.add_argument("--lookahead-us", type=float, default=20.0)
+    ap.add_argument("--policies", default="BLESS,ISO,STATIC,UNBOUND")
     a = ap.parse_args()
     from paper_conf_eurosys_zhangcc0xz0g25_b200 import build, capi, models
     from synth import trace as tr
@@ -35,10 +38,11 @@ def main():
     out = {}
     for seed in (1, 2, 3):
         trace = tr.poisson([t / a.rho for t in T], a.requests, seed=seed)
-        for pol in ("BLESS", "ISO", "STATIC", "UNBOUND"):
+        for pol in a.policies.split(","):
             filts = [{j} for j in range(len(ms))] if pol == "ISO" else [None]
             for filt in filts:
-                p = capi.default_params(policy=pol, squad_max=a.squad_max, split_pct=a.split_pct)
+                p = capi.default_params(policy=pol, squad_max=a.squad_max, split_pct=a.split_pct,
+                                        max_inflight_squads=a.max_inflight, lookahead_ns=int(a.lookahead_us * 1000))
                 ctx.reset(p)
                 ctx.start()
                 ents = [(0, x.tenant, x.arrival_ns) for x in trace if filt is None or x.tenant in filt]
