@@ -385,6 +385,29 @@ def roofline_of(rep, launches_all, peaks, args):
             "top_layers": [{"layer": nm, "event_ns": round(ev), "roofline_time_frac": round(fr, 3)}
                            for _, nm, ev, fr in per_layer[:5]],
             "peak_source": peak_src}
+    # the same family at the SM range its launches actually got in the timed
+    # BLESS steps (median hi - lo per layer), against the SM-share peak
+    # P * s/S ("against the chip's peak scaled by the tenant's
+    # SM share")
+    rng = {}
+    for r in launches_all:
+        if r.end_ns > r.start_ns and r.nsm > 0 and fam_of.get((r.tenant, r.kernel)) == fam:
+            rng.setdefault((r.tenant, r.kernel), []).append(r.hi - r.lo)
+    Fr = Tr = Pr = 0.0
+    for tk, sizes in rng.items():
+        s_med = int(np.median(sizes))
+        ki = ctx.kernel_info(*tk)
+        ev, _ = ctx.profile_kernel(tk[0], tk[1], s_med, reps=10)
+        n = nlaunch[tk]
+        Fr += n * ki.flops
+        Tr += n * ev
+        Pr += n * ev * (tc_peak * s_med / S)   # time-weighted share of the peak
+    if Tr > 0:
+        peak_share = Pr / Tr
+        roof["at_range"] = {"achieved": Fr / Tr / 1e3, "peak_share": peak_share, "unit": "TFLOP/s",
+                            "frac": Fr / Tr / 1e3 / peak_share,
+                            "note": "each layer timed on its median SM range in the timed steps; peak = "
+                                    "measured bf16 peak x s/S, time-weighted"}
     hb = [tk for tk in busy if (lambda k: k.flops / max(k.bytes, 1.0) < ridge)(ctx.kernel_info(*tk))]
     if hb:
         tk = max(hb, key=lambda x: busy[x] / nlaunch[x])
