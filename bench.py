@@ -790,6 +790,16 @@ def native(args):
         "other_configs": others or None,
         "device": {"sm_count": r0.S, "globaltimer_res_ns": r0.info.globaltimer_res_ns, "host_cores": os.cpu_count()},
     }
+    # compact summary again at the END of the line (a truncated tail keeps it)
+    out["summary"] = {"value_ms": mean_ms, "min_attainment_pct": out["min_attainment_pct"],
+                      "attainment_pct": {k: v.get("attainment_pct") for k, v in per_tenant.items()},
+                      "mean_ms": {"BLESS": mean_ms, **bmean}, "vs_static": out["vs_static"],
+                      "vs_temporal_twc": out["vs_temporal_twc"], "vs_temporal_tcap": out["vs_temporal_tcap"],
+                      "vs_unbound": out["vs_unbound"], "deviation_ms": out["deviation_ms"],
+                      "roofline_frac": roofline["frac"], "replay": replay_ok,
+                      "other_configs": {c: {rho: {"BLESS": x["mean_ms"]["BLESS"], "STATIC": x["mean_ms"]["STATIC"],
+                                                  "min_attainment_pct": x["min_attainment_pct"]}
+                                            for rho, x in o["rho"].items()} for c, o in others.items()}}
     if rank == 0:
         print(json.dumps(out))
     for r in reps:
