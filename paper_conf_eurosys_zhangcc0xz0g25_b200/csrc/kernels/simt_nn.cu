@@ -4,8 +4,9 @@
 // (MobileNetV2), strided per-channel affine + activation (DenseNet BN-ReLU on
 // a channel slice of the concat buffer).  bf16 storage, fp32 math; semantics
 // as oracle/layers_ref.py.  None of these is a dense contraction worth the
-// tensor cores at the configs' sizes except attention, whose tcgen05 version
-// is future work.
+// tensor cores at the configs' sizes except attention: L % 128 == 0 runs on
+// the fused tcgen05 kernel (attn_tc.cu); the CUDA-core attention here covers
+// the other sequence lengths (and BLESS_ATTN_SIMT=1).
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 

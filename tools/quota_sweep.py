@@ -20,7 +20,7 @@ BIASED = ((1 / 9, 8 / 9), (0.9, 0.2))
 
 
 def run(quotas, rhos, steps):
-    args = [sys.executable, os.path.join(ROOT, "bench.py"), "--config", "C2", "--no-cpu-baseline", "--no-slo",
+    args = [sys.executable, os.path.join(ROOT, "bench.py"), "--config", "C2", "--no-cpu-baseline", "--no-slo", "--also", "",
             "--steps", str(steps), "--warmup", "3", "--quotas", ",".join(f"{q:.6f}" for q in quotas)]
     if rhos:
         args += ["--rhos", ",".join(str(r) for r in rhos)]
