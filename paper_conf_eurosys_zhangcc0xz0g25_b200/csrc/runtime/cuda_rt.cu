@@ -258,9 +258,23 @@ bool DeviceRT::calibrate_clock(std::string& err) {
   return true;
 }
 
+// Shared-memory carveout of every tenant kernel (BLESS_CARVEOUT = percent of
+// the unified L1/shared array given to shared memory; unset = driver default).
+// One carveout for all kernels means an SM never has to drain and
+// reconfigure L1/shared between a tcgen05 kernel (~100 KB of shared memory)
+// and a SIMT kernel (a few KB) of the same or another tenant.
+static void apply_carveout(const void* fn) {
+  static const int pct = [] {
+    const char* e = std::getenv("BLESS_CARVEOUT");
+    return e ? std::atoi(e) : -1;
+  }();
+  if (fn && pct >= 0 && pct <= 100) cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
+}
+
 int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
   std::unique_ptr<KernelDesc> kd(new KernelDesc());
   if (!build_kernel(op, caps_, *kd, err)) return -1;
+  apply_carveout(kd->kernel_fn);
   // grid = S x (resident blocks per SM): see gate_linger in executor.cuh
   if (kd->kernel_fn) {
     kd->grid = full_occupancy_grid(kd->kernel_fn, kd->block, (size_t)kd->smem, caps_.S, kd->max_occ);
@@ -295,6 +309,7 @@ int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
       }
     }
   }
+  apply_carveout(kd->kernel_fn);
   kernels_.push_back(std::move(kd));
   return (int)kernels_.size() - 1;
 }
