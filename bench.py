@@ -74,6 +74,8 @@ def parse():
     ap.add_argument("--squad-max", type=int, default=None,
                     help="S_max (L406-L408); default per config from the B200 sweeps: C1 4, C2 20, C3 10, C4 10")
     ap.add_argument("--split-pct", type=int, default=25)
+    ap.add_argument("--squad-max-solo", type=int, default=0,
+                    help="reading R36: cap of a squad with a single active request (0 = S_max)")
     ap.add_argument("--ablate", type=int, default=0,
                     help="PAPER.md §6.8 ablation (R32): 1 = no multi-task scheduler, 2 = no determiner, 3 = both")
     ap.add_argument("--lookahead-us", type=float, default=20.0)
@@ -238,7 +240,8 @@ class Replica:
 
     def params(self, capi, args, pol="BLESS", extra=None):
         return capi.default_params(squad_max=self.squad_max, policy=pol, split_pct=args.split_pct,
-                                   ablate=args.ablate, lookahead_ns=int(args.lookahead_us * 1000),
+                                   ablate=args.ablate, squad_max_solo=args.squad_max_solo,
+                                   lookahead_ns=int(args.lookahead_us * 1000),
                                    max_inflight_squads=args.max_inflight, **(extra or {}))
 
 
@@ -726,7 +729,8 @@ def native(args):
     if rank == 0:
         from oracle.sched_ref import Params, Prof
         r0 = reps[0]
-        prm = Params(squad_max=r0.squad_max, split_pct=args.split_pct, ablate=args.ablate)
+        prm = Params(squad_max=r0.squad_max, split_pct=args.split_pct, ablate=args.ablate,
+                     squad_max_solo=args.squad_max_solo)
         replay_ok = replay_all(dec, r0.prof_path, prm)
         if world == 1 and nrep == 1 and not args.no_cpu_baseline:
             prof = Prof(synprof.load(r0.prof_path))
@@ -766,7 +770,7 @@ def native(args):
                    "trace": f"{'MMPP-2 bursty' if args.config == 'C4' else 'Poisson'} rho={args.rhos or args.rho} "
                    f"per tenant, {args.requests} requests/tenant/step, seeds 1-3, box-wide trace routed by the "
                    "native dispatcher (bl_dispatch)", "squad_max": r0.squad_max,
-                   "split_pct": args.split_pct, "ablate": args.ablate,
+                   "split_pct": args.split_pct, "ablate": args.ablate, "squad_max_solo": args.squad_max_solo,
                    "parallelism": f"replicas x{n_box} (no collective; "
                                   f"{'one process per GPU, gloo host barrier' if world > 1 else 'one process'})",
                    "quotas": [m.quota for m in r0.tms],

@@ -108,6 +108,12 @@ typedef struct {
                                  SMs [0, sm_limit) for the run, the way the paper restricts
                                  the GPU with MIG.  BL_E_INVALID at bl_start unless
                                  g <= sm_limit <= S. */
+  int32_t squad_max_solo;     /* reading R36 (L57/L121: a request arriving while another
+                                 runs alone should get its SMs "instantly"): a squad with a
+                                 single active request closes after min(squad_max,
+                                 squad_max_solo) kernels, bounding how long an arrival
+                                 waits for the next decision; 0 = squad_max (default). */
+  int32_t reserved1;          /* 0 */
 } bl_params;
 
 /* Fill *p with the defaults listed above. */

@@ -126,11 +126,17 @@ class Params:
     # one kernel each per round, no progress ordering); bit 1 = no execution
     # configuration determiner (no search: every squad runs NSP on [0, S)).
     ablate: int = 0
+    # Reading R36: a squad with a single active request closes after
+    # min(squad_max, squad_max_solo) kernels (L57 / L121: an arriving request
+    # should get its share "instantly"; squads are waited for lazily, so a
+    # short solo squad bounds the wait).  0 = squad_max.
+    squad_max_solo: int = 0
 
     @staticmethod
     def from_dict(d: dict) -> "Params":
         return Params(int(d.get("squad_max", 50)), int(d.get("split_pct", 50)),
-                      bool(d.get("seed_all", True)), int(d.get("squad_overhead_ns", 0)), int(d.get("ablate", 0)))
+                      bool(d.get("seed_all", True)), int(d.get("squad_overhead_ns", 0)), int(d.get("ablate", 0)),
+                      int(d.get("squad_max_solo", 0)))
 
 
 @dataclass(frozen=True)
@@ -189,6 +195,9 @@ def generate_squad(now: int, active: Sequence[Active], prof: Prof, params: Param
         return behind_key(now, j, arr[j], tau_done(j))
 
     picks: List[Tuple[int, int]] = []
+    cap = params.squad_max
+    if len(active) == 1 and params.squad_max_solo > 0:     # R36
+        cap = min(params.squad_max, params.squad_max_solo)
 
     def pick(j: int) -> bool:
         """Append kernel nxt_j of request j; True when the squad must close:
@@ -197,7 +206,7 @@ def generate_squad(now: int, active: Sequence[Active], prof: Prof, params: Param
         k = nxt[j]
         picks.append((j, k))
         nxt[j] = k + 1
-        return len(picks) >= params.squad_max or k == prof.m[j] - 1
+        return len(picks) >= cap or k == prof.m[j] - 1
 
     closed = False
     tenants = sorted(nxt)

@@ -41,7 +41,8 @@ class bl_params(C.Structure):
                 ("squad_overhead_ns", C.c_int64), ("temporal_period_ns", C.c_int64),
                 ("temporal_work_conserving", C.c_int32), ("max_inflight_squads", C.c_int32),
                 ("lookahead_ns", C.c_int64), ("max_requests", C.c_int64),
-                ("ablate", C.c_int32), ("sm_limit", C.c_int32)]
+                ("ablate", C.c_int32), ("sm_limit", C.c_int32),
+                ("squad_max_solo", C.c_int32), ("reserved1", C.c_int32)]
 
 
 class bl_op(C.Structure):

@@ -55,6 +55,7 @@ void bl_params_default(bl_params* p) {
   p->max_inflight_squads = 2;
   p->lookahead_ns = 20000;
   p->max_requests = 1 << 20;
+  p->squad_max_solo = 0;
 }
 
 bl_status bl_create(int device, const bl_params* params, void* ws, size_t ws_bytes, bl_ctx** out) {

@@ -42,7 +42,7 @@ Engine::~Engine() {
 
 bl_status Engine::init(void* ws, size_t ws_bytes, std::string& err) {
   if (prm_.sm_unit < 1 || prm_.squad_max < 1 || prm_.squad_max > BL_MAX_SQUAD || prm_.split_pct < 0 ||
-      prm_.ablate < 0 || prm_.ablate > 3 ||
+      prm_.ablate < 0 || prm_.ablate > 3 || prm_.squad_max_solo < 0 || prm_.squad_max_solo > BL_MAX_SQUAD ||
       prm_.split_pct > 100 || prm_.max_requests < 1) {
     err = "invalid bl_params";
     return BL_E_INVALID;
@@ -588,7 +588,7 @@ bl_status Engine::time_decide(const bl_decision* recs, size_t n, int reps, int64
       in[r].push_back({t, d.act_arrival[i], d.act_next[i]});
     }
   }
-  SchedParams sp{prm_.squad_max, prm_.split_pct, prm_.seed_all != 0, prm_.ablate};
+  SchedParams sp{prm_.squad_max, prm_.split_pct, prm_.seed_all != 0, prm_.ablate, prm_.squad_max_solo};
   Decision d;
   DecideScratch sc;
   int64_t np = 0;
@@ -661,7 +661,7 @@ bl_status Engine::decide_pure(int64_t now, int n, const int32_t* ten, const int6
     }
     a[i] = {ten[i], arr[i], nxt[i]};
   }
-  SchedParams sp{prm_.squad_max, prm_.split_pct, prm_.seed_all != 0, prm_.ablate};
+  SchedParams sp{prm_.squad_max, prm_.split_pct, prm_.seed_all != 0, prm_.ablate, prm_.squad_max_solo};
   Decision d;
   DecideScratch sc;
   decide(now, a.data(), n, prof_, sp, d, sc);
@@ -1093,7 +1093,7 @@ void Engine::loop_bless() {
   std::vector<int64_t> act_req(nt, -1);
   std::vector<int> act_next(nt, 0);
   std::vector<ActiveReq> av;
-  SchedParams sp{prm_.squad_max, prm_.split_pct, prm_.seed_all != 0, prm_.ablate};
+  SchedParams sp{prm_.squad_max, prm_.split_pct, prm_.seed_all != 0, prm_.ablate, prm_.squad_max_solo};
   int64_t vnow = 0;   // VIRTUAL clock
   int64_t E = 0;      // WALL: predicted end of the last launched squad
   const size_t max_inflight = (size_t)std::max(1, prm_.max_inflight_squads);

@@ -202,12 +202,16 @@ void decide(int64_t now, const ActiveReq* act, int n_act, const Profile& prof, c
   tenants.clear();
   for (auto& a : out.active) tenants.push_back(a.tenant);
 
+  // R36: a squad of a single active request closes after squad_max_solo
+  // kernels (an arrival then waits at most that long for the next decision)
+  const int cap = (out.active.size() == 1 && prm.squad_max_solo > 0) ? std::min(prm.squad_max, prm.squad_max_solo)
+                                                                       : prm.squad_max;
   // §4.3.2 squad generation (L181-L187).
   auto pick = [&](int j) -> bool {
     const int k = sc.nxt[j];
     out.picks.push_back({j, k, 0, S});
     sc.nxt[j] = k + 1;
-    return (int)out.picks.size() >= prm.squad_max || k == (int)prof.ten[j].k.size() - 1;  // R5, R7
+    return (int)out.picks.size() >= cap || k == (int)prof.ten[j].k.size() - 1;  // R5 / R36, R7
   };
   bool closed = false;
   if (prm.ablate & 1) {

@@ -71,6 +71,7 @@ struct SchedParams {
   int split_pct = 50;   // R16
   bool seed_all = true; // R6
   int ablate = 0;       // §6.8 ablation (R32): bit0 no multi-task scheduler, bit1 no determiner
+  int squad_max_solo = 0;  // R36: cap of a squad with ONE active request (0 = squad_max)
 };
 
 struct ActiveReq {

@@ -120,7 +120,8 @@ def world(draw):
     active = [(j, draw(st.integers(0, 300)), draw(st.integers(0, m[j] - 1))) for j in who]
     now = draw(st.integers(0, 1500))
     params = dict(squad_max=draw(st.integers(1, 12)), split_pct=draw(st.sampled_from([0, 30, 50, 75, 100])),
-                  seed_all=int(draw(st.booleans())), ablate=draw(st.sampled_from([0, 0, 1, 2, 3])))
+                  seed_all=int(draw(st.booleans())), ablate=draw(st.sampled_from([0, 0, 1, 2, 3])),
+                  squad_max_solo=draw(st.sampled_from([0, 0, 1, 2, 5])))
     return pf, active, now, params
 
 
@@ -132,7 +133,7 @@ def test_decide_bit_exact_small(tmp_path_factory, w):
     ctx = _ctx_from(pf, tmp, **params)
     ref = decide_ref(now, [Active(*a) for a in active], Prof(pf),
                      Params(params["squad_max"], params["split_pct"], bool(params["seed_all"]),
-                            ablate=params["ablate"]))
+                            ablate=params["ablate"], squad_max_solo=params["squad_max_solo"]))
     assert _cpp_tuple(ctx.decide(now, active)) == _ref_tuple(ref)
     ctx.close()
 

@@ -365,3 +365,22 @@ def test_ablation_without_determiner_is_nsp():
     picks = [tuple(p) for p in fx["picks_order"]]
     assert all((lo, hi) == (0, prof.S) for _, _, lo, hi in semi_sp_ranges(picks, sorted(ks), config, prof,
                                                                             fx["split_pct"]))
+
+
+def test_r36_solo_squad_cap_hand_worked():
+    """Reading R36: with ONE active request the squad closes after
+    min(S_max, squad_max_solo) kernels; with two active requests the solo cap
+    does not apply.  Fixture E3's tables (t = 100 / 200 per kernel at quota,
+    4 kernels each, both arriving at 0)."""
+    from oracle.sched_ref import Active, Params, Prof, decide_ref
+    from tests.helpers import golden_profile, load_golden
+    prof = Prof(golden_profile(load_golden("e3_squad_generation.json")))
+    one = [Active(0, 0, 0)]
+    assert [tuple(p)[:2] for p in decide_ref(0, one, prof, Params(squad_max=4, seed_all=False)).picks] == \
+        [(0, 0), (0, 1), (0, 2), (0, 3)]
+    assert [tuple(p)[:2] for p in decide_ref(0, one, prof, Params(squad_max=4, seed_all=False,
+                                                                   squad_max_solo=2)).picks] == [(0, 0), (0, 1)]
+    two = [Active(0, 0, 0), Active(1, 0, 0)]
+    a = decide_ref(0, two, prof, Params(squad_max=4, seed_all=False))
+    b = decide_ref(0, two, prof, Params(squad_max=4, seed_all=False, squad_max_solo=2))
+    assert a.picks == b.picks and len(a.picks) == 4
