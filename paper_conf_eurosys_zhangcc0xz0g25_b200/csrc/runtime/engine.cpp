@@ -925,7 +925,11 @@ void Engine::launcher_main(int t) {
           if (L.quit.load() || failed_) return;
           cpu_relax();
         }
-      for (void* ev : job.wait_events) rt_->stream_wait(ten_[t].stream, ev);
+      // the previous squad's event on this tenant's own stream is already
+      // ordered by the stream: waiting on it would only cut the programmatic
+      // (PDL) overlap between this stream's consecutive kernels
+      for (size_t i = 0; i < job.wait_events.size(); ++i)
+        if (i >= job.wait_parts.size() || job.wait_parts[i] != t) rt_->stream_wait(ten_[t].stream, job.wait_events[i]);
     }
     if (!exec_items(t, job.items, ten_[t].stream, err)) {
       fail(err);
@@ -1044,7 +1048,8 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
   };
   if (launchers_.empty()) {   // single launch thread (BLESS_LAUNCH_THREADS=0)
     for (int j : d.parts) {
-      for (void* ev : prev_events_) rt_->stream_wait(ten_[j].stream, ev);
+      for (size_t i = 0; i < prev_events_.size(); ++i)   // own stream: already ordered (see launcher_main)
+        if (i >= prev_parts_.size() || prev_parts_[i] != j) rt_->stream_wait(ten_[j].stream, prev_events_[i]);
       ten_[j].prev_light = 0;
     }
     for (size_t i = 0; i < d.picks.size(); ++i) {

@@ -24,6 +24,7 @@ def main():
     ap.add_argument("--squad-max", type=int, default=20)
     ap.add_argument("--split-pct", type=int, default=25)
     ap.add_argument("--max-inflight", type=int, default=2)
+    ap.add_argument("--squad-max-solo", type=int, default=0)
     ap.add_argument("--lookahead-us", type=float, default=20.0)
     ap.add_argument("--policies", default="BLESS,ISO,STATIC,UNBOUND")
     a = ap.parse_args()
@@ -42,19 +43,32 @@ def main():
             filts = [{j} for j in range(len(ms))] if pol == "ISO" else [None]
             for filt in filts:
                 p = capi.default_params(policy=pol, squad_max=a.squad_max, split_pct=a.split_pct,
-                                        max_inflight_squads=a.max_inflight, lookahead_ns=int(a.lookahead_us * 1000))
+                                        max_inflight_squads=a.max_inflight, lookahead_ns=int(a.lookahead_us * 1000),
+                                        squad_max_solo=a.squad_max_solo)
                 ctx.reset(p)
                 ctx.start()
                 ents = [(0, x.tenant, x.arrival_ns) for x in trace if filt is None or x.tenant in filt]
                 ids = capi.dispatch([ctx], ents, capi.now_ns() + 3_000_000)
                 ctx.drain(int(120e9))
                 ctx.stop()
+                infos = []
                 for (_, t, _), r in zip(ents, ids):
                     st, info = ctx.poll(r)
+                    infos.append((t, info.arrival_ns, info.start_ns, info.finish_ns))
                     d = out.setdefault(pol, {}).setdefault(ms[t].name, {"wait": [], "service": [], "lat": []})
                     d["wait"].append(info.start_ns - info.arrival_ns)
                     d["service"].append(info.finish_ns - info.start_ns)
                     d["lat"].append(info.finish_ns - info.arrival_ns)
+                if filt is None:
+                    # wait split by what the GPU was doing at the arrival: another
+                    # tenant's request in progress or not; own previous request
+                    # still in progress (FIFO) or not
+                    for t, arr, s0, _f in infos:
+                        other = any(t2 != t and a2 <= arr < f2 for t2, a2, _, f2 in infos)
+                        own = any(t2 == t and a2 < arr < f2 for t2, a2, _, f2 in infos)
+                        key = ("other_busy" if other else "other_idle") + ("+own_queue" if own else "")
+                        ws = out.setdefault(pol + "_wait_by_state", {}).setdefault(ms[t].name, {}).setdefault(key, [])
+                        ws.append(s0 - arr)
                 if pol == "BLESS":
                     decs = [capi.decision_to_tuple(x) for x in ctx.decisions()]
                     mix = out.setdefault("squads", {"solo": 0, "mixed_nsp": 0, "mixed_sp": 0})
@@ -69,6 +83,10 @@ def main():
     for pol, per in out.items():
         if pol == "squads":
             summ[pol] = per
+            continue
+        if pol.endswith("_wait_by_state"):
+            summ[pol] = {n: {k: {"n": len(v), "mean_us": float(np.mean(v)) / 1e3} for k, v in d.items()}
+                         for n, d in per.items()}
             continue
         summ[pol] = {n: {k: float(np.mean(v)) / 1e3 for k, v in d.items()} for n, d in per.items()}
     print(json.dumps(summ, indent=1))
