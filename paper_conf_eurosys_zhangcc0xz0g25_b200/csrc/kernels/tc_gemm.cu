@@ -414,9 +414,12 @@ constexpr int kTcThreads = 64 + 32 * kEpiWarps;
 constexpr int kMaxStages = 8;
 constexpr int kDynSmemMax = 227 * 1024 - 2048;   // opt-in limit minus the executor's static smem
 
-template <int BN, int BK>
+template <int BN, int BK, int MH = 1>
 struct TcCfg {
-  static constexpr int kStageA = 128 * BK * 2;
+  // MH = 2: the CTA's M tile is 256 rows -- one A box of 256 rows and TWO
+  // M = 128 MMAs per K step sharing the B tile (twice the FLOPs per TMA box:
+  // B200 charges a floor of ~130 ns per box)
+  static constexpr int kStageA = MH * 128 * BK * 2;
   static constexpr int kStageB = BN * BK * 2;
   static constexpr int kStageBytes = kStageA + kStageB;
   // default pipeline: ~96 KB of stages, so two CTAs (the next kernel's, under
@@ -425,16 +428,16 @@ struct TcCfg {
   // TMEM accumulators: double buffered (epilogue of tile i overlaps the MMAs of
   // tile i+1) up to BN = 128; BN = 256 keeps one so a second co-resident CTA
   // (another tenant's kernel on the same SM) can still allocate.
-  static constexpr int kAcc = BN >= 256 ? 1 : 2;
-  static constexpr int kTmemCols = (kAcc * BN) < 32 ? 32 : kAcc * BN;
+  static constexpr int kAcc = (BN * MH) >= 256 ? 1 : 2;
+  static constexpr int kTmemCols = (kAcc * MH * BN) < 32 ? 32 : kAcc * MH * BN;
   static constexpr int kFixed = 1024 /*align*/ + 256 /*barriers*/ + 2 * BN * 4 /*sc, sh*/;
   static constexpr int kSmem = kStages * kStageBytes + kFixed;
   static constexpr int kSmemMax = kMaxStages * kStageBytes + kFixed;
 };
 
-template <int BN, int BK, bool HALO>
+template <int BN, int BK, bool HALO, int MH>
 __device__ void tc_work(const TcParams& p, const GateArgs& g) {
-  using Cfg = TcCfg<BN, BK>;
+  using Cfg = TcCfg<BN, BK, MH>;
   const int ST = p.stages;                           // B stages (A and B stages when !HALO)
   const int NA = HALO ? p.astages : ST;              // A stages
   const int a_bytes = HALO ? p.a_stage_bytes : Cfg::kStageA;
@@ -571,13 +574,13 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         auto load_A = [&](int kb, int st) {
           unsigned char* a = sA + st * Cfg::kStageA;
           if (BK > 64 && p.mode == 0) {   // 3-D view (64, M, K/64)
-            tma_load_3d_e(a, &p.tmA, &full[st], 0, tm * 128, kb * 2);
+            tma_load_3d_e(a, &p.tmA, &full[st], 0, tm * 128 * MH, kb * 2);
           } else if (BK > 64) {            // 4-D view (64, W, H, C/64), stride 1 only
             const int tap = kb / p.kc_per_tap, ch = (kb - tap * p.kc_per_tap) * 2;
             const int r = tap / p.S_, s = tap - r * p.S_;
             tma_load_4d_e(a, &p.tmA, &full[st], 0, ow0 - p.pad + s, oh0 - p.pad + r, ch);
           } else if (p.mode == 0) {
-            tma_load_2d_e(a, &p.tmA, &full[st], kb * BK, tm * 128);
+            tma_load_2d_e(a, &p.tmA, &full[st], kb * BK, tm * 128 * MH);
           } else {
             const int tap = kb / p.kc_per_tap, c0 = (kb - tap * p.kc_per_tap) * BK;
             const int r = tap / p.S_, s = tap - r * p.S_;
@@ -674,7 +677,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       const int kb0 = ks * p.kbs, kb1 = min(p.num_kb, kb0 + p.kbs);
       mbar_wait(&tempty[acc], aph ^ 1);
       tc_fence_after();
-      const uint32_t d_tmem = tmem_u + acc * BN;
+      const uint32_t d_tmem = tmem_u + acc * MH * BN;
       if constexpr (HALO) {
         for (int c = kb0; c < kb1; ++c) {
           { TW_BEGIN(); mbar_wait(&fullA[astage], aphase); TW_END(0); }
@@ -717,7 +720,10 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
             // BK = 128: slab k / 4 (128 x 64 of A, BN x 64 of B), K step k % 4
             const uint32_t ao = BK > 64 ? (k >> 2) * (128 * 128) + (k & 3) * 32 : k * 32;
             const uint32_t bo = BK > 64 ? (k >> 2) * (BN * 128) + (k & 3) * 32 : k * 32;
-            tc_mma_e(d_tmem, smem_desc<BK>(a0 + ao), smem_desc<BK>(b0 + bo), idesc, (kb != kb0 || k) ? 1u : 0u);
+#pragma unroll
+            for (int h = 0; h < MH; ++h)   // M half h: A rows 128h.. (SW128 rows of BK*2 bytes), accumulator h
+              tc_mma_e(d_tmem + h * BN, smem_desc<BK>(a0 + h * (128 * BK * 2) + ao), smem_desc<BK>(b0 + bo), idesc,
+                       (kb != kb0 || k) ? 1u : 0u);
           }
           tc_commit_e(&empty[stage]);
         }
@@ -752,17 +758,21 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       const int tile = t / p.splits;
       const int tm = tile / p.tiles_n, tn = tile - tm * p.tiles_n;
       const int row = q * 32 + lane;
+      // output row of this thread in M half h (MH = 2 only for GEMM / 1x1 tiles)
+      auto out_row = [&](int h, int& m_, bool& valid_) {
+        if (p.mode == 0) {
+          m_ = (tm * MH + h) * 128 + row;
+          valid_ = m_ < p.M;
+        } else {
+          const int th = tm / p.tiles_w;
+          const int oh = th * p.BH + row / p.BW, ow = (tm - th * p.tiles_w) * p.BW + row % p.BW;
+          valid_ = oh < p.OH && ow < p.OW;
+          m_ = oh * p.OW + ow;
+        }
+      };
       int m;
       bool valid;
-      if (p.mode == 0) {
-        m = tm * 128 + row;
-        valid = m < p.M;
-      } else {
-        const int th = tm / p.tiles_w;
-        const int oh = th * p.BH + row / p.BW, ow = (tm - th * p.tiles_w) * p.BW + row % p.BW;
-        valid = oh < p.OH && ow < p.OW;
-        m = oh * p.OW + ow;
-      }
+      out_row(0, m, valid);
       // stage this tile's scale/shift (independent of the previous kernel)
       asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiWarps) : "memory");   // previous tile's readers are done
       for (int i = threadIdx.x - 64; i < BN; i += 32 * kEpiWarps) {
@@ -775,34 +785,49 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         pdl_wait();
         dep_waited = true;
       }
-      if (p.R && valid && c1 > c0) {  // pull this row's residual segment into L2 while the MMAs run
-        const char* rr = reinterpret_cast<const char*>(p.R + (size_t)m * p.ldr + tn * BN + c0);
-        for (int b = 0; b < (c1 - c0) * 2; b += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(rr + b));
+      for (int h = 0; h < MH; ++h) {   // pull this row's residual segment into L2 while the MMAs run
+        int mh;
+        bool vh;
+        out_row(h, mh, vh);
+        if (p.R && vh && c1 > c0) {
+          const char* rr = reinterpret_cast<const char*>(p.R + (size_t)mh * p.ldr + tn * BN + c0);
+          for (int b = 0; b < (c1 - c0) * 2; b += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(rr + b));
+        }
       }
       mbar_wait(&tfull[acc], aph);
       tc_fence_after();
       if (threadIdx.x == 64) TR(6);      // 6: accumulator ready (last tile)
-      const uint32_t tbase = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN;
+      const uint32_t tbase0 = tmem_base + ((uint32_t)(q * 32) << 16) + acc * MH * BN;
       if (p.splits == 1) {
-        TC_ACT_DISPATCH(p.act, (epi_cols<A_>(p, tbase, c0, c1, tn, BN, m, valid, epi_sc, epi_sh)))
+        for (int h = 0; h < MH; ++h) {
+          out_row(h, m, valid);
+          const uint32_t tbase = tbase0 + h * BN;
+          TC_ACT_DISPATCH(p.act, (epi_cols<A_>(p, tbase, c0, c1, tn, BN, m, valid, epi_sc, epi_sh)))
+        }
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty[acc]);
         if (threadIdx.x == 64) TR(7);    // 7: epilogue stores issued (last tile)
       } else {
         // split-K: add this unit's partial tile into the fp32 workspace
+        // (sub-tile tile*MH + h per M half)
+        for (int h = 0; h < MH; ++h) {
+          out_row(h, m, valid);
+          const uint32_t tbase = tbase0 + h * BN;
 #pragma unroll 1
-        for (int c = c0; c < c1; c += 16) {
-          uint32_t v[16];
-          tmem_ld16(tbase + c, v);
-          tmem_ld_wait();
-          if (!valid || tn * BN + c >= p.N) continue;
+          for (int c = c0; c < c1; c += 16) {
+            uint32_t v[16];
+            tmem_ld16(tbase + c, v);
+            tmem_ld_wait();
+            if (!valid || tn * BN + c >= p.N) continue;
 #pragma unroll
-          for (int i = 0; i < 4; ++i)
-            asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(ws_at(p, 0, tile, c, i, row, BN)),
-                         "f"(__uint_as_float(v[4 * i])), "f"(__uint_as_float(v[4 * i + 1])),
-                         "f"(__uint_as_float(v[4 * i + 2])), "f"(__uint_as_float(v[4 * i + 3]))
-                         : "memory");
+            for (int i = 0; i < 4; ++i)
+              asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(
+                               ws_at(p, 0, tile * MH + h, c, i, row, BN)),
+                           "f"(__uint_as_float(v[4 * i])), "f"(__uint_as_float(v[4 * i + 1])),
+                           "f"(__uint_as_float(v[4 * i + 2])), "f"(__uint_as_float(v[4 * i + 3]))
+                           : "memory");
+          }
         }
         tc_fence_before();
         __syncwarp();
@@ -827,7 +852,10 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
 #ifdef BLESS_TC_SPLIT_FENCE_ALL
           __threadfence();
 #endif
-          if (valid) TC_ACT_DISPATCH(p.act, (epi_ws<A_>(p, tile, row, c0, c1, tn, BN, m, epi_sc, epi_sh)))
+          for (int h = 0; h < MH; ++h) {
+            out_row(h, m, valid);
+            if (valid) TC_ACT_DISPATCH(p.act, (epi_ws<A_>(p, tile * MH + h, row, c0, c1, tn, BN, m, epi_sc, epi_sh)))
+          }
           if (threadIdx.x == 64) {
             p.sem[tile] = 0;
             TR(11);                        // 11: last unit's reduction epilogue done (split-K)
@@ -846,10 +874,10 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   __syncthreads();
 }
 
-template <int BN, int BK, bool HALO>
+template <int BN, int BK, bool HALO, int MH>
 __global__ void __launch_bounds__(kTcThreads, 2) k_tc_gemm(const __grid_constant__ TcParams p, const GateArgs g) {
   if (threadIdx.x == 0) TR(0);   // 0: CTA start
-  if (gate_in_range(g) || gate_linger(g)) tc_work<BN, BK, HALO>(p, g);
+  if (gate_in_range(g) || gate_linger(g)) tc_work<BN, BK, HALO, MH>(p, g);
   pdl_trigger();
   if (threadIdx.x == 0) TR(8);   // 8: work done, before the exit atomic
   if (!g.stamp) {                // light exit
@@ -858,18 +886,18 @@ __global__ void __launch_bounds__(kTcThreads, 2) k_tc_gemm(const __grid_constant
   }
   int last = 0;
   const bool fb = gate_leave(g, last);
-  if (fb) tc_work<BN, BK, HALO>(p, g);
+  if (fb) tc_work<BN, BK, HALO, MH>(p, g);
   if (last) gate_finalize(g, fb);
   if (threadIdx.x == 0) TR(9);   // 9: CTA exit
 }
 #endif  // __CUDACC__
 
 // ------------------------------------------------------------------ host side
-template <int BN, int BK, bool HALO>
+template <int BN, int BK, bool HALO, int MH>
 static cudaError_t launch_tc(const KernelDesc& d, const GateArgs& g, cudaStream_t st) {
   void* args[2] = {(void*)d.params, (void*)&g};
-  return launch_kernel((const void*)k_tc_gemm<BN, BK, HALO>, dim3(launch_grid(d, g)), dim3(d.block), (size_t)d.smem,
-                       st, args);
+  return launch_kernel((const void*)k_tc_gemm<BN, BK, HALO, MH>, dim3(launch_grid(d, g)), dim3(d.block),
+                       (size_t)d.smem, st, args);
 }
 
 // Halo stages: NA halo stages + NB weight stages (one filter row each) within
@@ -885,20 +913,21 @@ static bool halo_stages(const TcParams& p, int& na, int& nb) {
   return nb >= 2;
 }
 
-template <int BN, int BK, bool HALO>
+template <int BN, int BK, bool HALO, int MH = 1>
 static bool prep(KernelDesc& d, TcParams& p, std::string& err) {
   static std::once_flag once;
   static cudaError_t attr_err = cudaSuccess;
   std::call_once(once, [] {
-    attr_err = cudaFuncSetAttribute((const void*)k_tc_gemm<BN, BK, HALO>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    HALO ? kDynSmemMax : std::min(TcCfg<BN, BK>::kSmemMax, kDynSmemMax));
+    attr_err = cudaFuncSetAttribute((const void*)k_tc_gemm<BN, BK, HALO, MH>,
+                                    cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    HALO ? kDynSmemMax : std::min(TcCfg<BN, BK, MH>::kSmemMax, kDynSmemMax));
   });
   if (attr_err != cudaSuccess) {
     err = std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(attr_err);
     return false;
   }
   // pipeline depth: BLESS_TC_SMEM_KB overrides the ~96 KB default budget (sweeps)
-  using Cfg = TcCfg<BN, BK>;
+  using Cfg = TcCfg<BN, BK, MH>;
   int st = Cfg::kStages;
   if (const char* e = std::getenv("BLESS_TC_SMEM_KB")) {
     const int kb = std::atoi(e);
@@ -917,8 +946,8 @@ static bool prep(KernelDesc& d, TcParams& p, std::string& err) {
     p.stages = nb;
     d.smem = na * p.a_stage_bytes + nb * p.b_stage_bytes + Cfg::kFixed;
   }
-  d.launch = launch_tc<BN, BK, HALO>;
-  d.kernel_fn = (const void*)k_tc_gemm<BN, BK, HALO>;
+  d.launch = launch_tc<BN, BK, HALO, MH>;
+  d.kernel_fn = (const void*)k_tc_gemm<BN, BK, HALO, MH>;
   return true;
 }
 
@@ -983,11 +1012,13 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     const char* e = std::getenv("BLESS_TC_BK128");
     return !e || std::atoi(e) != 0;
   }();
+  int lda = 0;   // A row pitch (elements) for a re-encode of the A map (MH = 2)
   if (op.kind == BL_OP_GEMM) {
     p.M = (int)op.dims[0];
     p.N = (int)op.dims[1];
     p.K = (int)op.dims[2];
     const int ldx = op.dims[3] ? (int)op.dims[3] : p.K;
+    lda = ldx;
     p.ldy = op.dims[4] ? (int)op.dims[4] : p.N;
     p.ldr = op.dims[5] ? (int)op.dims[5] : p.N;
     if (p.M <= 8 || p.N % 16 || p.K % 8 || ldx % 8 || p.ldy % 8 || p.ldr % 8) return false;  // GEMV / SIMT
@@ -1010,6 +1041,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     const int K = (int)op.dims[4], R = (int)op.dims[5], S = (int)op.dims[6];
     const int stride = (int)op.dims[7], pad = (int)op.dims[8], groups = (int)op.dims[9];
     const int ldx = op.dims[10] ? (int)op.dims[10] : C;
+    lda = ldx;
     p.ldy = op.dims[11] ? (int)op.dims[11] : K;
     p.ldr = p.ldy;
     const bool one_by_one = R == 1 && S == 1 && stride == 1 && pad == 0;
@@ -1103,8 +1135,18 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   } else {
     return false;
   }
+  // M tile of 256 rows (two M = 128 MMAs per K step sharing one B tile):
+  // GEMM / 1x1 tiles with 64-deep stages (autotuner candidate, or BLESS_TC_MT=256)
+  const char* mte = std::getenv("BLESS_TC_MT");
+  const int want_mt = force ? force->mt : (mte ? std::atoi(mte) : 0);
+  const int MH = (want_mt == 256 && p.mode == 0 && BK == 64) ? 2 : 1;
+  if (MH == 2) {
+    cuuint64_t da[2] = {(cuuint64_t)p.K, (cuuint64_t)p.M}, sa[1] = {(cuuint64_t)lda * 2};
+    cuuint32_t ba[2] = {64, 256};
+    if (!encode(&p.tmA, 2, X, da, sa, ba, 64, err)) return false;
+  }
   // N tile: as wide as possible while keeping >= S tiles when the problem allows
-  const int tiles_m = (p.mode == 0) ? (p.M + 127) / 128 : p.tiles_w * ((p.OH + p.BH - 1) / p.BH);
+  const int tiles_m = (p.mode == 0) ? (p.M + 128 * MH - 1) / (128 * MH) : p.tiles_w * ((p.OH + p.BH - 1) / p.BH);
   // N tile: the widest that still yields >= S tiles; if even 32 does not,
   // split K (>= 3 K blocks per work unit) until there are ~S work units, so a
   // batch-1 layer with few output tiles can still spread over every SM of its
@@ -1134,6 +1176,10 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     BN = 64;
     p.tiles_n = (p.N + BN - 1) / BN;
   }
+  if (MH == 2 && BN > 128) {   // 2 x 128 TMEM columns at most (one accumulator pair)
+    BN = 128;
+    p.tiles_n = (p.N + BN - 1) / BN;
+  }
   if (p.mode == 3) {   // halo: the widest BN whose 1 halo + 2 weight stages fit (halo_stages)
     auto tpb = [&](int bn) { return bn >= 128 ? 1 : p.S_; };
     auto fits = [&](int bn) {
@@ -1151,8 +1197,8 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     const size_t nt = (size_t)ntiles(BN);
     // (a per-unit fp32 slab variant -- plain stores summed by the last unit --
     // was no faster on B200 and slower beyond 3 splits, profiles/round1/tc_splitk_*)
-    p.sk_tiles = (int)nt;
-    const size_t wsb = nt * 128 * BN * sizeof(float);
+    p.sk_tiles = (int)nt * MH;   // workspace sub-tiles of 128 rows
+    const size_t wsb = nt * MH * 128 * BN * sizeof(float);
     void* buf = nullptr;
     if (cudaMalloc(&buf, wsb + nt * sizeof(unsigned)) != cudaSuccess ||
         cudaMemset(buf, 0, wsb + nt * sizeof(unsigned)) != cudaSuccess) {
@@ -1190,7 +1236,9 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   if (const char* e = std::getenv("BLESS_TC_MAX_OCC")) d.max_occ = std::max(1, std::atoi(e));   // sweeps
   bool ok = false;
 #define TC_CASE(bn, bk) \
-  if (BN == bn && BK == bk && p.mode != 3) ok = prep<bn, bk, false>(d, p, err);
+  if (BN == bn && BK == bk && p.mode != 3 && MH == 1) ok = prep<bn, bk, false>(d, p, err);
+#define TC_MT2(bn) \
+  if (BN == bn && BK == 64 && p.mode == 0 && MH == 2) ok = prep<bn, 64, false, 2>(d, p, err);
 #define TC_HALO(bn) \
   if (BN == bn && p.mode == 3) ok = prep<bn, 64, true>(d, p, err);
   TC_CASE(16, 16) TC_CASE(16, 32) TC_CASE(16, 64)
@@ -1200,8 +1248,10 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   TC_CASE(256, 16) TC_CASE(256, 32) TC_CASE(256, 64)
   TC_CASE(16, 128) TC_CASE(32, 128) TC_CASE(64, 128)
   TC_HALO(16) TC_HALO(32) TC_HALO(64) TC_HALO(128)
+  TC_MT2(32) TC_MT2(64) TC_MT2(128)
 #undef TC_CASE
 #undef TC_HALO
+#undef TC_MT2
   if (!ok) {
     if (err.empty()) err = "no tc instantiation";
     return false;
@@ -1212,6 +1262,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
   d.choice_splits = p.splits;
   d.choice_bk = BK;
   d.choice_halo = p.mode == 3 ? 1 : 0;
+  d.choice_mt = 128 * MH;
   d.family = op.kind == BL_OP_GEMM ? "tc_gemm_bf16" : (p.mode == 0 ? "tc_conv1x1_bf16" : "tc_conv_bf16");
   if (BK == 128 && BN > 64 && p.mode == 3) { err = "halo BN"; return false; }
   d.flops = 2.0 * p.M * p.N * p.K;
@@ -1231,13 +1282,14 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
 // reduction costs several us), BK = 128 wins the 3x3 convs, BN = 128 with
 // BK = 64 wins large GEMMs; BN = 256 never won with 96 KB of stages.
 int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int max) {
-  long long M, N, num_kb, tiles_m, halo_tiles_m = 0, chunks = 0, halo_bw = 8;
-  bool bk128_ok = false, halo_ok = false;
+  long long M = 0, N, num_kb, tiles_m, halo_tiles_m = 0, chunks = 0, halo_bw = 8;
+  bool bk128_ok = false, halo_ok = false, gemm_like = false;
   if (op.kind == BL_OP_GEMM) {
     M = op.dims[0], N = op.dims[1];
     num_kb = (op.dims[2] + 63) / 64;
     tiles_m = (M + 127) / 128;
     bk128_ok = op.dims[2] % 64 == 0;
+    gemm_like = true;
   } else if (op.kind == BL_OP_CONV) {
     const long long H = op.dims[1], W = op.dims[2], C = op.dims[3], R = op.dims[5], S = op.dims[6];
     const long long st = op.dims[7] ? op.dims[7] : 1, pad = op.dims[8];
@@ -1249,6 +1301,8 @@ int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int ma
     while (BW < OW && BW < 128) BW <<= 1;
     tiles_m = ((OW + BW - 1) / BW) * ((OH + (128 / BW) - 1) / (128 / BW));
     bk128_ok = st == 1 && (one ? C % 64 == 0 : C % 128 == 0);
+    gemm_like = one;
+    M = OH * OW;
     halo_ok = st == 1 && R == 3 && S == 3 && pad == 1 && C % 64 == 0 && OW + 2 <= 128;
     if (halo_ok) {
       long long hw = 8;
@@ -1273,6 +1327,19 @@ int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int ma
       if (tiles < caps.S && chunks >= 2 && n < max) {
         const long long want = std::min<long long>((caps.S + tiles - 1) / tiles, chunks);
         if (want >= 2) out[n++] = TcChoice{bn, (int)want, 64, 1};
+      }
+    }
+  }
+  if (gemm_like) {
+    // M tiles of 256 rows (two M = 128 MMAs per K step): half the tiles, twice
+    // the FLOPs per TMA box
+    const long long tiles_m2 = (M + 255) / 256;
+    for (int bn = std::min(64, nmax); bn <= nmax && n < max; bn <<= 1) {
+      const long long tiles = tiles_m2 * ((N + bn - 1) / bn);
+      out[n++] = TcChoice{bn, 1, 64, 0, 256};
+      if (tiles < caps.S && num_kb >= 6 && n < max) {
+        const long long want = std::min<long long>((caps.S + tiles - 1) / tiles, num_kb / 3);
+        if (want >= 2) out[n++] = TcChoice{bn, (int)want, 64, 0, 256};
       }
     }
   }

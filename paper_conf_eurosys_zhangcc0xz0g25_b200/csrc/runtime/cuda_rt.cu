@@ -149,9 +149,9 @@ std::unique_ptr<DeviceRT> DeviceRT::create(int device, void* ws, size_t ws_bytes
     rt->tune_file_ = e;
     if (FILE* f = std::fopen(e, "r")) {
       char sig[512];
-      int bn = 0, sp = 0, bk = 0, halo = 0;
-      while (std::fscanf(f, "%511s %d %d %d %d", sig, &bn, &sp, &bk, &halo) == 5)
-        rt->tune_cache_[sig] = TcChoice{bn, sp, bk, halo};
+      int bn = 0, sp = 0, bk = 0, halo = 0, mt = 0;
+      while (std::fscanf(f, "%511s %d %d %d %d %d", sig, &bn, &sp, &bk, &halo, &mt) == 6)
+        rt->tune_cache_[sig] = TcChoice{bn, sp, bk, halo, mt};
       std::fclose(f);
     }
   }
@@ -286,7 +286,8 @@ int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
     auto it = tune_cache_.find(sig);
     if (it != tune_cache_.end()) {
       if (it->second.bn != kd->choice_bn || it->second.splits != kd->choice_splits ||
-          it->second.bk != kd->choice_bk || it->second.halo != kd->choice_halo) {
+          it->second.bk != kd->choice_bk || it->second.halo != kd->choice_halo ||
+          it->second.mt != kd->choice_mt) {
         std::unique_ptr<KernelDesc> k2(new KernelDesc());
         std::string e2;
         if (build_tc_gemm(op, caps_, *k2, e2, &it->second)) {
@@ -299,11 +300,11 @@ int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
       }
     } else {
       if (!autotune_tc(op, kd, err)) return -1;
-      tune_cache_[sig] = TcChoice{kd->choice_bn, kd->choice_splits, kd->choice_bk, kd->choice_halo};
+      tune_cache_[sig] = TcChoice{kd->choice_bn, kd->choice_splits, kd->choice_bk, kd->choice_halo, kd->choice_mt};
       if (!tune_file_.empty()) {
         if (FILE* f = std::fopen(tune_file_.c_str(), "a")) {
-          std::fprintf(f, "%s %d %d %d %d\n", sig.c_str(), kd->choice_bn, kd->choice_splits, kd->choice_bk,
-                       kd->choice_halo);
+          std::fprintf(f, "%s %d %d %d %d %d\n", sig.c_str(), kd->choice_bn, kd->choice_splits, kd->choice_bk,
+                       kd->choice_halo, kd->choice_mt);
           std::fclose(f);
         }
       }
@@ -317,7 +318,7 @@ int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
 // Shape signature of a tc op for the tuning cache (pointers excluded).
 std::string DeviceRT::tc_signature(const bl_op& op) const {
   // "v2": tune files since the autotuner also picks BK (older lines never match)
-  std::string s = "v3k" + std::to_string(op.kind) + "_t" + std::to_string(op.dtype) + "_r" + (op.ptr[4] ? "1" : "0");
+  std::string s = "v4k" + std::to_string(op.kind) + "_t" + std::to_string(op.dtype) + "_r" + (op.ptr[4] ? "1" : "0");
   for (int i = 0; i < 12; ++i) s += "_" + std::to_string(op.dims[i]);
   return s;
 }
@@ -328,8 +329,8 @@ std::string DeviceRT::tc_signature(const bl_op& op) const {
 // events, all S SMs) on the layer's own buffers; the fastest wins, and within
 // 3 % of it the one with fewer tiles (smaller d leaves more SMs to co-runners).
 bool DeviceRT::autotune_tc(const bl_op& op, std::unique_ptr<KernelDesc>& best, std::string& err) {
-  TcChoice cand[24];
-  const int nc = tc_candidates(op, caps_, cand, 24);
+  TcChoice cand[32];
+  const int nc = tc_candidates(op, caps_, cand, 32);
   if (nc <= 1) return true;
   if (!tune_stream_ && cudaStreamCreateWithFlags((cudaStream_t*)&tune_stream_, cudaStreamNonBlocking) != cudaSuccess) {
     err = "autotune stream";
@@ -346,13 +347,13 @@ bool DeviceRT::autotune_tc(const bl_op& op, std::unique_ptr<KernelDesc>& best, s
   }
   for (int i = 0; i < nc; ++i) {
     if (cand[i].bn == best->choice_bn && cand[i].splits == best->choice_splits && cand[i].bk == best->choice_bk &&
-        cand[i].halo == best->choice_halo)
+        cand[i].halo == best->choice_halo && (cand[i].mt ? cand[i].mt : 128) == best->choice_mt)
       continue;
     std::unique_ptr<KernelDesc> kd(new KernelDesc());
     std::string e2;
     if (!build_tc_gemm(op, caps_, *kd, e2, &cand[i])) continue;
     if (kd->choice_bn == best->choice_bn && kd->choice_splits == best->choice_splits &&
-        kd->choice_bk == best->choice_bk && kd->choice_halo == best->choice_halo) {
+        kd->choice_bk == best->choice_bk && kd->choice_halo == best->choice_halo && kd->choice_mt == best->choice_mt) {
       if (kd->owned) cudaFree(kd->owned);
       continue;
     }

@@ -31,7 +31,7 @@ struct KernelDesc {
   LaunchFn launch = nullptr;
   const void* kernel_fn = nullptr;  // for the occupancy query (grid = S x blocks/SM)
   void* owned = nullptr;   // device scratch owned by this kernel (split-K workspace), cudaFree'd with it
-  int choice_bn = 0, choice_splits = 0, choice_bk = 0, choice_halo = 0;  // tcgen05 tile configuration (0 = not a tc kernel)
+  int choice_bn = 0, choice_splits = 0, choice_bk = 0, choice_halo = 0, choice_mt = 0;  // tcgen05 tile config (0 = not tc)
   alignas(128) unsigned char params[4096];  // family-specific parameter block
 };
 
@@ -60,6 +60,7 @@ struct TcChoice {
   int bn = 0, splits = 0;
   int bk = 0;   // K depth per pipeline stage (64 or 128; 0 = the builder's default)
   int halo = 0; // 1: halo implicit-GEMM conv (one input box per channel chunk serves all 3x3 taps)
+  int mt = 0;   // M tile rows: 256 = two M = 128 MMAs per K step (GEMM / 1x1), 0/128 = one
 };
 bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& out, std::string& err,
                    const TcChoice* force = nullptr);

@@ -140,6 +140,34 @@ def test_tc_forced_configs(ctx, cfg, shape, monkeypatch):
     run_and_check(ctx, m, "bf16")
 
 
+@pytest.mark.parametrize("cfg", ["64,64,1", "128,64,1", "128,64,3", "64,64,2"])
+@pytest.mark.parametrize("shape", [("gemm", (384, 1024, 320)), ("gemm", (200, 272, 136)), ("gemm", (1000, 128, 64)),
+                                   ("gemm", (128, 3072, 768)), ("conv", (14, 14, 256, 512, 1, 1, 0)),
+                                   ("conv", (9, 9, 192, 64, 1, 1, 0))])
+def test_tc_mt256(ctx, cfg, shape, monkeypatch):
+    """M tiles of 256 rows (BLESS_TC_MT=256): one A box of 256 rows and two
+    M = 128 tcgen05.mma per K step into two TMEM accumulators sharing the B
+    tile; ragged M (384, 200, 81 pixels), K tails, split-K over 256-row tiles
+    (workspace sub-tiles), residual + GELU/ReLU epilogue."""
+    monkeypatch.setenv("BLESS_TC_MT", "256")
+    monkeypatch.setenv("BLESS_TC_CFG", cfg)
+    kind, dims = shape
+
+    def mk(b):
+        if kind == "conv":
+            H, W, C, K, k, s_, p_ = dims
+            x = b.input((1, H, W, C))
+            r = b.param(np.random.default_rng(2).standard_normal((1, H, W, K)).astype(np.float32))
+            b.conv(x, K, k, s_, p_, act="relu", bn=True, res=r)
+        else:
+            M, N, K = dims
+            r = b.param(np.random.default_rng(2).standard_normal((M, N)).astype(np.float32))
+            b.gemm(b.input((M, K)), N, act="gelu", bias=True, res=r)
+    m = one_layer(ctx, "bf16", mk)
+    assert ctx.kernel_info(m.tenant, 0).family.decode().startswith("tc_")
+    run_and_check(ctx, m, "bf16")
+
+
 @pytest.mark.parametrize("cfg", ["32,64,1", "64,64,1", "128,64,1", "64,64,3", "32,64,4"])
 @pytest.mark.parametrize("dims", [(56, 56, 64, 256), (28, 28, 128, 256), (14, 14, 256, 256), (7, 7, 512, 512),
                                   (20, 27, 256, 96), (112, 112, 64, 128), (13, 11, 64, 48)])
