@@ -1330,9 +1330,11 @@ int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int ma
       }
     }
   }
-  if (gemm_like) {
+  if (gemm_like && M >= 1024) {
     // M tiles of 256 rows (two M = 128 MMAs per K step): half the tiles, twice
-    // the FLOPs per TMA box
+    // the FLOPs per TMA box; only where M leaves enough tiles (B200: never
+    // faster on the configs' batch-1 GEMMs at ~96 KB of stages, 1.33x on a
+    // large HBM-streaming GEMM with 160-200 KB, profiles/round2/mt256/)
     const long long tiles_m2 = (M + 255) / 256;
     for (int bn = std::min(64, nmax); bn <= nmax && n < max; bn <<= 1) {
       const long long tiles = tiles_m2 * ((N + bn - 1) / bn);
