@@ -84,7 +84,7 @@ def parse():
     ap.add_argument("--no-baselines", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-slo", action="store_true", help="skip the SLO-mode experiment (§6.5)")
-    ap.add_argument("--also", default="C3,C4", help="other configs reported beside the headline (N=1 only)")
+    ap.add_argument("--also", default="C2,C3,C4", help="other configs reported beside the headline (N=1 only)")
     ap.add_argument("--also-rhos", default="0.3,0.5")
     ap.add_argument("--also-requests", type=int, default=40)
     ap.add_argument("--load-profile", default="", help="reuse a saved profile table instead of profiling")
@@ -438,17 +438,19 @@ def roofline_of(rep, launches_all, peaks, args):
 
 
 # ---------------------------------------------------------------------------- other configs (N=1)
-def other_config(cfg, args, capi, models, metrics, out_dir):
+def other_config(cfg, args, capi, models, metrics, out_dir, rhos=None):
     """A compact run of another config beside the headline: profile, then per
     load rho BLESS / STATIC / TEMPORAL T-wc / ISO on seeds 1-3 (same traces):
-    mean latency per policy, attainment per tenant, deviation (L320)."""
+    mean latency per policy, attainment per tenant, deviation (L320).  For the
+    headline config itself: the loads other than the headline's (its load
+    boundary)."""
     rep = Replica(0, 0, cfg, args, capi, models)
     rep.squad_max = args.squad_max or SQUAD_MAX[cfg]
     rep.profile(argparse.Namespace(**{**vars(args), "load_profile": ""}), out_dir, "also")
     res = {"workload": f"{cfg}: {CONFIG_NAMES[cfg]}", "squad_max": rep.squad_max, "T_iso_profile_ms":
            {n: t / 1e6 for n, t in zip(rep.names, rep.T_iso)}, "rho": {}}
     nt = len(rep.tms)
-    for rho in [float(x) for x in args.also_rhos.split(",") if x]:
+    for rho in (rhos if rhos is not None else [float(x) for x in args.also_rhos.split(",") if x]):
         lat = {}
         for pol, extra in (("BLESS", None), ("STATIC", None), ("TEMPORAL_Twc", {"temporal_work_conserving": 1}),
                            ("ISO", None)):
@@ -754,8 +756,13 @@ def native(args):
 
     others = {}
     if rank == 0 and world == 1 and nrep == 1 and args.also and not args.no_baselines:
-        for cfg in [c for c in args.also.split(",") if c and c != args.config]:
-            others[cfg] = other_config(cfg, args, capi, models, metrics, args.out_dir)
+        for cfg in [c for c in args.also.split(",") if c]:
+            if cfg == args.config:   # the headline config at the other loads (not when --rhos biases it)
+                rl = [float(x) for x in args.also_rhos.split(",") if x and abs(float(x) - args.rho) > 1e-9]
+                if rl and not args.rhos:
+                    others[cfg] = other_config(cfg, args, capi, models, metrics, args.out_dir, rl)
+            else:
+                others[cfg] = other_config(cfg, args, capi, models, metrics, args.out_dir)
 
     fallbacks = sum(r.fallback for la in launches_all for r in la)
     seed_means = {str(sd): float(np.mean(v)) / 1e6 for sd, v in sorted(seed_lat.items())}

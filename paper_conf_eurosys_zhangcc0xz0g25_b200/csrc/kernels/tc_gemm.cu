@@ -88,10 +88,32 @@ __device__ __forceinline__ unsigned long long tr_now() {
   return t;
 }
 #define TW_BEGIN() const unsigned long long tw0_ = tr_now()
-#define TW_END(slot) \
-  if ((threadIdx.x & 31) == 0 && blockIdx.x < kTrMax) { g_tc_wait[blockIdx.x][slot] += tr_now() - tw0_; g_tc_wait[blockIdx.x][slot + 1] += 1; }
+#define TW_END(slot) TW_END_K(slot, 0)
+// + an event log of the first kEvCta CTAs: per role (0 MMA warp, 1 producer)
+// {kind, time before the wait, time after it}; kind 1 weight/operand stage,
+// 2 halo stage, 9 commit of a stage's MMAs (MMA warp)
+constexpr int kEvCta = 8, kEvN = 192;
+__device__ unsigned long long g_tc_ev[2][kEvCta][kEvN][3];
+__device__ int g_tc_evn[2][kEvCta];
+__device__ __forceinline__ void ev_log(int role, int& n, int kind, unsigned long long t0, unsigned long long t1) {
+  if ((threadIdx.x & 31) == 0 && blockIdx.x < kEvCta && n < kEvN) {
+    g_tc_ev[role][blockIdx.x][n][0] = kind;
+    g_tc_ev[role][blockIdx.x][n][1] = t0;
+    g_tc_ev[role][blockIdx.x][n][2] = t1;
+    g_tc_evn[role][blockIdx.x] = ++n;
+  }
+}
+#define TW_END_K(slot, kind) \
+  { const unsigned long long tw1_ = tr_now(); \
+    if ((threadIdx.x & 31) == 0 && blockIdx.x < kTrMax) { g_tc_wait[blockIdx.x][slot] += tw1_ - tw0_; g_tc_wait[blockIdx.x][slot + 1] += 1; } \
+    ev_log(slot / 2, ev_n_, kind ? kind : 1, tw0_, tw1_); }
+#define EV_COMMIT() { const unsigned long long tc_ = tr_now(); ev_log(0, ev_n_, 9, tc_, tc_); }
+#define EV_DECL() int ev_n_ = 0
 #else
 #define TR(i) ((void)0)
+#define TW_END_K(slot, kind) ((void)0)
+#define EV_COMMIT() ((void)0)
+#define EV_DECL() ((void)0)
 #define TW_BEGIN() ((void)0)
 #define TW_END(slot) ((void)0)
 #endif
@@ -113,6 +135,22 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
       "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
       "r"(parity)
       : "memory");
+}
+// Warp-uniform wait (every lane polls, the loop exits on a warp vote): keeps
+// the MMA warp's control flow provably convergent, so ptxas can keep the
+// descriptor arithmetic on the uniform datapath instead of an ELECT +
+// R2UR.BROADCAST sequence per tcgen05.mma.
+__device__ __forceinline__ void mbar_wait_u(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  do {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+  } while (!__all_sync(0xffffffffu, ok));
 }
 __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1) {
   asm volatile(
@@ -465,6 +503,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   // warp index through a shuffle: provably warp-uniform, so role branches and
   // the MMA warp's loop stay on the uniform datapath
   const int warp = __shfl_sync(0xffffffffu, (int)(threadIdx.x >> 5), 0), lane = threadIdx.x & 31;
+  EV_DECL();
   if (threadIdx.x == 0) TR(1);   // 1: work entry
   // the first tile claim (an L2 atomic round trip) overlaps the barrier/TMEM setup
   bool marked = false;
@@ -604,7 +643,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
             if (++stage == ST) { stage = 0; phase ^= 1; }
           };
           auto load_halo = [&](int c) {
-            { TW_BEGIN(); mbar_wait(&emptyA[astage], aphase ^ 1); TW_END(2); }
+            { TW_BEGIN(); mbar_wait(&emptyA[astage], aphase ^ 1); TW_END_K(2, 2); }
             mbar_expect_tx_e(&fullA[astage], (uint32_t)p.a_tx);
             tma_load_4d_e(sA + astage * a_bytes, &p.tmA, &fullA[astage], c * 64, -p.pad, oh0 - p.pad, 0);
             if (++astage == NA) { astage = 0; aphase ^= 1; }
@@ -680,24 +719,27 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       const uint32_t d_tmem = tmem_u + acc * MH * BN;
       if constexpr (HALO) {
         for (int c = kb0; c < kb1; ++c) {
-          { TW_BEGIN(); mbar_wait(&fullA[astage], aphase); TW_END(0); }
+          { TW_BEGIN(); mbar_wait_u(&fullA[astage], aphase); TW_END_K(0, 2); }
           tc_fence_after();
           const uint32_t a_base = smem_u32(sA + astage * a_bytes);
           const int nbox = p.R_ * p.S_ / p.taps_per_b;
+          int r = 0, s_ = 0;   // filter tap of the next MMA group (no division: uniform datapath)
           for (int j = 0; j < nbox; ++j) {   // one weight stage = taps_per_b consecutive taps
-            { TW_BEGIN(); mbar_wait(&full[stage], phase); TW_END(0); }
+            { TW_BEGIN(); mbar_wait_u(&full[stage], phase); TW_END(0); }
             tc_fence_after();
             const uint32_t b_row = smem_u32(sB + stage * b_bytes);
             for (int u = 0; u < p.taps_per_b; ++u) {
-              const int tap = j * p.taps_per_b + u, r = tap / p.S_, s_ = tap - r * p.S_;
               const uint32_t a0 = a_base + (uint32_t)(r * p.BW + s_) * 128u;
               const uint32_t b0 = b_row + (uint32_t)u * (BN * 128u);
+              const uint32_t first = (c == kb0 && r == 0 && s_ == 0) ? 1u : 0u;
 #pragma unroll
               for (int k = 0; k < 4; ++k)
                 tc_mma_e(d_tmem, smem_desc_row(a0 + k * 32), smem_desc<64>(b0 + k * 32), idesc,
-                         (c != kb0 || tap || k) ? 1u : 0u);
+                         (first && k == 0) ? 0u : 1u);
+              if (++s_ == p.S_) { s_ = 0; ++r; }
             }
             tc_commit_e(&empty[stage]);
+            EV_COMMIT();
             __syncwarp();
             if (++stage == ST) { stage = 0; phase ^= 1; }
           }
@@ -707,7 +749,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         }
       }
       for (int kb = HALO ? kb1 : kb0; kb < kb1; ++kb) {
-        { TW_BEGIN(); mbar_wait(&full[stage], phase); TW_END(0); }
+        { TW_BEGIN(); mbar_wait_u(&full[stage], phase); TW_END(0); }
         tc_fence_after();
         if (lane == 0 && kb == kb0) TR(5);   // 5: first stage landed (last tile of this CTA)
         const uint32_t a0 = smem_u32(sA + stage * Cfg::kStageA);
@@ -726,6 +768,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
                        (kb != kb0 || k) ? 1u : 0u);
           }
           tc_commit_e(&empty[stage]);
+          EV_COMMIT();
         }
         __syncwarp();
         if (++stage == ST) { stage = 0; phase ^= 1; }
@@ -766,7 +809,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         } else {
           const int th = tm / p.tiles_w;
           const int oh = th * p.BH + row / p.BW, ow = (tm - th * p.tiles_w) * p.BW + row % p.BW;
-          valid_ = oh < p.OH && ow < p.OW;
+          valid_ = row < p.BH * p.BW && oh < p.OH && ow < p.OW;   // BH*BW < 128: tight halo tiles
           m_ = oh * p.OW + ow;
         }
       };
@@ -877,16 +920,28 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
 template <int BN, int BK, bool HALO, int MH>
 __global__ void __launch_bounds__(kTcThreads, 2) k_tc_gemm(const __grid_constant__ TcParams p, const GateArgs g) {
   if (threadIdx.x == 0) TR(0);   // 0: CTA start
-  if (gate_in_range(g) || gate_linger(g)) tc_work<BN, BK, HALO, MH>(p, g);
-  pdl_trigger();
-  if (threadIdx.x == 0) TR(8);   // 8: work done, before the exit atomic
-  if (!g.stamp) {                // light exit
-    if (threadIdx.x == 0) TR(9);
-    return;
-  }
+  // ONE inlined copy of tc_work (pass 0: in range / lingering; pass 1: the
+  // exit protocol's fallback): with two copies ptxas moved the MMA warp's
+  // descriptor arithmetic off the uniform datapath (an ELECT + 5 x
+  // R2UR.BROADCAST sequence per tcgen05.mma, ~50 ns per MMA issued instead of
+  // the tensor pipe's ~30)
+  bool run = gate_in_range(g) || gate_linger(g);
+  bool fb = false;
   int last = 0;
-  const bool fb = gate_leave(g, last);
-  if (fb) tc_work<BN, BK, HALO, MH>(p, g);
+#pragma unroll 1
+  for (int pass = 0; pass < 2; ++pass) {
+    if (run) tc_work<BN, BK, HALO, MH>(p, g);
+    if (pass == 1) break;
+    pdl_trigger();
+    if (threadIdx.x == 0) TR(8);   // 8: work done, before the exit atomic
+    if (!g.stamp) {                // light exit
+      if (threadIdx.x == 0) TR(9);
+      return;
+    }
+    fb = gate_leave(g, last);
+    run = fb;
+    if (!fb) break;
+  }
   if (last) gate_finalize(g, fb);
   if (threadIdx.x == 0) TR(9);   // 9: CTA exit
 }
@@ -903,14 +958,49 @@ static cudaError_t launch_tc(const KernelDesc& d, const GateArgs& g, cudaStream_
 // Halo stages: NA halo stages + NB weight stages (one filter row each) within
 // ~113 KB, so that two halo convs (or a halo conv and any other tile) still
 // share an SM's 228 KB: two halo stages when two weight stages fit beside
-// them, else one halo stage.  Returns false if not even 1 + 2 fit.
+// them (the next chunk's halo lands while this chunk's nine taps run), else
+// one.  Returns false if not even 1 + 2 fit.  BLESS_TC_HALO_KB overrides the
+// budget, BLESS_TC_HALO_NA=1 forces one halo stage (A/B sweeps).
+static int halo_budget_kb() {
+  const char* e = std::getenv("BLESS_TC_HALO_KB");
+  return e ? std::max(64, std::min(226, std::atoi(e))) : 113;
+}
 template <int BN>
 static bool halo_stages(const TcParams& p, int& na, int& nb) {
   using Cfg = TcCfg<BN, 64>;
-  const int budget = 113 * 1024 - Cfg::kFixed;
-  na = (2 * p.a_stage_bytes + 2 * p.b_stage_bytes <= budget) ? 2 : 1;
+  const int budget = halo_budget_kb() * 1024 - Cfg::kFixed;
+  const char* fe = std::getenv("BLESS_TC_HALO_NA");
+  const bool one = fe && std::atoi(fe) == 1;
+  na = (!one && 2 * p.a_stage_bytes + 2 * p.b_stage_bytes <= budget) ? 2 : 1;
   nb = std::min(4, (budget - na * p.a_stage_bytes) / p.b_stage_bytes);
   return nb >= 2;
+}
+
+// Halo tile geometry: a tile is BH output rows of BW >= OW + 2 pixels (the
+// halo row of every valid output column stays inside the tile row), BH*BW <=
+// 128.  BW = OW + 2 exactly ("tight": 58 for OW = 56 -- a 30 KB halo stage, so
+// two halo stages and two weight stages fit 113 KB) unless BLESS_TC_HALO_POW2=1
+// (the power-of-two width of round 2's first halo kernel).  A stage holds the
+// (BH + 2) x BW halo plus the rows the shifted tap views of the rows >= BH*BW
+// (outputs discarded) can reach: row 127 + 2*BW + 2.
+struct HaloGeo {
+  int bw, bh, rows, a_stage;
+};
+static HaloGeo halo_geo(int OW) {
+  const char* pe = std::getenv("BLESS_TC_HALO_POW2");
+  const bool pow2 = pe && std::atoi(pe) != 0;
+  HaloGeo g;
+  g.bw = std::max(8, OW + 2);
+  if (pow2) {
+    int hw = 8;
+    while (hw < OW + 2) hw <<= 1;
+    g.bw = hw;
+  }
+  g.bh = 128 / g.bw;
+  const int need = std::max((g.bh + 2) * g.bw, 130 + 2 * g.bw);
+  g.rows = (need + 7) / 8 * 8;
+  g.a_stage = (g.rows * 128 + 1023) / 1024 * 1024;
+  return g;
 }
 
 template <int BN, int BK, bool HALO, int MH = 1>
@@ -1115,17 +1205,15 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     const int halo_env = he ? std::atoi(he) : 0;
     const bool want_halo = force ? force->halo != 0 : halo_env != 0;
     if (want_halo && stride == 1 && R == 3 && S == 3 && pad == 1 && C % 64 == 0 && p.OW + 2 <= 128) {
-      int hw = 8;
-      while (hw < p.OW + 2) hw <<= 1;
+      const HaloGeo hg = halo_geo(p.OW);
       p.mode = 3;
       BK = 64;
-      p.BW = hw;
-      p.BH = 128 / hw;
+      p.BW = hg.bw;
+      p.BH = hg.bh;
       p.tiles_w = 1;
       p.kc_per_tap = C / 64;
       p.num_kb = C / 64;            // K blocks = channel chunks (nine taps each)
-      const int rows = (p.BH + 2) * p.BW + 8;   // + the s-shift overrun rows (only invalid outputs read them)
-      p.a_stage_bytes = (rows * 128 + 1023) / 1024 * 1024;
+      p.a_stage_bytes = hg.a_stage;   // + the shifted-view overrun rows (only invalid outputs read them)
       p.a_tx = 64 * 2 * p.BW * (p.BH + 2);
       cuuint64_t da[4] = {(cuuint64_t)C, (cuuint64_t)Wd, (cuuint64_t)H, 1};
       cuuint64_t sa[3] = {(cuuint64_t)ldx * 2, (cuuint64_t)Wd * ldx * 2, (cuuint64_t)H * Wd * ldx * 2};
@@ -1184,7 +1272,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
     auto tpb = [&](int bn) { return bn >= 128 ? 1 : p.S_; };
     auto fits = [&](int bn) {
       const int fixed = 1024 + 256 + 2 * bn * 4;
-      return p.a_stage_bytes + 2 * tpb(bn) * bn * 128 <= 113 * 1024 - fixed;
+      return p.a_stage_bytes + 2 * tpb(bn) * bn * 128 <= halo_budget_kb() * 1024 - fixed;
     };
     while (BN > 16 && !fits(BN)) BN >>= 1;
     p.tiles_n = (p.N + BN - 1) / BN;
@@ -1282,7 +1370,7 @@ bool build_tc_gemm(const bl_op& op, const DeviceCaps& caps, KernelDesc& d, std::
 // reduction costs several us), BK = 128 wins the 3x3 convs, BN = 128 with
 // BK = 64 wins large GEMMs; BN = 256 never won with 96 KB of stages.
 int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int max) {
-  long long M = 0, N, num_kb, tiles_m, halo_tiles_m = 0, chunks = 0, halo_bw = 8;
+  long long M = 0, N, num_kb, tiles_m, halo_tiles_m = 0, chunks = 0, halo_a_stage = 0;
   bool bk128_ok = false, halo_ok = false, gemm_like = false;
   if (op.kind == BL_OP_GEMM) {
     M = op.dims[0], N = op.dims[1];
@@ -1305,10 +1393,9 @@ int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int ma
     M = OH * OW;
     halo_ok = st == 1 && R == 3 && S == 3 && pad == 1 && C % 64 == 0 && OW + 2 <= 128;
     if (halo_ok) {
-      long long hw = 8;
-      while (hw < OW + 2) hw <<= 1;
-      halo_tiles_m = (OH + (128 / hw) - 1) / (128 / hw);
-      halo_bw = hw;
+      const HaloGeo hg = halo_geo((int)OW);
+      halo_tiles_m = (OH + hg.bh - 1) / hg.bh;
+      halo_a_stage = hg.a_stage;
     }
     chunks = C / 64;
   } else {
@@ -1318,10 +1405,9 @@ int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int ma
   const int nmax = N <= 16 ? 16 : (N <= 32 ? 32 : (N <= 64 ? 64 : 128));
   if (halo_ok) {
     // halo tiles: BH x BW with BW >= OW + 2; K blocks = 64-channel chunks
-    const long long a_stage = (((128 / halo_bw) + 2) * halo_bw + 8) * 128;
     for (int bn = std::min(32, nmax); bn <= nmax && n < max; bn <<= 1) {
       const int tpb = bn >= 128 ? 1 : 3;
-      if ((a_stage + 1023) / 1024 * 1024 + 2 * tpb * bn * 128 > 113 * 1024 - (1024 + 256 + 2 * bn * 4)) break;
+      if (halo_a_stage + 2 * tpb * bn * 128 > halo_budget_kb() * 1024 - (1024 + 256 + 2 * bn * 4)) break;
       const long long tiles = halo_tiles_m * ((N + bn - 1) / bn);
       out[n++] = TcChoice{bn, 1, 64, 1};
       if (tiles < caps.S && chunks >= 2 && n < max) {
@@ -1373,7 +1459,13 @@ extern "C" int bl_debug_tc_wait(unsigned long long* host, int n_cta) {
   const size_t n = (size_t)std::min(n_cta, bless::kTrMax) * 4 * sizeof(unsigned long long);
   return (int)cudaMemcpyFromSymbol(host, bless::g_tc_wait, n);
 }
+extern "C" int bl_debug_tc_events(unsigned long long* host, int* counts) {
+  cudaMemcpyFromSymbol(counts, bless::g_tc_evn, sizeof(bless::g_tc_evn));
+  return (int)cudaMemcpyFromSymbol(host, bless::g_tc_ev, sizeof(bless::g_tc_ev));
+}
 extern "C" int bl_debug_tc_trace_clear() {
+  static int zn[2][bless::kEvCta];
+  cudaMemcpyToSymbol(bless::g_tc_evn, zn, sizeof(zn));
   static unsigned long long z[bless::kTrMax][bless::kTrN];
   static unsigned long long zw[bless::kTrMax][4];
   cudaMemcpyToSymbol(bless::g_tc_wait, zw, sizeof(zw));

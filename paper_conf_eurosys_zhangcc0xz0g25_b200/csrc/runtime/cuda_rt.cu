@@ -318,7 +318,7 @@ int DeviceRT::add_kernel(const bl_op& op, std::string& err) {
 // Shape signature of a tc op for the tuning cache (pointers excluded).
 std::string DeviceRT::tc_signature(const bl_op& op) const {
   // "v2": tune files since the autotuner also picks BK (older lines never match)
-  std::string s = "v4k" + std::to_string(op.kind) + "_t" + std::to_string(op.dtype) + "_r" + (op.ptr[4] ? "1" : "0");
+  std::string s = "v5k" + std::to_string(op.kind) + "_t" + std::to_string(op.dtype) + "_r" + (op.ptr[4] ? "1" : "0");
   for (int i = 0; i < 12; ++i) s += "_" + std::to_string(op.dims[i]);
   return s;
 }

@@ -170,15 +170,22 @@ def test_tc_mt256(ctx, cfg, shape, monkeypatch):
 
 @pytest.mark.parametrize("cfg", ["32,64,1", "64,64,1", "128,64,1", "64,64,3", "32,64,4"])
 @pytest.mark.parametrize("dims", [(56, 56, 64, 256), (28, 28, 128, 256), (14, 14, 256, 256), (7, 7, 512, 512),
-                                  (20, 27, 256, 96), (112, 112, 64, 128), (13, 11, 64, 48)])
-def test_tc_halo_conv(ctx, cfg, dims, monkeypatch):
+                                  (20, 27, 256, 96), (112, 112, 64, 128), (13, 11, 64, 48), (56, 56, 256, 64)])
+@pytest.mark.parametrize("geom", ["tight", "pow2", "tight_na1"])
+def test_tc_halo_conv(ctx, cfg, dims, geom, monkeypatch):
     """Halo implicit-GEMM 3x3 conv (mode 3): one TMA box of the tile's
     (BH + 2) x BW input halo per 64-channel chunk, each tap's A operand read
-    from it at row offset r*BW + s (UMMA descriptor with the swizzle base
-    offset).  Exact vs the oracle for square, ragged and 112-wide maps, every
-    BN, split-K over channel chunks, with residual + ReLU epilogue."""
+    from it at row offset r*BW + s.  Tile width BW = OW + 2 ("tight": BH*BW <
+    128, rows past BH*BW masked in the epilogue, two halo stages where they
+    fit) or the power-of-two width; one halo stage forced.  Exact vs the oracle
+    for square, ragged and 112-wide maps, every BN, split-K over channel
+    chunks, with residual + ReLU epilogue."""
     monkeypatch.setenv("BLESS_TC_HALO", "1")
     monkeypatch.setenv("BLESS_TC_CFG", cfg)
+    if geom == "pow2":
+        monkeypatch.setenv("BLESS_TC_HALO_POW2", "1")
+    if geom == "tight_na1":
+        monkeypatch.setenv("BLESS_TC_HALO_NA", "1")
     H, W, C, K = dims
 
     def mk(b):

@@ -22,6 +22,52 @@ NAMES = ["start", "entry", "setup", "claim", "pdl_wait", "stage0", "acc_ready", 
          "sk_arrived", "sk_reduced"]   # 10/11: split-K units only
 
 
+def events(L):
+    """Per-stage event log of the first CTAs of the last launch: when the
+    producer issued each load (after its free-stage wait), when the MMA warp saw
+    it land, and when it committed the stage's MMAs."""
+    ev = np.zeros((2, 8, 192, 3), dtype=np.uint64)
+    cnt = np.zeros((2, 8), dtype=np.int32)
+    L.bl_debug_tc_events.argtypes = [C.c_void_p, C.c_void_p]
+    L.bl_debug_tc_events(ev.ctypes.data, cnt.ctypes.data)
+    ev = ev.astype(np.int64)
+    lat = {1: [], 2: []}
+    gaps, mwait, pwait = [], [], []
+    for cta in range(8):
+        nm, npd = cnt[0, cta], cnt[1, cta]
+        if nm == 0 or npd == 0:
+            continue
+        m, pr = ev[0, cta, :nm], ev[1, cta, :npd]
+        for kind in (1, 2):
+            iss = pr[pr[:, 0] == kind, 2]
+            seen = m[m[:, 0] == kind, 2]
+            k = min(len(iss), len(seen))
+            lat[kind] += list(seen[:k] - iss[:k])
+        com = m[m[:, 0] == 9, 1]
+        gaps += list(np.diff(com))
+        mwait += list(m[m[:, 0] != 9, 2] - m[m[:, 0] != 9, 1])
+        pwait += list(pr[:, 2] - pr[:, 1])
+        if cta == 0:
+            t0 = min(pr[0, 1], m[0, 1])
+            print("  CTA 0 event log (us from its first event): P = producer (wait start -> issue), "
+                  "M = MMA warp (wait start -> landed), C = commit")
+            rows = [(x[1], f"P{'W' if x[0] == 1 else 'H'} {(x[1] - t0) / 1e3:6.2f}->{(x[2] - t0) / 1e3:6.2f}") for x in pr]
+            rows += [(x[1], (f"C  {(x[1] - t0) / 1e3:6.2f}" if x[0] == 9 else
+                             f"M{'W' if x[0] == 1 else 'H'} {(x[1] - t0) / 1e3:6.2f}->{(x[2] - t0) / 1e3:6.2f}")) for x in m]
+            rows.sort()
+            line = []
+            for _, r in rows:
+                line.append(r)
+                if len(line) == 5:
+                    print("    " + " | ".join(line))
+                    line = []
+            if line:
+                print("    " + " | ".join(line))
+    f = lambda a: f"{np.mean(a) / 1e3:.3f}" if len(a) else "-"
+    print(f"  (first 8 CTAs) issue -> MMA-warp-sees-landed: weights {f(lat[1])} us, halo {f(lat[2])} us; "
+          f"commit-to-commit {f(gaps)} us; MMA warp wait per stage {f(mwait)} us; producer wait per load {f(pwait)} us")
+
+
 def main():
     assert "BLESS_TC_TRACE" in os.environ.get("BLESS_EXTRA_NVFLAGS", ""), "set BLESS_EXTRA_NVFLAGS=-DBLESS_TC_TRACE"
     from paper_conf_eurosys_zhangcc0xz0g25_b200 import build, capi
@@ -63,6 +109,8 @@ def main():
                 print(f"  {i} {nm:10s} {col.min() / 1e3:8.2f} {np.median(col) / 1e3:8.2f} {col.max() / 1e3:8.2f}")
         allx = v[v[:, 9] > 0, 9] - t0
         print(f"  last CTA exit (all CTAs) {allx.max() / 1e3:.2f} us")
+        if reps > 1:
+            events(L)
         if reps == 1:   # wait accounting of that single launch (counters accumulate over launches)
             wb = np.zeros((2048, 4), dtype=np.uint64)
             L.bl_debug_tc_wait.argtypes = [C.c_void_p, C.c_int]
