@@ -86,7 +86,7 @@ def parse():
     ap.add_argument("--no-slo", action="store_true", help="skip the SLO-mode experiment (§6.5)")
     ap.add_argument("--also", default="C2,C3,C4", help="other configs reported beside the headline (N=1 only)")
     ap.add_argument("--also-rhos", default="0.3,0.5")
-    ap.add_argument("--also-requests", type=int, default=40)
+    ap.add_argument("--also-requests", type=int, default=80)
     ap.add_argument("--load-profile", default="", help="reuse a saved profile table instead of profiling")
     ap.add_argument("--light", action="store_true", help="timed steps only (for ncu launch lists)")
     ap.add_argument("--out-dir", default=os.path.join(ROOT, "gpurun_out"))

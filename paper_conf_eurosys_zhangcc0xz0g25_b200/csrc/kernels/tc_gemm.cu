@@ -71,12 +71,18 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)_
 // Debug builds only (-DBLESS_TC_TRACE, tools/tctrace.py): per-CTA %globaltimer
 // stamps of the pipeline phases of the last launch.
 #ifdef BLESS_TC_TRACE
-constexpr int kTrMax = 2048, kTrN = 12;
+constexpr int kTrMax = 2048, kTrN = 13;
 __device__ unsigned long long g_tc_trace[kTrMax][kTrN];
+// latest CTA exit of any launch so far: read at griddepcontrol.wait's return
+// (slot 12) it is the predecessor's last exit, so slot 4 - slot 12 = the
+// programmatic-dependent-launch release latency
+__device__ unsigned long long g_tc_last_exit;
 __device__ __forceinline__ void tr_mark(int i) {
   unsigned long long t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   if (blockIdx.x < kTrMax) g_tc_trace[blockIdx.x][i] = t;
+  if (i == 9) atomicMax(&g_tc_last_exit, t);
+  if (i == 4 && blockIdx.x < kTrMax) g_tc_trace[blockIdx.x][12] = *(volatile unsigned long long*)&g_tc_last_exit;
 }
 #define TR(i) tr_mark(i)
 // wait accounting per CTA: [0] MMA warp waiting for operands (ns), [1] count,
@@ -340,6 +346,21 @@ __device__ __forceinline__ float act_t(float y) {
   return y;
 }
 
+// 256-bit global accesses (sm_100: LDG/STG.E.ENL2.256): one full 32-byte
+// sector per lane -- half the store instructions of two 128-bit stores, and no
+// half-sector writes, for the per-thread output rows of the epilogue.
+__device__ __forceinline__ void st_global_256(void* ptr, const uint4& a, const uint4& b) {
+  asm volatile("st.global.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(ptr), "r"(a.x), "r"(a.y), "r"(a.z),
+               "r"(a.w), "r"(b.x), "r"(b.y), "r"(b.z), "r"(b.w)
+               : "memory");
+}
+__device__ __forceinline__ void ld_global_256(const void* ptr, uint4& a, uint4& b) {
+  asm volatile("ld.global.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(a.x), "=r"(a.y), "=r"(a.z), "=r"(a.w), "=r"(b.x), "=r"(b.y), "=r"(b.z), "=r"(b.w)
+               : "l"(ptr)
+               : "memory");
+}
+
 // Fused epilogue for 16 consecutive columns of one output row:
 // y = act(acc * scale + shift + R), rounded to bf16 (RNE), vector stores.
 // sc/sh: the tile's per-column scale/shift staged in shared memory (1 / 0
@@ -353,8 +374,13 @@ __device__ __forceinline__ void epi_store16(const TcParams& p, int m, int n0, fl
   if (p.R) {
     const __nv_bfloat16* rr = p.R + (size_t)m * p.ldr + n0;
     if (full16 && ((p.ldr & 7) == 0)) {
-      uint4 r0 = *reinterpret_cast<const uint4*>(rr);
-      uint4 r1 = *reinterpret_cast<const uint4*>(rr + 8);
+      uint4 r0, r1;
+      if ((((uintptr_t)rr) & 31) == 0) {
+        ld_global_256(rr, r0, r1);
+      } else {
+        r0 = *reinterpret_cast<const uint4*>(rr);
+        r1 = *reinterpret_cast<const uint4*>(rr + 8);
+      }
       const __nv_bfloat16* e0 = reinterpret_cast<const __nv_bfloat16*>(&r0);
       const __nv_bfloat16* e1 = reinterpret_cast<const __nv_bfloat16*>(&r1);
 #pragma unroll
@@ -377,8 +403,12 @@ __device__ __forceinline__ void epi_store16(const TcParams& p, int m, int n0, fl
     __nv_bfloat162* ob = reinterpret_cast<__nv_bfloat162*>(o);
 #pragma unroll
     for (int i = 0; i < 8; ++i) ob[i] = __floats2bfloat162_rn(act_t<ACT>(y[2 * i]), act_t<ACT>(y[2 * i + 1]));
-    *reinterpret_cast<uint4*>(yy) = o[0];
-    *reinterpret_cast<uint4*>(yy + 8) = o[1];
+    if ((((uintptr_t)yy) & 31) == 0) {
+      st_global_256(yy, o[0], o[1]);
+    } else {
+      *reinterpret_cast<uint4*>(yy) = o[0];
+      *reinterpret_cast<uint4*>(yy + 8) = o[1];
+    }
   } else {
     for (int i = 0; i < 16; ++i)
       if (n0 + i < p.N) yy[i] = __float2bfloat16_rn(act_t<ACT>(y[i]));
@@ -1403,7 +1433,8 @@ int tc_candidates(const bl_op& op, const DeviceCaps& caps, TcChoice* out, int ma
   }
   int n = 0;
   const int nmax = N <= 16 ? 16 : (N <= 32 ? 32 : (N <= 64 ? 64 : 128));
-  if (halo_ok) {
+  const char* he = std::getenv("BLESS_TC_HALO");   // "0": no halo candidates (A/B sweeps)
+  if (halo_ok && !(he && std::atoi(he) == 0)) {
     // halo tiles: BH x BW with BW >= OW + 2; K blocks = 64-channel chunks
     for (int bn = std::min(32, nmax); bn <= nmax && n < max; bn <<= 1) {
       const int tpb = bn >= 128 ? 1 : 3;

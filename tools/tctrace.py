@@ -91,7 +91,7 @@ def main():
     for reps in (1, 20):
         L.bl_debug_tc_trace_clear()
         ns, _ = ctx.profile_kernel(t, 0, S, reps)
-        buf = np.zeros((2048, 12), dtype=np.uint64)
+        buf = np.zeros((2048, 13), dtype=np.uint64)
         L.bl_debug_tc_trace(buf.ctypes.data, 2048)
         v = buf.astype(np.int64)
         ok = (v[:, 0] > 0) & (v[:, 1] >= v[:, 0]) & (v[:, 9] >= v[:, 1]) & (v[:, 7] > 0)
@@ -109,6 +109,11 @@ def main():
                 print(f"  {i} {nm:10s} {col.min() / 1e3:8.2f} {np.median(col) / 1e3:8.2f} {col.max() / 1e3:8.2f}")
         allx = v[v[:, 9] > 0, 9] - t0
         print(f"  last CTA exit (all CTAs) {allx.max() / 1e3:.2f} us")
+        rel = w[:, 4] - w[:, 12]
+        rel = rel[(w[:, 12] > 0) & (rel > -1e6) & (rel < 1e6)]
+        if reps > 1 and len(rel):
+            print(f"  griddepcontrol.wait return - predecessor's last CTA exit: min {rel.min() / 1e3:.2f} "
+                  f"med {np.median(rel) / 1e3:.2f} max {rel.max() / 1e3:.2f} us")
         if reps > 1:
             events(L)
         if reps == 1:   # wait accounting of that single launch (counters accumulate over launches)
