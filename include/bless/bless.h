@@ -423,8 +423,20 @@ bl_status bl_dispatch(bl_ctx* const* ctxs, int n_ctx, const bl_dispatch_entry* e
  * queue + exit protocol, 2: 1 + device completion stamps, 3: 2 with
  * programmatic dependent launch).  variant | 4 (4..7) returns instead the
  * mean HOST time per launch call of the same loop (enqueue cost, ns).
- * BL_E_INVALID for variant outside 0..7 or reps < 1. */
+ * variant | 8 captures the reps launches into one CUDA graph and launches
+ * that instead (capture untimed).
+ * BL_E_INVALID for variant outside 0..15 or reps < 1. */
 bl_status bl_debug_overhead(bl_ctx* ctx, int variant, int reps, int64_t* ns_out);
+
+/* Diagnostics: one whole request of 'tenant' (every kernel, in order, on
+ * logical SMs [lo, hi), light exits for the middle kernels, programmatic
+ * dependent launch) launched on the tenant's stream (graph = 0) or captured
+ * into a CUDA graph and launched as one graph (graph = 1; capture and
+ * instantiation untimed).  Medians over reps: device_ns = CUDA-event time of
+ * the chain, host_ns = host time spent enqueueing it.  BL_E_STATE while
+ * running; BL_E_INVALID for a bad tenant/range or reps < 1. */
+bl_status bl_debug_chain(bl_ctx* ctx, int tenant, int lo, int hi, int graph, int reps, int64_t* device_ns,
+                         int64_t* host_ns);
 
 int64_t bl_now_ns(void);
 const char* bl_last_error(void);

@@ -145,6 +145,8 @@ _SIGS = {
     "bl_place": (C.c_int, [C.c_int, _P(C.c_int64), _P(C.c_int64), C.c_int, _P(C.c_int64), C.c_int32,
                            _P(C.c_int32)]),
     "bl_debug_overhead": (C.c_int, [C.c_void_p, C.c_int, C.c_int, _P(C.c_int64)]),
+    "bl_debug_chain": (C.c_int, [C.c_void_p, C.c_int, C.c_int, C.c_int, C.c_int, C.c_int, _P(C.c_int64),
+                                 _P(C.c_int64)]),
     "bl_now_ns": (C.c_int64, []),
     "bl_last_error": (C.c_char_p, []),
     "bl_version": (C.c_char_p, []),
@@ -244,6 +246,11 @@ class Ctx:
         ns = C.c_int64()
         check("bl_debug_overhead", lib().bl_debug_overhead(self.h, variant, reps, C.byref(ns)))
         return ns.value
+
+    def debug_chain(self, tenant: int, lo: int, hi: int, graph: int, reps: int = 5):
+        dv, hv = C.c_int64(), C.c_int64()
+        check("bl_debug_chain", lib().bl_debug_chain(self.h, tenant, lo, hi, graph, reps, C.byref(dv), C.byref(hv)))
+        return dv.value, hv.value
 
     def kernel_info(self, tenant: int, k: int) -> bl_kernel_info:
         out = bl_kernel_info()

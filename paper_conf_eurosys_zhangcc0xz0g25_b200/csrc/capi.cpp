@@ -254,6 +254,12 @@ bl_status bl_debug_overhead(bl_ctx* ctx, int variant, int reps, int64_t* ns) {
   return wrap([&](std::string& e) { return ctx->eng->debug_overhead(variant, reps, ns, e); });
 }
 
+bl_status bl_debug_chain(bl_ctx* ctx, int tenant, int lo, int hi, int graph, int reps, int64_t* device_ns,
+                         int64_t* host_ns) {
+  GUARD(ctx);
+  return wrap([&](std::string& e) { return ctx->eng->debug_chain(tenant, lo, hi, graph, reps, device_ns, host_ns, e); });
+}
+
 int64_t bl_now_ns(void) {
   return std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now().time_since_epoch())
       .count();

@@ -495,6 +495,7 @@ bool DeviceRT::overhead(int variant, int reps, int64_t* ns_out, std::string& err
   RT_CHECK(cudaEventCreate(&e1));
   const int S = info_.sm_count;
   const bool host_time = (variant & 4) != 0;
+  const bool graph = (variant & 8) != 0;
   variant &= 3;
   const int saved_pdl = g_use_pdl;
   g_use_pdl = variant == 3 ? 1 : 0;
@@ -511,9 +512,24 @@ bool DeviceRT::overhead(int variant, int reps, int64_t* ns_out, std::string& err
   };
   for (int i = 0; i < 10; ++i) one();
   RT_CHECK(cudaStreamSynchronize(s));
+  cudaGraphExec_t ge = nullptr;
+  if (graph) {   // the same reps launches captured into one graph (launch cost off the host)
+    cudaGraph_t gr = nullptr;
+    RT_CHECK(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+    for (int i = 0; i < reps; ++i) one();
+    RT_CHECK(cudaStreamEndCapture(s, &gr));
+    RT_CHECK(cudaGraphInstantiate(&ge, gr, 0));
+    cudaGraphDestroy(gr);
+    RT_CHECK(cudaGraphUpload(ge, s));
+    RT_CHECK(cudaStreamSynchronize(s));
+  }
   RT_CHECK(cudaEventRecord(e0, s));
   const auto h0 = std::chrono::steady_clock::now();
-  for (int i = 0; i < reps; ++i) one();
+  if (graph) {
+    RT_CHECK(cudaGraphLaunch(ge, s));
+  } else {
+    for (int i = 0; i < reps; ++i) one();
+  }
   const auto h1 = std::chrono::steady_clock::now();
   RT_CHECK(cudaEventRecord(e1, s));
   RT_CHECK(cudaEventSynchronize(e1));
@@ -522,9 +538,68 @@ bool DeviceRT::overhead(int variant, int reps, int64_t* ns_out, std::string& err
   *ns_out = host_time ? (int64_t)(std::chrono::duration<double, std::nano>(h1 - h0).count() / reps)
                       : (int64_t)(ms * 1e6 / reps);
   g_use_pdl = saved_pdl;
+  if (ge) cudaGraphExecDestroy(ge);
   cudaEventDestroy(e0);
   cudaEventDestroy(e1);
   cudaStreamDestroy(s);
+  return true;
+}
+
+bool DeviceRT::chain_time(const std::vector<int>& hs, int lo, int hi, int graph, int reps, void* stream,
+                          int64_t* device_ns, int64_t* host_ns, std::string& err) {
+  cudaStream_t s = (cudaStream_t)stream;
+  cudaEvent_t e0, e1;
+  RT_CHECK(cudaEventCreate(&e0));
+  RT_CHECK(cudaEventCreate(&e1));
+  std::vector<int64_t> dv, hv;
+  const int n = (int)hs.size();
+  auto enqueue = [&]() -> bool {
+    uint64_t prev = 0;
+    for (int k = 0; k < n; ++k) {
+      const bool stamp = k == 0 || k == n - 1;
+      const uint64_t seq = alloc_seq();
+      if (!launch_seq(hs[k], seq, lo, hi, s, err, stamp, prev)) return false;
+      prev = stamp ? 0 : seq;
+    }
+    return true;
+  };
+  for (int r = 0; r < reps + 1; ++r) {   // rep 0 is a warm-up
+    RT_CHECK(cudaStreamSynchronize(s));
+    cudaGraphExec_t ge = nullptr;
+    if (graph) {
+      cudaGraph_t g = nullptr;
+      RT_CHECK(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+      if (!enqueue()) { cudaStreamEndCapture(s, &g); return false; }
+      RT_CHECK(cudaStreamEndCapture(s, &g));
+      RT_CHECK(cudaGraphInstantiate(&ge, g, 0));
+      cudaGraphDestroy(g);
+      RT_CHECK(cudaGraphUpload(ge, s));
+      RT_CHECK(cudaStreamSynchronize(s));
+    }
+    RT_CHECK(cudaEventRecord(e0, s));
+    const auto h0 = std::chrono::steady_clock::now();
+    if (graph) {
+      RT_CHECK(cudaGraphLaunch(ge, s));
+    } else if (!enqueue()) {
+      return false;
+    }
+    const auto h1 = std::chrono::steady_clock::now();
+    RT_CHECK(cudaEventRecord(e1, s));
+    RT_CHECK(cudaEventSynchronize(e1));
+    float ms = 0.f;
+    RT_CHECK(cudaEventElapsedTime(&ms, e0, e1));
+    if (ge) cudaGraphExecDestroy(ge);
+    if (r > 0) {
+      dv.push_back((int64_t)(ms * 1e6));
+      hv.push_back((int64_t)std::chrono::duration<double, std::nano>(h1 - h0).count());
+    }
+  }
+  std::sort(dv.begin(), dv.end());
+  std::sort(hv.begin(), hv.end());
+  *device_ns = dv[dv.size() / 2];
+  *host_ns = hv[hv.size() / 2];
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
   return true;
 }
 

@@ -48,6 +48,13 @@ class DeviceRT {
   // Diagnostics: per-launch time of back-to-back S-CTA launches.  variant 0:
   // empty kernel; 1: gate + tile queue + exit protocol; 2: 1 + host-mapped stamps.
   bool overhead(int variant, int reps, int64_t* ns_out, std::string& err);
+  // Diagnostics: one request chain (kernels hs[0..n) on [lo, hi), light exits
+  // for the middle kernels, PDL) launched on stream (graph = 0) or captured
+  // into a CUDA graph and launched as one graph (graph = 1; capture and
+  // instantiation not timed).  Median over reps of the event-timed chain
+  // (device_ns) and of the host time spent enqueueing it (host_ns).
+  bool chain_time(const std::vector<int>& hs, int lo, int hi, int graph, int reps, void* stream,
+                  int64_t* device_ns, int64_t* host_ns, std::string& err);
   // Non-blocking: true if launch seq's stats are in the host mirror.
   bool poll(uint64_t seq, LaunchStats* out);
   void peek(uint64_t seq, LaunchStats* out);

@@ -169,9 +169,22 @@ bl_status Engine::set_io(int t, const void* hin, void* din, size_t inb, const vo
 bl_status Engine::debug_overhead(int variant, int reps, int64_t* ns, std::string& err) {
   if (!rt_) { err = "no device"; return BL_E_STATE; }
   if (started_) { err = "diagnostics while running"; return BL_E_STATE; }
-  if (!ns || variant < 0 || variant > 7 || reps < 1) { err = "bad args"; return BL_E_INVALID; }
+  if (!ns || variant < 0 || variant > 15 || reps < 1) { err = "bad args"; return BL_E_INVALID; }
   rt_->set_device();
   return rt_->overhead(variant, reps, ns, err) ? BL_OK : BL_E_CUDA;
+}
+
+bl_status Engine::debug_chain(int t, int lo, int hi, int graph, int reps, int64_t* dev_ns, int64_t* host_ns,
+                              std::string& err) {
+  if (!rt_) { err = "no device"; return BL_E_STATE; }
+  if (started_) { err = "diagnostics while running"; return BL_E_STATE; }
+  if (t < 0 || t >= nten() || lo < 0 || hi > S() || lo >= hi || reps < 1 || !dev_ns || !host_ns) {
+    err = "bad args";
+    return BL_E_INVALID;
+  }
+  rt_->set_device();
+  return rt_->chain_time(ten_[t].handles, lo, hi, graph, reps, ten_[t].stream, dev_ns, host_ns, err) ? BL_OK
+                                                                                                       : BL_E_CUDA;
 }
 
 bl_status Engine::kernel_info(int t, int k, bl_kernel_info* out, std::string& err) {

@@ -100,6 +100,7 @@ class Engine {
   bl_status run_kernel(int t, int k, int lo, int hi, std::string& err);
   bl_status kernel_info(int t, int k, bl_kernel_info* out, std::string& err);
   bl_status debug_overhead(int variant, int reps, int64_t* ns, std::string& err);
+  bl_status debug_chain(int t, int lo, int hi, int graph, int reps, int64_t* dev_ns, int64_t* host_ns, std::string& err);
   bl_status set_io(int t, const void* hin, void* din, size_t inb, const void* dout, void* hout, size_t outb,
                    std::string& err);
   bl_status profile_kernel(int t, int k, int sm_count, int reps, int64_t* ns, int* d, std::string& err);

@@ -19,13 +19,16 @@ def main():
     ap.add_argument("--grid", nargs="+", default=["split_pct=0,50"])
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--requests", type=int, default=60)
+    ap.add_argument("--rho", default="0.5")
+    ap.add_argument("--reuse-profile", action="store_true",
+                    help="profile once into profiles/ and reuse it (default: every point profiles its own kernels)")
     a = ap.parse_args()
     axes = []
     for g in a.grid:
         k, vs = g.split("=")
         axes.append([(k, v) for v in vs.split(",")])
     prof = os.path.join(ROOT, "profiles", f"profile_{a.config}_b200.txt")
-    if not os.path.exists(prof):   # profile once (kernel configs are autotuned at registration), reuse for all points
+    if a.reuse_profile and not os.path.exists(prof):   # profile once (kernel configs are autotuned at registration), reuse for all points
         os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
         subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--config", a.config, "--no-cpu-baseline",
                         "--no-baselines", "--steps", "1", "--warmup", "1", "--requests", "10"], capture_output=True)
@@ -37,8 +40,9 @@ def main():
                     g.write(f.read())
     for point in itertools.product(*axes):
         args = [sys.executable, os.path.join(ROOT, "bench.py"), "--config", a.config, "--no-cpu-baseline", "--no-slo",
-                "--steps", str(a.steps), "--warmup", "1", "--requests", str(a.requests)]
-        if os.path.exists(prof):
+                "--steps", str(a.steps), "--warmup", "1", "--requests", str(a.requests), "--also", ""]
+        args += ["--rho", a.rho]
+        if a.reuse_profile and os.path.exists(prof):
             args += ["--load-profile", prof]
         for k, v in point:
             args += ["--" + k.replace("_", "-"), v]
