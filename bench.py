@@ -78,7 +78,12 @@ def parse():
                     help="reading R36: cap of a squad with a single active request (0 = S_max)")
     ap.add_argument("--ablate", type=int, default=0,
                     help="PAPER.md §6.8 ablation (R32): 1 = no multi-task scheduler, 2 = no determiner, 3 = both")
+    ap.add_argument("--barrier", type=int, default=0,
+                    help="squad barrier: 0 = every participant waits for the previous squad (L276); "
+                         "1 = SM-range barrier (reading R37)")
     ap.add_argument("--lookahead-us", type=float, default=20.0)
+    ap.add_argument("--dump-squads", type=int, default=0,
+                    help="write the first N squads of the timed steps (picks, ranges, predicted vs measured) to out-dir")
     ap.add_argument("--max-inflight", type=int, default=2)
     ap.add_argument("--profile-reps", type=int, default=5)
     ap.add_argument("--no-baselines", action="store_true")
@@ -146,7 +151,7 @@ class ClockSampler:
 
 
 # ---------------------------------------------------------------------------- helpers
-def squad_timeline(decisions, launches):
+def squad_timeline(decisions, launches, m_of=None, S=148, barrier=0):
     """Map each BLESS decision to its launches (logged in pick order) and
     measure: squad makespan vs the predicted t_hat (Eq. 1 for SP, Eq. 2 for
     NSP; PAPER.md L214/L227 report 6.7%/7.1% error on A100) and the GPU idle
@@ -158,14 +163,38 @@ def squad_timeline(decisions, launches):
     spans = []
     viol = 0
     prev = None
+    # squad shape (a squad closes at S_max picks or on a
+    # request's last kernel) and SM-time busy fraction inside squads
+    npk, npt, by_last, sm_busy, sm_span = [], [], 0, 0.0, 0.0
+    last = {}   # barrier = 1: tenant -> (end of its latest chain, SM mask of that chain)
     for d in decisions:
         ls = launches[i:i + d.n_picks]
         i += d.n_picks
+        npk.append(d.n_picks)
+        npt.append(d.n_part)
+        if m_of is not None and d.n_picks and d.pick_kernel[d.n_picks - 1] == m_of[d.pick_tenant[d.n_picks - 1]] - 1:
+            by_last += 1
         if len(ls) != d.n_picks or any(r.end_ns <= 0 or r.nsm <= 0 for r in ls):
             prev = None
+            last = {}
             continue
         spans.append((min(r.start_ns for r in ls), max(r.end_ns for r in ls), d.t_hat, bool(d.config_sp)))
-        if prev is not None:   # barrier: no launch starts before ANOTHER tenant's squad-s end
+        sm_busy += sum((r.end_ns - r.start_ns) * r.nsm for r in ls)
+        sm_span += (spans[-1][1] - spans[-1][0]) * S
+        if barrier == 1:
+            # SM-range barrier (R37): no launch starts before the end of another
+            # tenant's latest chain whose kernels used any SM this tenant's
+            # chain in this squad uses
+            umask = {}
+            for r in ls:
+                umask[r.tenant] = umask.get(r.tenant, 0) | (((1 << (r.hi - r.lo)) - 1) << r.lo)
+            for r in ls:
+                for t, (e, msk) in last.items():
+                    if t != r.tenant and msk & umask[r.tenant]:
+                        viol += int(r.start_ns < e - 64)
+            for t, msk in umask.items():
+                last[t] = (max(r.end_ns for r in ls if r.tenant == t), msk)
+        elif prev is not None:   # barrier: no launch starts before ANOTHER tenant's squad-s end
             for r in ls:
                 others = [e for t, e in prev.items() if t != r.tenant]
                 viol += int(bool(others) and r.start_ns < max(others) - 64)
@@ -194,7 +223,13 @@ def squad_timeline(decisions, launches):
             # ANOTHER tenant's end would be a broken barrier
             "pdl_overlapped_switches": int(sum(1 for g in gaps if g < 0)),
             "barrier_violations": viol,
-            "makespan_us_median": med([e - s for s, e, _, _ in spans])}
+            "makespan_us_median": med([e - s for s, e, _, _ in spans]),
+            "picks_per_squad_mean": float(np.mean(npk)), "participants_per_squad_mean": float(np.mean(npt)),
+            "closed_by_last_kernel_pct": 100.0 * by_last / max(1, len(decisions)) if m_of is not None else None,
+            # sum over launches of (end - start) x SMs that ran a tile, over
+            # sum over squads of makespan x S: the fraction of SM-time inside
+            # squads that holds a running kernel (1 - bubbles)
+            "in_squad_sm_busy_frac": sm_busy / sm_span if sm_span else None}
 
 
 def make_trace(T_iso, rho, n, seed, bursty=False):
@@ -242,7 +277,8 @@ class Replica:
         return capi.default_params(squad_max=self.squad_max, policy=pol, split_pct=args.split_pct,
                                    ablate=args.ablate, squad_max_solo=args.squad_max_solo,
                                    lookahead_ns=int(args.lookahead_us * 1000),
-                                   max_inflight_squads=args.max_inflight, **(extra or {}))
+                                   max_inflight_squads=args.max_inflight, barrier=args.barrier,
+                                   **(extra or {}))
 
 
 def run_box(reps, capi, params_of, box, gpu_to_ctx, tenants_filter=None):
@@ -740,7 +776,21 @@ def native(args):
                        for j in range(len(r0.tms))]
             cpu = oracle_timing(r0.names, dec, prof, prm, [len(lat_all[0][j]) for j in range(len(r0.tms))], sq_seen)
 
-    tl = [squad_timeline(d, l) for d, l in timelines]
+    tl = [squad_timeline(d, l, [len(m.layers) for m in reps[0].tms], reps[0].S, args.barrier) for d, l in timelines]
+    if args.dump_squads and timelines and rank == 0:
+        dump, (dd, ll) = [], timelines[0]
+        i = 0
+        for d in dd[:args.dump_squads]:
+            ls = ll[i:i + d.n_picks]
+            i += d.n_picks
+            t0 = min(r.start_ns for r in ls) if ls else 0
+            dump.append({"now": d.now, "t_hat_us": d.t_hat / 1e3, "t_nsp_us": d.t_nsp / 1e3, "sp": bool(d.config_sp),
+                         "active": [(d.act_tenant[x], d.act_next[x], d.act_arrival[x]) for x in range(d.n_active)],
+                         "p": [d.part_p[x] for x in range(d.n_part)] if d.config_sp else None,
+                         "launches": [(r.tenant, r.kernel, r.lo, r.hi, r.nsm, round((r.start_ns - t0) / 1e3, 1),
+                                       round((r.end_ns - t0) / 1e3, 1)) for r in ls]})
+        with open(os.path.join(args.out_dir, f"squads_{args.config}.json"), "w") as f:
+            json.dump(dump, f)
     tl = [t for t in tl if t]
     timeline = {}
     if tl:
@@ -777,7 +827,7 @@ def native(args):
                    "trace": f"{'MMPP-2 bursty' if args.config == 'C4' else 'Poisson'} rho={args.rhos or args.rho} "
                    f"per tenant, {args.requests} requests/tenant/step, seeds 1-3, box-wide trace routed by the "
                    "native dispatcher (bl_dispatch)", "squad_max": r0.squad_max,
-                   "split_pct": args.split_pct, "ablate": args.ablate, "squad_max_solo": args.squad_max_solo,
+                   "split_pct": args.split_pct, "ablate": args.ablate, "squad_max_solo": args.squad_max_solo, "barrier": args.barrier,
                    "parallelism": f"replicas x{n_box} (no collective; "
                                   f"{'one process per GPU, gloo host barrier' if world > 1 else 'one process'})",
                    "quotas": [m.quota for m in r0.tms],

@@ -42,7 +42,7 @@ class bl_params(C.Structure):
                 ("temporal_work_conserving", C.c_int32), ("max_inflight_squads", C.c_int32),
                 ("lookahead_ns", C.c_int64), ("max_requests", C.c_int64),
                 ("ablate", C.c_int32), ("sm_limit", C.c_int32),
-                ("squad_max_solo", C.c_int32), ("reserved1", C.c_int32)]
+                ("squad_max_solo", C.c_int32), ("barrier", C.c_int32)]
 
 
 class bl_op(C.Structure):

@@ -3,6 +3,7 @@
 #include "engine.hpp"
 
 #include <algorithm>
+#include <array>
 #include <chrono>
 #include <climits>
 #include <cmath>
@@ -43,7 +44,7 @@ Engine::~Engine() {
 bl_status Engine::init(void* ws, size_t ws_bytes, std::string& err) {
   if (prm_.sm_unit < 1 || prm_.squad_max < 1 || prm_.squad_max > BL_MAX_SQUAD || prm_.split_pct < 0 ||
       prm_.ablate < 0 || prm_.ablate > 3 || prm_.squad_max_solo < 0 || prm_.squad_max_solo > BL_MAX_SQUAD ||
-      prm_.split_pct > 100 || prm_.max_requests < 1) {
+      prm_.split_pct > 100 || prm_.max_requests < 1 || prm_.barrier < 0 || prm_.barrier > 1) {
     err = "invalid bl_params";
     return BL_E_INVALID;
   }
@@ -411,6 +412,7 @@ bl_status Engine::start(std::string& err) {
   prev_events_.clear();
   prev_parts_.clear();
   prev_squad_ = 0;
+  last_chain_.assign(nten(), LastChain{});
   stop_ = false;
   failed_ = false;
   t0_ = now_ns() + 1000000;  // VIRTUAL on a device: wall anchor of trace time 0
@@ -551,6 +553,7 @@ bl_status Engine::reset(const bl_params* p, std::string& err) {
   if (st != BL_OK && st != BL_E_CUDA) return st;
   if (p) {
     if (p->max_requests != prm_.max_requests) { err = "max_requests cannot change on reset"; return BL_E_INVALID; }
+    if (p->barrier < 0 || p->barrier > 1) { err = "invalid bl_params.barrier"; return BL_E_INVALID; }
     prm_ = *p;
     prof_.g = prm_.sm_unit;
     prof_.derive();
@@ -933,11 +936,14 @@ void Engine::launcher_main(int t) {
     if (job.wait_squad) {
       // squad barrier: the previous squad's events must have been recorded
       // (by their launchers) before this stream waits on them
-      for (int l : job.wait_parts)
-        while (launchers_[l]->recorded.load(std::memory_order_acquire) < job.wait_squad) {
+      for (size_t i = 0; i < job.wait_parts.size(); ++i) {
+        const int l = job.wait_parts[i];
+        const uint64_t need = job.wait_sq.empty() ? job.wait_squad : job.wait_sq[i];
+        while (launchers_[l]->recorded.load(std::memory_order_acquire) < need) {
           if (L.quit.load() || failed_) return;
           cpu_relax();
         }
+      }
       // the previous squad's event on this tenant's own stream is already
       // ordered by the stream: waiting on it would only cut the programmatic
       // (PDL) overlap between this stream's consecutive kernels
@@ -1059,10 +1065,43 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
     const Pick& p = d.picks[i];
     return p.kernel == 0 || p.kernel == (int)prof_.ten[p.tenant].k.size() - 1 || last_pick[p.tenant] == (int)i;
   };
+  // What each participant's chain waits for.  barrier = 0 (paper-literal,
+  // L276): every other participant of the previous squad.  barrier = 1
+  // (reading R37): the latest chain of every other tenant that is still in
+  // flight and whose kernels ran on logical SMs this participant's kernels
+  // will use -- per SM the squads still run one after the other, but a chain
+  // no longer waits for chains on SMs it does not touch.
+  const int nt = nten();
+  std::vector<std::array<uint64_t, 3>> umask(nt, std::array<uint64_t, 3>{0, 0, 0});
+  for (const Pick& p : d.picks)
+    for (int x = p.lo; x < p.hi && x < 192; ++x) umask[p.tenant][x >> 6] |= 1ull << (x & 63);
+  std::vector<std::vector<int>> wparts(nt);
+  std::vector<std::vector<void*>> wevs(nt);
+  std::vector<std::vector<uint64_t>> wsqs(nt);
+  if ((int)last_chain_.size() != nt) last_chain_.assign(nt, LastChain{});
+  for (int j : d.parts) {
+    if (prm_.barrier == 1) {
+      for (int l = 0; l < nt; ++l) {
+        const LastChain& c = last_chain_[l];
+        if (l == j || !c.ev) continue;
+        if (inflight_.empty() || c.squad < inflight_.front().squad) continue;   // retired: complete
+        if (!((c.mask[0] & umask[j][0]) | (c.mask[1] & umask[j][1]) | (c.mask[2] & umask[j][2]))) continue;
+        wparts[j].push_back(l);
+        wevs[j].push_back(c.ev);
+        wsqs[j].push_back(c.squad);
+      }
+    } else {
+      for (size_t i = 0; i < prev_events_.size(); ++i) {   // own stream: already ordered (see launcher_main)
+        if (i < prev_parts_.size() && prev_parts_[i] == j) continue;
+        wparts[j].push_back(i < prev_parts_.size() ? prev_parts_[i] : -1);
+        wevs[j].push_back(prev_events_[i]);
+        wsqs[j].push_back(prev_squad_);
+      }
+    }
+  }
   if (launchers_.empty()) {   // single launch thread (BLESS_LAUNCH_THREADS=0)
     for (int j : d.parts) {
-      for (size_t i = 0; i < prev_events_.size(); ++i)   // own stream: already ordered (see launcher_main)
-        if (i >= prev_parts_.size() || prev_parts_[i] != j) rt_->stream_wait(ten_[j].stream, prev_events_[i]);
+      for (void* e : wevs[j]) rt_->stream_wait(ten_[j].stream, e);
       ten_[j].prev_light = 0;
     }
     for (size_t i = 0; i < d.picks.size(); ++i) {
@@ -1076,9 +1115,10 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
   if (!launchers_.empty()) {
     for (int j : d.parts) {
       jobs[j].squad = sq;
-      jobs[j].wait_squad = prev_squad_;
-      jobs[j].wait_parts = prev_parts_;
-      jobs[j].wait_events = prev_events_;
+      jobs[j].wait_squad = wparts[j].empty() ? 0 : 1;
+      jobs[j].wait_parts = wparts[j];
+      jobs[j].wait_sq = wsqs[j];
+      jobs[j].wait_events = wevs[j];
     }
     for (size_t i = 0; i < d.picks.size(); ++i) {
       const Pick& p = d.picks[i];
@@ -1099,6 +1139,12 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
   }
   for (int j : d.parts)
     if (!launchers_.empty()) push_job(j, std::move(jobs[j]));
+  for (size_t i = 0; i < d.parts.size(); ++i) {
+    LastChain& c = last_chain_[d.parts[i]];
+    c.ev = inf.events[i];
+    c.squad = sq;
+    for (int w = 0; w < 3; ++w) c.mask[w] = umask[d.parts[i]][w];
+  }
   prev_events_ = inf.events;
   prev_parts_ = d.parts;
   prev_squad_ = sq;

@@ -64,7 +64,8 @@ struct LaunchItem {
 struct LaunchJob {
   uint64_t squad = 0;             // squad id (0: none -- baseline policies)
   uint64_t wait_squad = 0;        // squad barrier: every launcher in wait_parts
-  std::vector<int> wait_parts;    //   must have recorded squad wait_squad first,
+  std::vector<int> wait_parts;    //   must have recorded squad wait_squad first
+  std::vector<uint64_t> wait_sq;  //   (per part when non-empty: barrier = 1),
   std::vector<void*> wait_events; //   then its stream waits on wait_events
   std::vector<LaunchItem> items;
   void* record_event = nullptr;   // recorded after the items (squad barrier)
@@ -201,6 +202,14 @@ class Engine {
   uint64_t prev_squad_ = 0;
   std::deque<Inflight> inflight_;
   std::vector<void*> prev_events_;
+  // SM-range barrier (bl_params.barrier = 1, reading R37): per tenant, its
+  // latest chain's end event, squad id and the logical SMs its kernels used
+  struct LastChain {
+    void* ev = nullptr;
+    uint64_t squad = 0;
+    uint64_t mask[3] = {0, 0, 0};
+  };
+  std::vector<LastChain> last_chain_;
   void* temporal_stream_ = nullptr;
 
   // logs

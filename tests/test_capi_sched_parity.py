@@ -230,6 +230,21 @@ def test_ablate_out_of_range_rejected():
     assert e.value.status == capi.BL_E_INVALID
 
 
+def test_barrier_out_of_range_rejected():
+    """bl_params.barrier outside 0..1 is BL_E_INVALID at bl_create and at
+    bl_reset (header); 0 and 1 are accepted."""
+    for b in (-1, 2):
+        with pytest.raises(capi.BlessError) as e:
+            capi.Ctx(capi.BL_DEVICE_NONE, clock=capi.BL_CLOCK_VIRTUAL, barrier=b)
+        assert e.value.status == capi.BL_E_INVALID
+    ctx = capi.Ctx(capi.BL_DEVICE_NONE, clock=capi.BL_CLOCK_VIRTUAL, barrier=1)
+    with pytest.raises(capi.BlessError) as e:
+        ctx.reset(capi.default_params(clock=capi.BL_CLOCK_VIRTUAL, barrier=3))
+    assert e.value.status == capi.BL_E_INVALID
+    ctx.reset(capi.default_params(clock=capi.BL_CLOCK_VIRTUAL, barrier=0))
+    ctx.close()
+
+
 @settings(max_examples=150, deadline=None)
 @given(world(), st.integers(0, 10_000))
 def test_predict_matches_oracle_eq1_eq2(tmp_path_factory, w, pseed):

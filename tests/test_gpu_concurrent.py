@@ -64,8 +64,8 @@ def poison(ms):
                 layer.y.fill_(float("nan"))
 
 
-def run_wave(ctx, ms, policy, stagger_ns, squad_max):
-    p = capi.default_params(policy=policy, squad_max=squad_max, split_pct=25)
+def run_wave(ctx, ms, policy, stagger_ns, squad_max, split_pct=25, barrier=0):
+    p = capi.default_params(policy=policy, squad_max=squad_max, split_pct=split_pct, barrier=barrier)
     ctx.reset(p)
     ctx.start()
     base = capi.now_ns() + 2_000_000
@@ -115,11 +115,34 @@ def check_squad_barrier(decisions, launches, res_ns=64):
     return n_pairs
 
 
-@pytest.mark.parametrize("policy", ["BLESS", "BLESS_1thread", "STATIC"])
+def check_range_barrier(decisions, launches, res_ns=64):
+    """bl_params.barrier = 1 (reading R37): a launch of tenant j in squad s+1
+    never starts before the end of another tenant's latest chain whose kernels
+    used a logical SM that j's chain in squad s+1 uses."""
+    last, n_pairs = {}, 0
+    for ls in squads_of(decisions, launches):
+        umask = {}
+        for r in ls:
+            assert r.end_ns > 0 and r.nsm > 0, (r.tenant, r.kernel)
+            umask[r.tenant] = umask.get(r.tenant, 0) | (((1 << (r.hi - r.lo)) - 1) << r.lo)
+        for r in ls:
+            for t, (e, msk) in last.items():
+                if t != r.tenant and msk & umask[r.tenant]:
+                    assert r.start_ns >= e - res_ns, ("range barrier broken", r.tenant, r.kernel, r.start_ns - e)
+                    n_pairs += 1
+        for t, msk in umask.items():
+            last[t] = (max(r.end_ns for r in ls if r.tenant == t), msk)
+    return n_pairs
+
+
+@pytest.mark.parametrize("policy", ["BLESS", "BLESS_1thread", "BLESS_range", "STATIC"])
 def test_concurrent_every_layer_vs_oracle(world, policy):
     cfg, ctx, ms, prof = world
     squad_max = {"C2": 20, "C3": 10, "C4": 10}[cfg]
-    waves = [(0, 11), (60_000, 12)] if policy == "BLESS" else [(0, 21)]
+    # BLESS_range: the SM-range barrier (R37) with strict SP squads (c = 100%),
+    # where chains on disjoint partitions stop waiting for each other
+    split_pct, barrier = (100, 1) if policy == "BLESS_range" else (25, 0)
+    waves = [(0, 11), (60_000, 12)] if policy in ("BLESS", "BLESS_range") else [(0, 21)]
     old = os.environ.get("BLESS_LAUNCH_THREADS")
     if policy == "BLESS_1thread":
         os.environ["BLESS_LAUNCH_THREADS"] = "0"
@@ -127,17 +150,18 @@ def test_concurrent_every_layer_vs_oracle(world, policy):
         for stagger, seed in waves:
             new_inputs(ms, seed)
             poison(ms)
-            decisions, launches = run_wave(ctx, ms, "STATIC" if policy == "STATIC" else "BLESS", stagger, squad_max)
+            decisions, launches = run_wave(ctx, ms, "STATIC" if policy == "STATIC" else "BLESS", stagger, squad_max,
+                                           split_pct, barrier)
             worst = check_all_layers(ms, (cfg, policy, stagger))
             msg = f"\n{cfg} {policy} stagger={stagger}: {sum(len(m.layers) for m in ms)} layers, worst {worst:.2e}"
             if policy != "STATIC":
                 assert decisions
-                pairs = check_squad_barrier(decisions, launches)
+                pairs = (check_range_barrier if barrier else check_squad_barrier)(decisions, launches)
                 sp_sq = sum(1 for d in decisions if d.config_sp)
                 for rec in decisions:
                     got = capi.decision_to_tuple(rec)
                     ref = decide_ref(got["now"], [Active(*a) for a in got["active"]], prof,
-                                     Params(squad_max=squad_max, split_pct=25))
+                                     Params(squad_max=squad_max, split_pct=split_pct))
                     assert got["picks"] == [tuple(p) for p in ref.picks] and got["config"] == ref.config
                 msg += f"; {len(decisions)} squads ({sp_sq} SP), barrier held on {pairs} cross-squad launches"
             for r in launches:

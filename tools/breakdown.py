@@ -26,6 +26,7 @@ def main():
     ap.add_argument("--max-inflight", type=int, default=2)
     ap.add_argument("--squad-max-solo", type=int, default=0)
     ap.add_argument("--lookahead-us", type=float, default=20.0)
+    ap.add_argument("--barrier", type=int, default=0)
     ap.add_argument("--policies", default="BLESS,ISO,STATIC,UNBOUND")
     a = ap.parse_args()
     from paper_conf_eurosys_zhangcc0xz0g25_b200 import build, capi, models
@@ -44,7 +45,7 @@ def main():
             for filt in filts:
                 p = capi.default_params(policy=pol, squad_max=a.squad_max, split_pct=a.split_pct,
                                         max_inflight_squads=a.max_inflight, lookahead_ns=int(a.lookahead_us * 1000),
-                                        squad_max_solo=a.squad_max_solo)
+                                        squad_max_solo=a.squad_max_solo, barrier=a.barrier)
                 ctx.reset(p)
                 ctx.start()
                 ents = [(0, x.tenant, x.arrival_ns) for x in trace if filt is None or x.tenant in filt]
