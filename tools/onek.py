@@ -20,6 +20,7 @@ def main():
     ap.add_argument("dims", type=int, nargs="+")
     ap.add_argument("--launches", type=int, default=0, help="launch N times (no timing) for ncu")
     ap.add_argument("--reps", type=int, default=20)
+    ap.add_argument("--sms", type=int, default=0, help="run on logical SMs [0, sms) (a tenant's range; 0 = all)")
     a = ap.parse_args()
     import torch
 
@@ -43,14 +44,15 @@ def main():
         H, W, C, K, k, s, p = d
         b.conv(b.input((1, H, W, C)), K, k, s, p, act="relu", bn=True)
     ki = ctx.kernel_info(t, 0)
+    sms = a.sms or S
     if a.launches:
         for _ in range(a.launches):
-            ctx.run_kernel(t, 0, 0, S)
+            ctx.run_kernel(t, 0, 0, sms)
         torch.cuda.synchronize()
         print(f"{ki.family.decode()} launched {a.launches}x")
         return
-    ns, dd = ctx.profile_kernel(t, 0, S, a.reps)
-    print(f"{a.kind} {d} {ki.family.decode()} tiles={ki.tiles} d={dd} t={ns / 1e3:.2f}us "
+    ns, dd = ctx.profile_kernel(t, 0, sms, a.reps)
+    print(f"{a.kind} {d} on {sms} SMs {ki.family.decode()} tiles={ki.tiles} d={dd} t={ns / 1e3:.2f}us "
           f"{ki.bytes / ns:.1f} GB/s {ki.flops / ns / 1e3:.1f} TF/s")
 
 
