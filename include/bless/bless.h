@@ -221,7 +221,10 @@ typedef struct {
   int32_t nsm;        /* distinct SMs that processed >= 1 tile; -1 = unknown (a light-exit
                          launch older than the last 2^18 of the run: its stats record was
                          reused, so no times or mask are reported) */
-  int32_t fallback;   /* 1 if no in-range CTA ran and the last CTA did the work */
+  int32_t fallback;   /* bit 0: no in-range CTA ran and the last CTA did the work; bit 1:
+                         lingering out-of-range CTAs helped (linger timeout); bit 2: a
+                         software-dependency wait timed out and fell back to
+                         griddepcontrol.wait (never expected; 0 = clean launch) */
   int64_t start_ns;   /* first tile claimed */
   int64_t end_ns;     /* last CTA exit */
   uint64_t req;

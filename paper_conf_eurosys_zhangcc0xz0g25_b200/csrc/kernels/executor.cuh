@@ -59,7 +59,7 @@ struct __align__(64) SlotStats {
 
 struct __align__(16) DevSlot {  // device memory, zero between launches
   unsigned long long ctr;       // [31:0] claims, [63:32] CTAs done
-  unsigned long long pad;
+  unsigned long long done;      // units finished (software dependency, count_done launches)
 };
 
 
@@ -75,6 +75,15 @@ struct GateArgs {
   int32_t lo, hi;
   uint32_t stamp;          // 1: full exit protocol (last CTA publishes end + seq); 0: light exit
   uint32_t linger_ns;      // bounded wait of out-of-range CTAs (default 30 us; BLESS_LINGER_NS, tests)
+  // Software dependency (tcgen05 GEMM/conv chains): a
+  // count_done launch adds 1 to slot->done after each finished unit (its
+  // stores fenced first); a launch with dep_ctr set waits for its stream
+  // predecessor's counter to reach dep_total instead of griddepcontrol.wait
+  // (the predecessor's last CTA exit, grid completion and memory flush are
+  // off the critical path).
+  const unsigned long long* dep_ctr;
+  uint32_t dep_total;
+  uint32_t count_done;
 };
 
 #ifdef __CUDACC__
@@ -100,6 +109,43 @@ __device__ __forceinline__ bool gate_in_range(const GateArgs& g) {
   return lid >= g.lo && lid < g.hi;
 }
 
+// Wait for the data of the previous kernel on the stream: the software
+// dependency when the predecessor counts its finished units (every lane
+// acquires the counter; the proxy fence orders the TMA loads that follow),
+// else griddepcontrol.wait.  Called by whole warps.
+__device__ __forceinline__ void dep_wait(const GateArgs& g) {
+  if (g.dep_ctr == nullptr) {
+    pdl_wait();
+    return;
+  }
+  // every lane polls (one broadcast load): the loop stays warp-uniform, which
+  // keeps ptxas on the uniform datapath for the TMA/MMA issue around it
+  uint64_t t0 = 0;
+  bool timed_out = false;
+  for (int i = 0;; ++i) {
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(g.dep_ctr) : "memory");
+    if (__all_sync(0xffffffffu, v >= g.dep_total)) break;
+    // safety net: a counter that does not reach its total within 5 ms (a
+    // host bookkeeping error) falls back to the hardware dependency, flagged
+    if ((i & 63) == 63) {
+      const uint64_t now = __shfl_sync(0xffffffffu, ptx_globaltimer(), 0);
+      if (!t0) {
+        t0 = now;
+      } else if (now - t0 > 5000000ull) {
+        timed_out = true;
+        break;
+      }
+    }
+    __nanosleep(32);
+  }
+  if (timed_out) {
+    if ((threadIdx.x & 31) == 0) atomicOr(&g.stats->flags, 4u);
+    pdl_wait();
+  }
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+
 // Claim the next tile (call from ONE thread).  Returns -1 when exhausted.
 // 'marked' tracks whether this CTA already set its SM bit in the mask.
 // The claimer of tile 0 stamps the start, zeroes the slot and the stats
@@ -117,6 +163,7 @@ __device__ __forceinline__ int gate_claim(const GateArgs& g, bool& marked, bool 
     const int64_t now = (int64_t)ptx_globaltimer();
     g.stats->start_gt = now;
     g.slot_ahead->ctr = 0ull;
+    g.slot_ahead->done = 0ull;
     g.stats_ahead->flags = 0u;
     uint4* fm = reinterpret_cast<uint4*>(g.stats_ahead->mask);
     fm[0] = make_uint4(0, 0, 0, 0);
@@ -221,6 +268,7 @@ __device__ __forceinline__ void gate_finalize(const GateArgs& g, bool fallback) 
     if (fallback) atomicOr(&out->flags, 1u);
     if (g.tiles == 0) {   // nothing was claimed: zero ahead here (marker launches)
       g.slot_ahead->ctr = 0ull;
+      g.slot_ahead->done = 0ull;
       g.stats_ahead->flags = 0u;
       uint4* fm = reinterpret_cast<uint4*>(g.stats_ahead->mask);
       fm[0] = make_uint4(0, 0, 0, 0);

@@ -503,6 +503,11 @@ struct TcCfg {
   static constexpr int kSmemMax = kMaxStages * kStageBytes + kFixed;
 };
 
+#ifdef TEST_A
+#define PROD_DEP_WAIT(g) pdl_wait()
+#else
+#define PROD_DEP_WAIT(g) dep_wait(g)
+#endif
 template <int BN, int BK, bool HALO, int MH>
 __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   using Cfg = TcCfg<BN, BK, MH>;
@@ -683,7 +688,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
             if (!dep_waited) {   // weights before the grid dependency resolves, activations after
               tap0 = min(taps, ST);
               for (int tap = 0; tap < tap0; ++tap) load_Bt(c, tap);
-              pdl_wait();
+              PROD_DEP_WAIT(g);
               if (t == 0 && lane == 0) gate_prev_end(g, (int64_t)ptx_globaltimer());
               if (lane == 0) TR(4);
               dep_waited = true;
@@ -704,7 +709,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
             mbar_expect_tx_e(&full[st], kTxBytes);
             if (!kSkipB) load_B(kb0 + i, st);
           }
-          pdl_wait();
+          PROD_DEP_WAIT(g);
           if (t == 0 && lane == 0) gate_prev_end(g, (int64_t)ptx_globaltimer());   // predecessor just completed
           if (lane == 0) TR(4);          // 4: producer past griddepcontrol.wait
           dep_waited = true;
@@ -855,7 +860,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
       }
       asm volatile("bar.sync 2, %0;" ::"n"(32 * kEpiWarps) : "memory");
       if (!dep_waited) {   // residual reads / output writes depend on earlier kernels
-        pdl_wait();
+        dep_wait(g);
         dep_waited = true;
       }
       for (int h = 0; h < MH; ++h) {   // pull this row's residual segment into L2 while the MMAs run
@@ -881,6 +886,13 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty[acc]);
         if (threadIdx.x == 64) TR(7);    // 7: epilogue stores issued (last tile)
+        if (g.count_done) {   // software dependency: this unit's stores, then the count
+          asm volatile("bar.sync 1, %0;" ::"n"(32 * kEpiWarps) : "memory");
+          if (threadIdx.x == 64) {
+            __threadfence();
+            atomicAdd(const_cast<unsigned long long*>(&g.slot->done), 1ull);
+          }
+        }
       } else {
         // split-K: add this unit's partial tile into the fp32 workspace
         // (sub-tile tile*MH + h per M half)
@@ -932,6 +944,13 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
           if (threadIdx.x == 64) {
             p.sem[tile] = 0;
             TR(11);                        // 11: last unit's reduction epilogue done (split-K)
+          }
+        }
+        if (g.count_done) {   // software dependency: partial (or the tile's final stores), then the count
+          asm volatile("bar.sync 1, %0;" ::"n"(32 * kEpiWarps) : "memory");
+          if (threadIdx.x == 64) {
+            __threadfence();
+            atomicAdd(const_cast<unsigned long long*>(&g.slot->done), 1ull);
           }
         }
       }
@@ -1068,6 +1087,7 @@ static bool prep(KernelDesc& d, TcParams& p, std::string& err) {
   }
   d.launch = launch_tc<BN, BK, HALO, MH>;
   d.kernel_fn = (const void*)k_tc_gemm<BN, BK, HALO, MH>;
+  d.counts_done = true;
   return true;
 }
 

@@ -144,6 +144,7 @@ std::unique_ptr<DeviceRT> DeviceRT::create(int device, void* ws, size_t ws_bytes
   if (const char* e = std::getenv("BLESS_PDL")) g_use_pdl = std::atoi(e) != 0;
   rt->linger_ns_ = (uint32_t)kLingerNs;
   if (const char* e = std::getenv("BLESS_LINGER_NS")) rt->linger_ns_ = (uint32_t)std::max(0, std::atoi(e));
+  if (const char* e = std::getenv("BLESS_SWDEP")) rt->swdep_ = std::atoi(e) != 0;
   if (const char* e = std::getenv("BLESS_TC_AUTOTUNE")) rt->autotune_ = std::atoi(e) != 0;
   if (const char* e = std::getenv("BLESS_TC_TUNE_FILE")) {   // "sig bn splits" lines, appended as tuned
     rt->tune_file_ = e;
@@ -399,6 +400,9 @@ GateArgs DeviceRT::make_gate(uint64_t seq, uint32_t tiles, int lo, int hi, bool 
   g.hi = hi;
   g.stamp = stamp ? 1u : 0u;
   g.linger_ns = linger_ns_;
+  g.dep_ctr = nullptr;
+  g.dep_total = 0;
+  g.count_done = 0;
   return g;
 }
 
@@ -415,9 +419,16 @@ uint64_t DeviceRT::launch(int h, int lo, int hi, void* stream, std::string& err,
 }
 
 bool DeviceRT::launch_seq(int h, uint64_t seq, int lo, int hi, void* stream, std::string& err, bool stamp,
-                          uint64_t prev_light) {
+                          uint64_t prev_light, uint64_t dep_seq, uint32_t dep_total) {
   const KernelDesc& kd = *kernels_[h];
-  const GateArgs g = make_gate(seq, kd.tiles, lo, hi, stamp, prev_light);
+  GateArgs g = make_gate(seq, kd.tiles, lo, hi, stamp, prev_light);
+  if (counts(h)) {
+    g.count_done = 1u;
+    if (dep_seq) {
+      g.dep_ctr = &(reinterpret_cast<DevSlot*>(slots_) + dep_seq % ring_)->done;
+      g.dep_total = dep_total;
+    }
+  }
   const cudaError_t e = kd.launch(kd, g, (cudaStream_t)stream);
   if (e != cudaSuccess) {
     err = std::string("launch ") + kd.family + ": " + cudaGetErrorString(e);
@@ -554,12 +565,15 @@ bool DeviceRT::chain_time(const std::vector<int>& hs, int lo, int hi, int graph,
   std::vector<int64_t> dv, hv;
   const int n = (int)hs.size();
   auto enqueue = [&]() -> bool {
-    uint64_t prev = 0;
+    uint64_t prev = 0, dep = 0;
+    uint32_t dep_tot = 0;
     for (int k = 0; k < n; ++k) {
       const bool stamp = k == 0 || k == n - 1;
       const uint64_t seq = alloc_seq();
-      if (!launch_seq(hs[k], seq, lo, hi, s, err, stamp, prev)) return false;
+      if (!launch_seq(hs[k], seq, lo, hi, s, err, stamp, prev, dep, dep_tot)) return false;
       prev = stamp ? 0 : seq;
+      dep = counts(hs[k]) ? seq : 0;
+      dep_tot = kernels_[hs[k]]->tiles;
     }
     return true;
   };
@@ -671,7 +685,7 @@ void DeviceRT::peek(uint64_t seq, LaunchStats* out) {
   int nsm = 0;
   for (int i = 0; i < 8; ++i) nsm += __builtin_popcount(s->mask[i]);
   out->nsm = nsm;
-  out->fallback = (int)(s->flags & 3u);
+  out->fallback = (int)(s->flags & 7u);
   for (int i = 0; i < 8; ++i) out->mask[i] = s->mask[i];
 }
 
@@ -686,7 +700,7 @@ bool DeviceRT::poll(uint64_t seq, LaunchStats* out) {
     int nsm = 0;
     for (int i = 0; i < 8; ++i) nsm += __builtin_popcount(s->mask[i]);
     out->nsm = nsm;
-    out->fallback = (int)(s->flags & 3u);  // bit0: last-CTA fallback, bit1: lingering CTAs helped
+    out->fallback = (int)(s->flags & 7u);  // bit0: last-CTA fallback, bit1: lingering CTAs helped, bit2: software dependency timed out
     for (int i = 0; i < 8; ++i) out->mask[i] = s->mask[i];
   }
   return true;
@@ -748,14 +762,23 @@ bool DeviceRT::profile(int h, int sm_count, int reps, void* stream, int64_t* ns_
     std::sort(ds, ds + 5);
     *d_out = ds[2];
   }
-  // timed launches use the light exit, as a request's middle kernels do
+  // timed launches use the light exit and the software dependency, as a
+  // request's middle kernels do
+  uint64_t prev = 0;
+  const uint32_t tot = kernels_[h]->tiles;
+  auto one = [&]() -> bool {
+    const uint64_t q = alloc_seq();
+    if (!launch_seq(h, q, 0, sm_count, s, err, false, 0, counts(h) ? prev : 0, tot)) return false;
+    prev = q;
+    return true;
+  };
   for (int w = 0; w < 2; ++w)
-    if (!launch(h, 0, sm_count, s, err, false)) return false;
+    if (!one()) return false;
   float ms[3];
   for (int b = 0; b < 3; ++b) {
     RT_CHECK(cudaEventRecord(e0, s));
     for (int r = 0; r < reps; ++r)
-      if (!launch(h, 0, sm_count, s, err, false)) return false;
+      if (!one()) return false;
     RT_CHECK(cudaEventRecord(e1, s));
     RT_CHECK(cudaEventSynchronize(e1));
     RT_CHECK(cudaEventElapsedTime(&ms[b], e0, e1));

@@ -73,8 +73,16 @@ class DeviceRT {
   // Parallel launch (Engine launcher threads): the scheduler thread allocates
   // the launch's seq; any thread may then launch it on its own stream.
   uint64_t alloc_seq() { return ++seq_; }
+  // dep_seq / dep_total: the stream predecessor's seq and unit count when that
+  // launch counted its units (counts() of its handle) -- this launch then
+  // waits on its counter instead of griddepcontrol.wait if counts(h);
+  // dep_seq = 0: hardware wait.
   bool launch_seq(int h, uint64_t seq, int lo, int hi, void* stream, std::string& err, bool stamp = true,
-                  uint64_t prev_light = 0);
+                  uint64_t prev_light = 0, uint64_t dep_seq = 0, uint32_t dep_total = 0);
+  // Software dependency: launches of kernel h count their
+  // finished units and can wait on a counting predecessor.  Opt-in
+  // (BLESS_SWDEP=1): correct on B200 but not faster than griddepcontrol.wait.
+  bool counts(int h) const { return swdep_ && kernels_[h]->counts_done; }
   bool launch_marker_seq(uint64_t seq, void* stream, std::string& err);
 
   // Streams / events (thin wrappers so the engine does not include CUDA headers).
@@ -119,6 +127,7 @@ class DeviceRT {
   bool identity_map_ = true;
   uint64_t seq_ = 0;
   uint32_t linger_ns_ = 30000;   // GateArgs::linger_ns (BLESS_LINGER_NS)
+  bool swdep_ = false;           // BLESS_SWDEP=1 enables (measured no gain on B200)
   uint64_t ring_ = kSlotRingDefault;
   uint64_t ahead_ = kSlotRingDefault / 2;
   std::vector<std::unique_ptr<KernelDesc>> kernels_;

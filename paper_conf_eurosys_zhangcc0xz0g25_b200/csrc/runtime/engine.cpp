@@ -251,13 +251,17 @@ bl_status Engine::profile_tenant(int t, int reps, std::string& err) {
     for (int r = 0; r < runs + 1; ++r) {   // run 0 warms up
       if (!rt_->device_sync()) { err = "device error before the tau run"; return BL_E_CUDA; }
       std::vector<uint64_t> seqs(m);
-      uint64_t prev_light = 0;
+      uint64_t prev_light = 0, dep = 0;
+      uint32_t dep_tot = 0;
       for (int k = 0; k < m; ++k) {
         const bool stamp = k == 0 || k == m - 1;
+        const int h = ten_[t].handles[k];
         seqs[k] = rt_->alloc_seq();
-        if (!rt_->launch_seq(ten_[t].handles[k], seqs[k], 0, q, ten_[t].stream, err, stamp, prev_light))
+        if (!rt_->launch_seq(h, seqs[k], 0, q, ten_[t].stream, err, stamp, prev_light, dep, dep_tot))
           return BL_E_CUDA;
         prev_light = stamp ? 0 : seqs[k];
+        dep = rt_->counts(h) ? seqs[k] : 0;
+        dep_tot = rt_->kernel(h).tiles;
       }
       if (!rt_->device_sync()) { err = "device error in the tau run"; return BL_E_CUDA; }
       if (r == 0) continue;
@@ -396,6 +400,8 @@ bl_status Engine::start(std::string& err) {
     ten_[j].lo = lo;
     ten_[j].hi = lo + prof_.ten[j].quota_sms;
     lo = ten_[j].hi;
+    ten_[j].prev_light = 0;   // no stream predecessor from before this run (its ring records may be reused)
+    ten_[j].dep_seq = 0;
   }
   if (!rt_ && prm_.policy != BL_POLICY_BLESS) { err = "device-less ctx runs the BLESS policy only"; return BL_E_STATE; }
   if (!rt_ && prm_.clock != BL_CLOCK_VIRTUAL) { err = "device-less ctx needs the VIRTUAL clock"; return BL_E_STATE; }
@@ -808,14 +814,20 @@ uint64_t Engine::launch_one(int t, int k, int lo, int hi, void* stream, int64_t 
       fail("H2D input copy failed");
       return 0;
     }
-    if (own) tr.prev_light = 0;
+    if (own) tr.prev_light = 0, tr.dep_seq = 0;
   }
   const uint64_t seq = rt_->alloc_seq();
-  if (!rt_->launch_seq(tr.handles[k], seq, lo, hi, stream, err, stamp, own ? tr.prev_light : 0)) {
+  const int h = tr.handles[k];
+  if (!rt_->launch_seq(h, seq, lo, hi, stream, err, stamp, own ? tr.prev_light : 0, own ? tr.dep_seq : 0,
+                       tr.dep_tot)) {
     fail(err);
     return 0;
   }
-  if (own) tr.prev_light = stamp ? 0 : seq;
+  if (own) {
+    tr.prev_light = stamp ? 0 : seq;
+    tr.dep_seq = rt_->counts(h) ? seq : 0;
+    tr.dep_tot = rt_->kernel(h).tiles;
+  }
   bl_launch_rec rec{};
   rec.seq = seq;
   rec.tenant = t;
@@ -841,7 +853,7 @@ uint64_t Engine::launch_one(int t, int k, int lo, int hi, void* stream, int64_t 
       fail(err);
       return 0;
     }
-    if (own) tr.prev_light = 0;
+    if (own) tr.prev_light = 0, tr.dep_seq = 0;
     pending_.push_back({seq, idx, req, k, 0});
     pending_.push_back({mseq, (size_t)-1, req, -1, 1});
     return seq;
@@ -887,11 +899,15 @@ bool Engine::prepare_one(int t, int k, int lo, int hi, int64_t req, bool last, s
 bool Engine::exec_items(int t, const std::vector<LaunchItem>& items, void* stream, std::string& err) {
   TenantRT& tr = ten_[t];
   for (const LaunchItem& it : items) {
-    if (it.kind != LaunchItem::KERNEL) tr.prev_light = 0;
+    if (it.kind != LaunchItem::KERNEL) tr.prev_light = 0, tr.dep_seq = 0;
     switch (it.kind) {
       case LaunchItem::KERNEL:
-        if (!rt_->launch_seq(it.handle, it.seq, it.lo, it.hi, stream, err, it.stamp != 0, tr.prev_light)) return false;
+        if (!rt_->launch_seq(it.handle, it.seq, it.lo, it.hi, stream, err, it.stamp != 0, tr.prev_light, tr.dep_seq,
+                             tr.dep_tot))
+          return false;
         tr.prev_light = it.stamp ? 0 : it.seq;
+        tr.dep_seq = rt_->counts(it.handle) ? it.seq : 0;
+        tr.dep_tot = rt_->kernel(it.handle).tiles;
         break;
       case LaunchItem::H2D:
         if (!rt_->memcpy_async(tr.dev_in, tr.host_in, tr.in_bytes, stream)) { err = "H2D input copy failed"; return false; }

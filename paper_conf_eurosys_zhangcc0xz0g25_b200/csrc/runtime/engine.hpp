@@ -44,6 +44,8 @@ struct TenantRT {
   void* host_out = nullptr;
   size_t out_bytes = 0;
   uint64_t prev_light = 0;   // last launch on the stream if it used the light exit (owned by its launcher)
+  uint64_t dep_seq = 0;      // last launch on the stream if it counted its units (software dependency), else 0
+  uint32_t dep_tot = 0;      //   and its unit count
 };
 
 // Parallel launch path.  Host launch calls cost ~3 us each on the B200 boxes

@@ -32,6 +32,7 @@ struct KernelDesc {
   const void* kernel_fn = nullptr;  // for the occupancy query (grid = S x blocks/SM)
   void* owned = nullptr;   // device scratch owned by this kernel (split-K workspace), cudaFree'd with it
   int choice_bn = 0, choice_splits = 0, choice_bk = 0, choice_halo = 0, choice_mt = 0;  // tcgen05 tile config (0 = not tc)
+  bool counts_done = false;  // can count finished units / wait on a predecessor's count (GateArgs dep_*)
   alignas(128) unsigned char params[4096];  // family-specific parameter block
 };
 
