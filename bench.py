@@ -433,20 +433,24 @@ def roofline_of(rep, launches_all, peaks, args):
         if r.end_ns > r.start_ns and r.nsm > 0 and fam_of.get((r.tenant, r.kernel)) == fam:
             rng.setdefault((r.tenant, r.kernel), []).append(r.hi - r.lo)
     Fr = Tr = Pr = 0.0
+    tensor = bound == "tensor"
     for tk, sizes in rng.items():
         s_med = int(np.median(sizes))
         ki = ctx.kernel_info(*tk)
         ev, _ = ctx.profile_kernel(tk[0], tk[1], s_med, reps=10)
         n = nlaunch[tk]
-        Fr += n * ki.flops
+        Fr += n * (ki.flops if tensor else ki.bytes)
         Tr += n * ev
-        Pr += n * ev * (tc_peak * s_med / S)   # time-weighted share of the peak
+        Pr += n * ev * ((tc_peak if tensor else hbm_peak) * s_med / S)   # time-weighted share of the peak
     if Tr > 0:
         peak_share = Pr / Tr
-        roof["at_range"] = {"achieved": Fr / Tr / 1e3, "peak_share": peak_share, "unit": "TFLOP/s",
-                            "frac": Fr / Tr / 1e3 / peak_share,
+        ach = Fr / Tr / 1e3 if tensor else Fr / Tr
+        roof["at_range"] = {"achieved": ach, "peak_share": peak_share, "unit": unit,
+                            "frac": ach / peak_share,
                             "note": "each layer timed on its median SM range in the timed steps; peak = "
-                                    "measured bf16 peak x s/S, time-weighted"}
+                                    f"measured {'bf16' if tensor else 'HBM'} peak x s/S, time-weighted"
+                                    + ("" if tensor else " (HBM is not partitioned by SMs: a share can "
+                                                         "exceed 1, SURVEY §8(d))")}
     hb = [tk for tk in busy if (lambda k: k.flops / max(k.bytes, 1.0) < ridge)(ctx.kernel_info(*tk))]
     if hb:
         tk = max(hb, key=lambda x: busy[x] / nlaunch[x])
