@@ -1088,15 +1088,25 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
   // will use -- per SM the squads still run one after the other, but a chain
   // no longer waits for chains on SMs it does not touch.
   const int nt = nten();
-  std::vector<std::array<uint64_t, 3>> umask(nt, std::array<uint64_t, 3>{0, 0, 0});
-  for (const Pick& p : d.picks)
-    for (int x = p.lo; x < p.hi && x < 192; ++x) umask[p.tenant][x >> 6] |= 1ull << (x & 63);
-  std::vector<std::vector<int>> wparts(nt);
-  std::vector<std::vector<void*>> wevs(nt);
-  std::vector<std::vector<uint64_t>> wsqs(nt);
-  if ((int)last_chain_.size() != nt) last_chain_.assign(nt, LastChain{});
-  for (int j : d.parts) {
-    if (prm_.barrier == 1) {
+  const bool rbar = prm_.barrier == 1;
+  // (the paper-literal barrier keeps the scheduler thread's per-squad work
+  // minimal: no masks, no per-participant lists)
+  std::vector<std::array<uint64_t, 3>> umask(rbar ? nt : 0, std::array<uint64_t, 3>{0, 0, 0});
+  std::vector<std::vector<int>> wparts(rbar ? nt : 0);
+  std::vector<std::vector<void*>> wevs(rbar ? nt : 0);
+  std::vector<std::vector<uint64_t>> wsqs(rbar ? nt : 0);
+  if (rbar) {
+    auto setbits = [](std::array<uint64_t, 3>& m, int lo, int hi) {
+      for (int w = 0; w < 3; ++w) {
+        const int a = std::max(lo, 64 * w), b = std::min(hi, 64 * w + 64);
+        if (a < b) m[w] |= (b - a == 64 ? ~0ull : ((1ull << (b - a)) - 1)) << (a - 64 * w);
+      }
+    };
+    for (const Pick& p : d.picks) setbits(umask[p.tenant], p.lo, p.hi);
+    if ((int)last_chain_.size() != nt) last_chain_.assign(nt, LastChain{});
+  }
+  if (rbar)
+    for (int j : d.parts)
       for (int l = 0; l < nt; ++l) {
         const LastChain& c = last_chain_[l];
         if (l == j || !c.ev) continue;
@@ -1106,18 +1116,14 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
         wevs[j].push_back(c.ev);
         wsqs[j].push_back(c.squad);
       }
-    } else {
-      for (size_t i = 0; i < prev_events_.size(); ++i) {   // own stream: already ordered (see launcher_main)
-        if (i < prev_parts_.size() && prev_parts_[i] == j) continue;
-        wparts[j].push_back(i < prev_parts_.size() ? prev_parts_[i] : -1);
-        wevs[j].push_back(prev_events_[i]);
-        wsqs[j].push_back(prev_squad_);
-      }
-    }
-  }
   if (launchers_.empty()) {   // single launch thread (BLESS_LAUNCH_THREADS=0)
     for (int j : d.parts) {
-      for (void* e : wevs[j]) rt_->stream_wait(ten_[j].stream, e);
+      if (rbar) {
+        for (void* e : wevs[j]) rt_->stream_wait(ten_[j].stream, e);
+      } else {
+        for (size_t i = 0; i < prev_events_.size(); ++i)   // own stream: already ordered (see launcher_main)
+          if (i >= prev_parts_.size() || prev_parts_[i] != j) rt_->stream_wait(ten_[j].stream, prev_events_[i]);
+      }
       ten_[j].prev_light = 0;
     }
     for (size_t i = 0; i < d.picks.size(); ++i) {
@@ -1131,10 +1137,16 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
   if (!launchers_.empty()) {
     for (int j : d.parts) {
       jobs[j].squad = sq;
-      jobs[j].wait_squad = wparts[j].empty() ? 0 : 1;
-      jobs[j].wait_parts = wparts[j];
-      jobs[j].wait_sq = wsqs[j];
-      jobs[j].wait_events = wevs[j];
+      if (rbar) {
+        jobs[j].wait_squad = wparts[j].empty() ? 0 : 1;
+        jobs[j].wait_parts = std::move(wparts[j]);
+        jobs[j].wait_sq = std::move(wsqs[j]);
+        jobs[j].wait_events = std::move(wevs[j]);
+      } else {
+        jobs[j].wait_squad = prev_squad_;
+        jobs[j].wait_parts = prev_parts_;
+        jobs[j].wait_events = prev_events_;
+      }
     }
     for (size_t i = 0; i < d.picks.size(); ++i) {
       const Pick& p = d.picks[i];
@@ -1155,7 +1167,7 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
   }
   for (int j : d.parts)
     if (!launchers_.empty()) push_job(j, std::move(jobs[j]));
-  for (size_t i = 0; i < d.parts.size(); ++i) {
+  for (size_t i = 0; rbar && i < d.parts.size(); ++i) {
     LastChain& c = last_chain_[d.parts[i]];
     c.ev = inf.events[i];
     c.squad = sq;

@@ -228,3 +228,45 @@ def test_linger_steal_path_exact(lib_built, monkeypatch):
             assert err <= tol, (m.name, k, err)
     print(f"\nsteal path: {steals}/{len(recs)} launches helped by out-of-range CTAs, outputs exact")
     ctx.close()
+
+
+def test_stats_ring_wraps_without_stale_records(lib_built, tmp_path, monkeypatch):
+    """A run with more launches than the stats-ring window (ADVICE round 1:
+    records older than ahead() launches are reused): with a 2^10 ring (ahead =
+    512) and ~1,500 launches every request still completes, every launch whose
+    record is reported has its SM mask inside its range and no fallback, and
+    light launches older than the window are reported as unknown (nsm = -1,
+    no times) instead of from a reused record."""
+    monkeypatch.setenv("BLESS_STATS_RING_LOG2", "10")
+    ctx = capi.Ctx(0, squad_max=4)
+    ms = models.build_config(ctx, "C1", "fp32")
+    for m in ms:
+        ctx.profile_tenant(m.tenant, reps=2)
+    path = str(tmp_path / "c1.profile")
+    ctx.save_profile(path)
+    prof = Prof(sp.load(path))
+    trace = tr.poisson([2.0 * prof.T[0], 2.0 * prof.T[1]], 320, seed=3)   # 320 requests, 1,600 launches
+    ctx.start()
+    ids = _run_trace(ctx, trace, capi.now_ns() + 2_000_000)
+    ctx.drain(int(60e9))
+    ctx.stop()
+    for r in ids:
+        st, info = ctx.poll(r)
+        assert st == capi.BL_OK and info.finish_ns > info.arrival_ns
+    recs = ctx.launches()
+    assert len(recs) > 1024
+    known = [r for r in recs if r.nsm > 0]
+    unknown = [r for r in recs if r.nsm < 0]
+    assert unknown, "no launch fell out of the 512-launch window"
+    assert all(r.start_ns == 0 and r.end_ns == 0 for r in unknown)
+    for r in known:
+        bits = mask_bits(r)
+        assert bits and all(r.lo <= b < r.hi for b in bits) and r.fallback == 0 and r.end_ns >= r.start_ns
+    # first and last kernels of every request publish their stamps (full exit
+    # protocol) and are harvested during the run, whatever their age
+    m_of = [len(m.layers) for m in ms]
+    for r in recs:
+        if r.kernel == 0 or r.kernel == m_of[r.tenant] - 1:
+            assert r.nsm > 0, (r.tenant, r.kernel, r.seq)
+    print(f"\n{len(recs)} launches, {len(known)} reported, {len(unknown)} older light launches unknown")
+    ctx.close()
