@@ -46,7 +46,7 @@ CONFIG_NAMES = {"C1": "tiny MLP (1/3) + tiny CNN (2/3), fp32",
                 "C3": "ResNet50 (0.4) + VGG16 (0.3) + BERT-base s128 (0.2) + MobileNetV2 (0.1), bf16 batch 1",
                 "C4": "BERT-large s384 (1/2) + ResNet152 (1/4) + DenseNet121 (1/4), bf16 batch 1, bursty",
                 "C5": "per-GPU mix of C2/C3/C4 (GPU g hosts C[2 + g mod 3])"}
-SQUAD_MAX = {"C1": 4, "C2": 20, "C3": 50, "C4": 10}   # C3: the paper's testbed value (L408); B200 A/B in profiles/round2/smax_defaults
+SQUAD_MAX = {"C1": 4, "C2": 40, "C3": 50, "C4": 10}   # C3: the paper's testbed value (L408); B200 A/B in profiles/round2/smax_defaults
 
 # tenant (name, quota) per config -- data only, so the reference arm imports
 # nothing from the product package
@@ -72,7 +72,7 @@ def parse():
     # B200 operating point chosen by the c% x S_max sweep, the
     # way the paper picks its own empirically (§6.7).
     ap.add_argument("--squad-max", type=int, default=None,
-                    help="S_max (L406-L408); default per config from the B200 sweeps: C1 4, C2 20, C3 50, C4 10")
+                    help="S_max (L406-L408); default per config from the B200 sweeps: C1 4, C2 40, C3 50, C4 10")
     ap.add_argument("--split-pct", type=int, default=25)
     ap.add_argument("--squad-max-solo", type=int, default=0,
                     help="reading R36: cap of a squad with a single active request (0 = S_max)")
