@@ -12,6 +12,7 @@
 
 #include <cstdint>
 #include <cstdio>
+#include <string>
 #include <vector>
 
 struct __align__(64) Maps {
@@ -149,7 +150,7 @@ __global__ void k_tma_pc(const __grid_constant__ Maps mp, int ST, int nbox, int 
 // 58-pixel-wide halo at row offset r*58 + s (not 8-row aligned), B from a
 // 3-tap weight stage; fill: 0 = zeros, 1 = bf16 ones.
 template <int BN>
-__global__ void k_mma_rate(int n, int elect, unsigned long long* out, int pattern = 0, int fill = 0) {
+__global__ void k_mma_rate(int n, int elect, unsigned long long* out, int pattern = 0, int fill = 0, int accs = 1) {
   extern __shared__ __align__(1024) unsigned char sm_raw[];
   unsigned char* sm = (unsigned char*)(((uintptr_t)sm_raw + 1023) & ~(uintptr_t)1023);
   __shared__ uint64_t bar;
@@ -185,10 +186,12 @@ __global__ void k_mma_rate(int n, int elect, unsigned long long* out, int patter
         ao += (uint32_t)(r * 58 + s_) * 128u;
         bo += (uint32_t)s_ * (BN * 128u);
       }
+      // accs > 1: consecutive MMAs rotate over independent TMEM accumulators
+      const int acc = accs > 1 ? i % accs : 0;
       asm volatile(
           "{\n\t.reg .pred p, e;\n\telect.sync _|e, 0xffffffff;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-          "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tm),
-          "l"(desc(a + ao)), "l"(desc(b + bo)), "r"(idesc), "r"(i)
+          "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tm + (uint32_t)(acc * BN)),
+          "l"(desc(a + ao)), "l"(desc(b + bo)), "r"(idesc), "r"(i >= accs ? 1 : 0)
           : "memory");
     }
     asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
@@ -314,7 +317,8 @@ typedef CUresult (*Enc)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, co
                         const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
                         CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
 
-int main() {
+int main(int argc, char** argv) {
+  const bool only_accs = argc > 1 && std::string(argv[1]) == "accs";
   void* fn = nullptr;
   cudaDriverEntryPointQueryResult q;
   cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q);
@@ -355,6 +359,30 @@ int main() {
        {(cuuint64_t)C * 2, (cuuint64_t)W * C * 2, 128}, {16, 64, 2, 1}, 1, H / 2, 8},
   };
   printf("S=%d sm_clock=%d MHz\n", S, clk_khz / 1000);
+  {  // MMA rate vs independent accumulators (is the ~60-cycle floor of N <= 64 a dependency chain?)
+    for (int bn : {32, 64, 128}) {
+      const void* kf = bn == 32 ? (const void*)k_mma_rate<32>
+                                : (bn == 64 ? (const void*)k_mma_rate<64> : (const void*)k_mma_rate<128>);
+      cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+      for (int accs : {1, 2, 4}) {
+        if (accs * bn > 256) continue;
+        const int n = 2048;
+        for (int rep = 0; rep < 2; ++rep) {
+          if (bn == 32) k_mma_rate<32><<<S, 32, 160 * 1024>>>(n, 1, d_out, 0, 0, accs);
+          else if (bn == 64) k_mma_rate<64><<<S, 32, 160 * 1024>>>(n, 1, d_out, 0, 0, accs);
+          else k_mma_rate<128><<<S, 32, 160 * 1024>>>(n, 1, d_out, 0, 0, accs);
+        }
+        cudaError_t e = cudaDeviceSynchronize();
+        if (e != cudaSuccess) { printf("mma: %s\n", cudaGetErrorString(e)); return 1; }
+        cudaMemcpy(h.data(), d_out, S * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
+        double avg = 0;
+        for (int i = 0; i < S; ++i) avg += (double)h[i] / S;
+        printf("MMA 128x%dx16 over %d accumulator(s): %.1f ns/mma = %.1f cycles (floor %d)\n", bn, accs, avg / n,
+               avg / n * clk_khz / 1e6, 128 * bn / 256);
+      }
+    }
+  }
+  if (only_accs) return 0;
   // MMA issue rate
   for (int elect = 0; elect < 2; ++elect) {
     for (int bn : {64, 128, 256}) {
