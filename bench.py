@@ -79,8 +79,8 @@ def parse():
     ap.add_argument("--ablate", type=int, default=0,
                     help="PAPER.md §6.8 ablation (R32): 1 = no multi-task scheduler, 2 = no determiner, 3 = both")
     ap.add_argument("--barrier", type=int, default=0,
-                    help="squad barrier: 0 = every participant waits for the previous squad (L276); "
-                         "1 = SM-range barrier (reading R37)")
+                    help="squad barrier bits: 0 = every participant waits for the previous squad (L276); "
+                         "1 = SM-range barrier (reading R37); 2 = arrivals join in-flight solo NSP squads (R38)")
     ap.add_argument("--lookahead-us", type=float, default=20.0)
     ap.add_argument("--dump-squads", type=int, default=0,
                     help="write the first N squads of the timed steps (picks, ranges, predicted vs measured) to out-dir")
@@ -166,7 +166,8 @@ def squad_timeline(decisions, launches, m_of=None, S=148, barrier=0):
     # squad shape (a squad closes at S_max picks or on a
     # request's last kernel) and SM-time busy fraction inside squads
     npk, npt, by_last, sm_busy, sm_span = [], [], 0, 0.0, 0.0
-    last = {}   # barrier = 1: tenant -> (end of its latest chain, SM mask of that chain)
+    last = {}   # barrier bit 0: tenant -> (end of its latest chain, SM mask of that chain)
+    prev_solo = False
     for d in decisions:
         ls = launches[i:i + d.n_picks]
         i += d.n_picks
@@ -181,7 +182,11 @@ def squad_timeline(decisions, launches, m_of=None, S=148, barrier=0):
         spans.append((min(r.start_ns for r in ls), max(r.end_ns for r in ls), d.t_hat, bool(d.config_sp)))
         sm_busy += sum((r.end_ns - r.start_ns) * r.nsm for r in ls)
         sm_span += (spans[-1][1] - spans[-1][0]) * S
-        if barrier == 1:
+        # R38 (barrier bit 2): a squad that follows a solo NSP squad may have
+        # been decided at an arrival and started beside it -- not checked
+        exempt = bool(barrier & 2) and prev_solo
+        prev_solo = d.n_part == 1 and not d.config_sp
+        if barrier & 1:
             # SM-range barrier (R37): no launch starts before the end of another
             # tenant's latest chain whose kernels used any SM this tenant's
             # chain in this squad uses
@@ -190,11 +195,11 @@ def squad_timeline(decisions, launches, m_of=None, S=148, barrier=0):
                 umask[r.tenant] = umask.get(r.tenant, 0) | (((1 << (r.hi - r.lo)) - 1) << r.lo)
             for r in ls:
                 for t, (e, msk) in last.items():
-                    if t != r.tenant and msk & umask[r.tenant]:
+                    if t != r.tenant and msk & umask[r.tenant] and not exempt:
                         viol += int(r.start_ns < e - 64)
             for t, msk in umask.items():
                 last[t] = (max(r.end_ns for r in ls if r.tenant == t), msk)
-        elif prev is not None:   # barrier: no launch starts before ANOTHER tenant's squad-s end
+        elif prev is not None and not exempt:   # barrier: no launch starts before ANOTHER tenant's squad-s end
             for r in ls:
                 others = [e for t, e in prev.items() if t != r.tenant]
                 viol += int(bool(others) and r.start_ns < max(others) - 64)

@@ -113,13 +113,17 @@ typedef struct {
                                  single active request closes after min(squad_max,
                                  squad_max_solo) kernels, bounding how long an arrival
                                  waits for the next decision; 0 = squad_max (default). */
-  int32_t barrier;            /* squad barrier (BLESS policy).  0 (default): every
-                                 participant of squad s+1 waits for every other participant
-                                 of squad s.  1 (reading R37): a participant's
-                                 chain waits for the latest in-flight chain of every other
-                                 tenant whose kernels ran on logical SMs its own kernels
-                                 will use, so on every SM the squads still run one after
-                                 the other.  BL_E_INVALID outside 0..1 at bl_create. */
+  int32_t barrier;            /* squad barrier (BLESS policy), bit flags.  0 (default):
+                                 every participant of squad s+1 waits for every other
+                                 participant of squad s.  Bit 0 (reading R37):
+                                 a participant's chain waits for the latest in-flight chain
+                                 of every other tenant whose kernels ran on logical SMs its
+                                 own kernels will use, so on every SM the squads still run
+                                 one after the other.  Bit 1 (reading R38, L57): a request
+                                 that arrives while the GPU runs only another tenant's solo
+                                 NSP squads is decided at once and its squad does not wait
+                                 for them (the solo kernels keep running and share the SMs).
+                                 BL_E_INVALID outside 0..3 at bl_create / bl_reset. */
 } bl_params;
 
 /* Fill *p with the defaults listed above. */

@@ -44,7 +44,7 @@ Engine::~Engine() {
 bl_status Engine::init(void* ws, size_t ws_bytes, std::string& err) {
   if (prm_.sm_unit < 1 || prm_.squad_max < 1 || prm_.squad_max > BL_MAX_SQUAD || prm_.split_pct < 0 ||
       prm_.ablate < 0 || prm_.ablate > 3 || prm_.squad_max_solo < 0 || prm_.squad_max_solo > BL_MAX_SQUAD ||
-      prm_.split_pct > 100 || prm_.max_requests < 1 || prm_.barrier < 0 || prm_.barrier > 1) {
+      prm_.split_pct > 100 || prm_.max_requests < 1 || prm_.barrier < 0 || prm_.barrier > 3) {
     err = "invalid bl_params";
     return BL_E_INVALID;
   }
@@ -559,7 +559,7 @@ bl_status Engine::reset(const bl_params* p, std::string& err) {
   if (st != BL_OK && st != BL_E_CUDA) return st;
   if (p) {
     if (p->max_requests != prm_.max_requests) { err = "max_requests cannot change on reset"; return BL_E_INVALID; }
-    if (p->barrier < 0 || p->barrier > 1) { err = "invalid bl_params.barrier"; return BL_E_INVALID; }
+    if (p->barrier < 0 || p->barrier > 3) { err = "invalid bl_params.barrier"; return BL_E_INVALID; }
     prm_ = *p;
     prof_.g = prm_.sm_unit;
     prof_.derive();
@@ -1067,7 +1067,16 @@ void Engine::thread_main() {
 }
 
 // BLESS: squads on the event-barriered tenant streams (§4.3-§4.5).
-void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req, const std::vector<int>& act_next) {
+int Engine::solo_inflight_tenant() const {
+  if (inflight_.empty()) return -1;
+  const int l = inflight_.front().parts.empty() ? -1 : inflight_.front().parts[0];
+  for (const Inflight& f : inflight_)
+    if (!f.solo_nsp || f.parts.size() != 1 || f.parts[0] != l) return -1;
+  return l;
+}
+
+void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req, const std::vector<int>& act_next,
+                          bool join_solo) {
   (void)act_next;
   // Squad barrier: every participant waits for the previous squad's kernels
   // (the paper synchronises after each squad, L276; here a GPU-side event
@@ -1088,7 +1097,7 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
   // will use -- per SM the squads still run one after the other, but a chain
   // no longer waits for chains on SMs it does not touch.
   const int nt = nten();
-  const bool rbar = prm_.barrier == 1;
+  const bool rbar = (prm_.barrier & 1) != 0;
   // (the paper-literal barrier keeps the scheduler thread's per-squad work
   // minimal: no masks, no per-participant lists)
   std::vector<std::array<uint64_t, 3>> umask(rbar ? nt : 0, std::array<uint64_t, 3>{0, 0, 0});
@@ -1116,9 +1125,15 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
         wevs[j].push_back(c.ev);
         wsqs[j].push_back(c.squad);
       }
+  if (join_solo) {   // R38: the arrival does not wait for the in-flight solo squads
+    for (auto& w : wparts) w.clear();
+    for (auto& w : wevs) w.clear();
+    for (auto& w : wsqs) w.clear();
+  }
   if (launchers_.empty()) {   // single launch thread (BLESS_LAUNCH_THREADS=0)
     for (int j : d.parts) {
-      if (rbar) {
+      if (join_solo) {
+      } else if (rbar) {
         for (void* e : wevs[j]) rt_->stream_wait(ten_[j].stream, e);
       } else {
         for (size_t i = 0; i < prev_events_.size(); ++i)   // own stream: already ordered (see launcher_main)
@@ -1137,7 +1152,9 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
   if (!launchers_.empty()) {
     for (int j : d.parts) {
       jobs[j].squad = sq;
-      if (rbar) {
+      if (join_solo) {
+        jobs[j].wait_squad = 0;
+      } else if (rbar) {
         jobs[j].wait_squad = wparts[j].empty() ? 0 : 1;
         jobs[j].wait_parts = std::move(wparts[j]);
         jobs[j].wait_sq = std::move(wsqs[j]);
@@ -1158,6 +1175,7 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
   Inflight inf;
   inf.squad = sq;
   inf.parts = d.parts;
+  inf.solo_nsp = d.parts.size() == 1 && !d.sp;
   for (int j : d.parts) {
     TenantRT& t = ten_[j];
     void* ev = t.events[t.ev_next++ % t.events.size()];
@@ -1188,6 +1206,7 @@ void Engine::loop_bless() {
   SchedParams sp{prm_.squad_max, prm_.split_pct, prm_.seed_all != 0, prm_.ablate, prm_.squad_max_solo};
   int64_t vnow = 0;   // VIRTUAL clock
   int64_t E = 0;      // WALL: predicted end of the last launched squad
+  bool join_solo = false;   // WALL, R38: this decision joins in-flight solo squads
   const size_t max_inflight = (size_t)std::max(1, prm_.max_inflight_squads);
   while (!stop_) {
     if (rt_) {
@@ -1218,9 +1237,23 @@ void Engine::loop_bless() {
     } else {
       const int64_t host = now_ns();
       const bool gpu_idle = inflight_.empty();
+      join_solo = false;
       if (!gpu_idle && (inflight_.size() >= max_inflight || host < E - prm_.lookahead_ns)) {
-        cpu_relax();
-        continue;
+        // R38 (barrier bit 1; L57 "shrinks its resources instantly when other
+        // requests arrive"): a request arriving while the GPU runs nothing but
+        // another tenant's solo NSP squads is decided now and its chain starts
+        // at once, beside the solo kernels (no preemption: they keep running,
+        // sharing the SMs through their tile queues)
+        const int l = (prm_.barrier & 2) ? solo_inflight_tenant() : -1;
+        bool arrival = false;
+        if (l >= 0 && inflight_.size() <= max_inflight)
+          for (int j = 0; j < nt && !arrival; ++j)
+            arrival = j != l && act_req[j] < 0 && !fifo_[j].empty() && reqs_[fifo_[j].front()].arrival <= host;
+        if (!arrival) {
+          cpu_relax();
+          continue;
+        }
+        join_solo = true;
       }
       for (int j = 0; j < nt; ++j)
         if (act_req[j] < 0 && !fifo_[j].empty() && reqs_[fifo_[j].front()].arrival <= host) {
@@ -1234,7 +1267,7 @@ void Engine::loop_bless() {
         cpu_relax();
         continue;
       }
-      now = gpu_idle ? host : std::max(host, E);
+      now = (gpu_idle || join_solo) ? host : std::max(host, E);
     }
     av.clear();
     for (int j = 0; j < nt; ++j)
@@ -1254,7 +1287,7 @@ void Engine::loop_bless() {
           cpu_relax();
         }
       }
-      launch_squad(dec_, act_req, act_next);
+      launch_squad(dec_, act_req, act_next, join_solo);
       if (failed_) return;
     }
     // advance the requests
@@ -1276,7 +1309,7 @@ void Engine::loop_bless() {
       }
     }
     if (virt) vnow = now + dec_.t_hat + prm_.squad_overhead_ns;
-    else E = now + dec_.t_hat;
+    else E = join_solo ? std::max(E, now + dec_.t_hat) : now + dec_.t_hat;
   }
 }
 

@@ -143,7 +143,8 @@ class Engine {
   void scan_submissions();
   void harvest();
   void retire_inflight();
-  void launch_squad(const Decision& d, const std::vector<int64_t>& act_req, const std::vector<int>& act_next);
+  void launch_squad(const Decision& d, const std::vector<int64_t>& act_req, const std::vector<int>& act_next,
+                    bool join_solo = false);
   uint64_t launch_one(int t, int k, int lo, int hi, void* stream, int64_t req, bool last, bool stamp = true);
   // parallel launch path
   bool prepare_one(int t, int k, int lo, int hi, int64_t req, bool last, std::vector<LaunchItem>& items,
@@ -196,7 +197,11 @@ class Engine {
     std::vector<void*> events;
     std::vector<int> parts;
     uint64_t squad = 0;
+    bool solo_nsp = false;   // one participant on [0, S) (R38)
   };
+  // R38 (bl_params.barrier bit 1): the tenant whose solo NSP squads are all
+  // that is in flight, or -1
+  int solo_inflight_tenant() const;
   std::vector<std::unique_ptr<Launcher>> launchers_;
   uint64_t squad_id_ = 0;
   bool par_launch_ = true;        // per-tenant launcher threads (BLESS_LAUNCH_THREADS=0 disables)

@@ -231,16 +231,17 @@ def test_ablate_out_of_range_rejected():
 
 
 def test_barrier_out_of_range_rejected():
-    """bl_params.barrier outside 0..1 is BL_E_INVALID at bl_create and at
-    bl_reset (header); 0 and 1 are accepted."""
-    for b in (-1, 2):
+    """bl_params.barrier outside 0..3 is BL_E_INVALID at bl_create and at
+    bl_reset (header); 0..3 are accepted."""
+    for b in (-1, 4):
         with pytest.raises(capi.BlessError) as e:
             capi.Ctx(capi.BL_DEVICE_NONE, clock=capi.BL_CLOCK_VIRTUAL, barrier=b)
         assert e.value.status == capi.BL_E_INVALID
     ctx = capi.Ctx(capi.BL_DEVICE_NONE, clock=capi.BL_CLOCK_VIRTUAL, barrier=1)
     with pytest.raises(capi.BlessError) as e:
-        ctx.reset(capi.default_params(clock=capi.BL_CLOCK_VIRTUAL, barrier=3))
+        ctx.reset(capi.default_params(clock=capi.BL_CLOCK_VIRTUAL, barrier=5))
     assert e.value.status == capi.BL_E_INVALID
+    ctx.reset(capi.default_params(clock=capi.BL_CLOCK_VIRTUAL, barrier=3))
     ctx.reset(capi.default_params(clock=capi.BL_CLOCK_VIRTUAL, barrier=0))
     ctx.close()
 

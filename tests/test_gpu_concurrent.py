@@ -98,10 +98,14 @@ def squads_of(decisions, launches):
     return out
 
 
-def check_squad_barrier(decisions, launches, res_ns=64):
+def check_squad_barrier(decisions, launches, res_ns=64, join_solo=False):
+    """join_solo (bl_params.barrier bit 1, reading R38): a squad that follows
+    a solo NSP squad may start beside it and is not checked against it."""
     sq = squads_of(decisions, launches)
     n_pairs = 0
-    for a, b in zip(sq, sq[1:]):
+    for (da, a), b in zip(zip(decisions, sq), sq[1:]):
+        if join_solo and da.n_part == 1 and not da.config_sp:
+            continue
         end_by_tenant = {}
         for r in a:
             assert r.end_ns > 0 and r.nsm > 0, (r.tenant, r.kernel)
@@ -135,14 +139,15 @@ def check_range_barrier(decisions, launches, res_ns=64):
     return n_pairs
 
 
-@pytest.mark.parametrize("policy", ["BLESS", "BLESS_1thread", "BLESS_range", "STATIC"])
+@pytest.mark.parametrize("policy", ["BLESS", "BLESS_1thread", "BLESS_range", "BLESS_join", "STATIC"])
 def test_concurrent_every_layer_vs_oracle(world, policy):
     cfg, ctx, ms, prof = world
     squad_max = {"C2": 20, "C3": 10, "C4": 10}[cfg]
     # BLESS_range: the SM-range barrier (R37) with strict SP squads (c = 100%),
     # where chains on disjoint partitions stop waiting for each other
-    split_pct, barrier = (100, 1) if policy == "BLESS_range" else (25, 0)
-    waves = [(0, 11), (60_000, 12)] if policy in ("BLESS", "BLESS_range") else [(0, 21)]
+    # BLESS_join: arrivals join in-flight solo NSP squads at once (R38)
+    split_pct, barrier = {"BLESS_range": (100, 1), "BLESS_join": (25, 2)}.get(policy, (25, 0))
+    waves = [(0, 11), (60_000, 12)] if policy in ("BLESS", "BLESS_range", "BLESS_join") else [(0, 21)]
     old = os.environ.get("BLESS_LAUNCH_THREADS")
     if policy == "BLESS_1thread":
         os.environ["BLESS_LAUNCH_THREADS"] = "0"
@@ -156,7 +161,8 @@ def test_concurrent_every_layer_vs_oracle(world, policy):
             msg = f"\n{cfg} {policy} stagger={stagger}: {sum(len(m.layers) for m in ms)} layers, worst {worst:.2e}"
             if policy != "STATIC":
                 assert decisions
-                pairs = (check_range_barrier if barrier else check_squad_barrier)(decisions, launches)
+                pairs = (check_range_barrier(decisions, launches) if barrier & 1 else
+                         check_squad_barrier(decisions, launches, join_solo=bool(barrier & 2)))
                 sp_sq = sum(1 for d in decisions if d.config_sp)
                 for rec in decisions:
                     got = capi.decision_to_tuple(rec)
