@@ -548,12 +548,16 @@ def native(args):
     world = int(os.environ.get("WORLD_SIZE", 1))
     local = int(os.environ.get("LOCAL_RANK", 0))
     dist = None
+    # BLESS_BENCH_DEVICE=d puts every replica on device d: a plumbing check of
+    # the multi-rank path on a one-GPU box (replicas never wait on each other;
+    # its numbers are not scaling measurements)
+    force_dev = os.environ.get("BLESS_BENCH_DEVICE")
     if world > 1:
         import torch.distributed as dist
         dist.init_process_group("gloo")   # host-side barrier and reductions only (no NCCL: nothing shards)
-        gpus = [(rank, local)]
+        gpus = [(rank, local if force_dev is None else int(force_dev))]
     else:
-        gpus = [(g, g) for g in range(max(1, args.gpus))]
+        gpus = [(g, g if force_dev is None else int(force_dev)) for g in range(max(1, args.gpus))]
     n_box = world if world > 1 else len(gpus)
     os.makedirs(args.out_dir, exist_ok=True)
     # tcgen05 tile configurations are autotuned at registration; a saved profile
