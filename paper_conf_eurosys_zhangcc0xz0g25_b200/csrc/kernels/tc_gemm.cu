@@ -503,11 +503,6 @@ struct TcCfg {
   static constexpr int kSmemMax = kMaxStages * kStageBytes + kFixed;
 };
 
-#ifdef TEST_A
-#define PROD_DEP_WAIT(g) pdl_wait()
-#else
-#define PROD_DEP_WAIT(g) dep_wait(g)
-#endif
 template <int BN, int BK, bool HALO, int MH>
 __device__ void tc_work(const TcParams& p, const GateArgs& g) {
   using Cfg = TcCfg<BN, BK, MH>;
@@ -688,7 +683,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
             if (!dep_waited) {   // weights before the grid dependency resolves, activations after
               tap0 = min(taps, ST);
               for (int tap = 0; tap < tap0; ++tap) load_Bt(c, tap);
-              PROD_DEP_WAIT(g);
+              dep_wait(g);
               if (t == 0 && lane == 0) gate_prev_end(g, (int64_t)ptx_globaltimer());
               if (lane == 0) TR(4);
               dep_waited = true;
@@ -709,7 +704,7 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
             mbar_expect_tx_e(&full[st], kTxBytes);
             if (!kSkipB) load_B(kb0 + i, st);
           }
-          PROD_DEP_WAIT(g);
+          dep_wait(g);
           if (t == 0 && lane == 0) gate_prev_end(g, (int64_t)ptx_globaltimer());   // predecessor just completed
           if (lane == 0) TR(4);          // 4: producer past griddepcontrol.wait
           dep_waited = true;
