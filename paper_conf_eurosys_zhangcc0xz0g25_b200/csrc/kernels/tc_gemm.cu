@@ -917,13 +917,23 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         __threadfence();
 #endif
         // release: the CTA barrier orders every epilogue thread's reds before
-        // thread 64's gpu-scope fence (fences are cumulative), which precedes
-        // its arrival on the tile's counter; one fence per unit instead of 256
+        // thread 64's gpu-scope release (cumulative), which is its arrival on
+        // the tile's counter; one release per unit instead of 256
         asm volatile("bar.sync 1, %0;" ::"n"(32 * kEpiWarps) : "memory");   // all epilogue warps
         if (threadIdx.x == 64) {
+#ifndef BLESS_TC_SPLIT_FENCE_ATOM
+          // one acq_rel atomic: release of this unit's reds (ordered before it
+          // by the barrier above), acquire of the other units' for the last one.
+          // B200: 0.35-0.7 us less per split-K launch than fence + atomic +
+          // fence (profiles/round2/splitk_acqrel/), same parity.
+          unsigned prev_arr;
+          asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(prev_arr) : "l"(p.sem + tile) : "memory");
+          const bool last = prev_arr == (unsigned)p.splits - 1;
+#else   // A/B reference: __threadfence + relaxed atomic (+ __threadfence on the last unit)
           __threadfence();
           const bool last = atomicAdd(p.sem + tile, 1u) == (unsigned)p.splits - 1;
           if (last) __threadfence();   // acquire: the other units' reds before our ld.cg reads
+#endif
           *last_flag = last ? 1 : 0;
           TR(10);                          // 10: fence + tile counter arrival done (split-K)
         }
