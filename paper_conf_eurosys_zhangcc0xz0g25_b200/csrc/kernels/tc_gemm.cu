@@ -881,12 +881,10 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty[acc]);
         if (threadIdx.x == 64) TR(7);    // 7: epilogue stores issued (last tile)
-        if (g.count_done) {   // software dependency: this unit's stores, then the count
+        if (g.count_done) {   // software dependency: this unit's stores, then the count (release)
           asm volatile("bar.sync 1, %0;" ::"n"(32 * kEpiWarps) : "memory");
-          if (threadIdx.x == 64) {
-            __threadfence();
-            atomicAdd(const_cast<unsigned long long*>(&g.slot->done), 1ull);
-          }
+          if (threadIdx.x == 64)
+            asm volatile("red.release.gpu.global.add.u64 [%0], 1;" ::"l"(&g.slot->done) : "memory");
         }
       } else {
         // split-K: add this unit's partial tile into the fp32 workspace
@@ -953,10 +951,8 @@ __device__ void tc_work(const TcParams& p, const GateArgs& g) {
         }
         if (g.count_done) {   // software dependency: partial (or the tile's final stores), then the count
           asm volatile("bar.sync 1, %0;" ::"n"(32 * kEpiWarps) : "memory");
-          if (threadIdx.x == 64) {
-            __threadfence();
-            atomicAdd(const_cast<unsigned long long*>(&g.slot->done), 1ull);
-          }
+          if (threadIdx.x == 64)
+            asm volatile("red.release.gpu.global.add.u64 [%0], 1;" ::"l"(&g.slot->done) : "memory");
         }
       }
       if (++acc == Cfg::kAcc) { acc = 0; aph ^= 1; }
