@@ -16,6 +16,8 @@ from __future__ import annotations
 from dataclasses import dataclass, field
 from typing import Dict, List, Optional, Sequence
 
+import os
+
 import numpy as np
 import torch
 
@@ -112,7 +114,10 @@ class Builder:
             # first layers (C = 3): explicit im2col into a zero-padded [M, Kpad]
             # matrix, then the conv is a tensor-core GEMM
             K = k * k * C
-            Kpad = (K + 63) // 64 * 64
+            # K padding of the im2col matrix: 32 (B200: VGG conv1 im2col 10.0 -> 7.7 us
+            # vs 64, profiles/round2/im2col_kalign/); BLESS_IM2COL_KALIGN for A/B
+            ka = int(os.environ.get("BLESS_IM2COL_KALIGN", "32"))
+            Kpad = (K + ka - 1) // ka * ka
             cols = self.act_buf((N * OH * OW, Kpad))
             op = self._op(capi.BL_OP_IM2COL, "none", [N, H, W, C, k, k, stride, pad, Kpad], [x, cols])
             self.ctx.append_kernel(self.m.tenant, op)
