@@ -1126,14 +1126,13 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
         wsqs[j].push_back(c.squad);
       }
   if (join_solo) {   // R38: the arrival does not wait for the in-flight solo squads
-    for (auto& w : wparts) w.clear();
-    for (auto& w : wevs) w.clear();
-    for (auto& w : wsqs) w.clear();
+    wparts.assign(nt, {});
+    wevs.assign(nt, {});
+    wsqs.assign(nt, {});
   }
   if (launchers_.empty()) {   // single launch thread (BLESS_LAUNCH_THREADS=0)
     for (int j : d.parts) {
-      if (join_solo) {
-      } else if (rbar) {
+      if (rbar || join_solo) {   // (join_solo: the lists were cleared above)
         for (void* e : wevs[j]) rt_->stream_wait(ten_[j].stream, e);
       } else {
         for (size_t i = 0; i < prev_events_.size(); ++i)   // own stream: already ordered (see launcher_main)
@@ -1152,9 +1151,7 @@ void Engine::launch_squad(const Decision& d, const std::vector<int64_t>& act_req
   if (!launchers_.empty()) {
     for (int j : d.parts) {
       jobs[j].squad = sq;
-      if (join_solo) {
-        jobs[j].wait_squad = 0;
-      } else if (rbar) {
+      if (rbar || join_solo) {
         jobs[j].wait_squad = wparts[j].empty() ? 0 : 1;
         jobs[j].wait_parts = std::move(wparts[j]);
         jobs[j].wait_sq = std::move(wsqs[j]);
