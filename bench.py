@@ -76,6 +76,7 @@ def parse():
     ap.add_argument("--split-pct", type=int, default=25)
     ap.add_argument("--squad-max-solo", type=int, default=0,
                     help="reading R36: cap of a squad with a single active request (0 = S_max)")
+    ap.add_argument("--seed-all", type=int, default=1, help="reading R6: seed every active request first (1) or pick by lag only (0)")
     ap.add_argument("--ablate", type=int, default=0,
                     help="PAPER.md §6.8 ablation (R32): 1 = no multi-task scheduler, 2 = no determiner, 3 = both")
     ap.add_argument("--barrier", type=int, default=0,
@@ -279,7 +280,7 @@ class Replica:
         self.quota_sms = [self.ctx.tenant_info(m.tenant)[0] for m in self.tms]
 
     def params(self, capi, args, pol="BLESS", extra=None):
-        return capi.default_params(squad_max=self.squad_max, policy=pol, split_pct=args.split_pct,
+        return capi.default_params(squad_max=self.squad_max, policy=pol, split_pct=args.split_pct, seed_all=args.seed_all,
                                    ablate=args.ablate, squad_max_solo=args.squad_max_solo,
                                    lookahead_ns=int(args.lookahead_us * 1000),
                                    max_inflight_squads=args.max_inflight, barrier=args.barrier,
@@ -781,7 +782,7 @@ def native(args):
         from oracle.sched_ref import Params, Prof
         r0 = reps[0]
         prm = Params(squad_max=r0.squad_max, split_pct=args.split_pct, ablate=args.ablate,
-                     squad_max_solo=args.squad_max_solo)
+                     squad_max_solo=args.squad_max_solo, seed_all=bool(args.seed_all))
         replay_ok = replay_all(dec, r0.prof_path, prm)
         if world == 1 and nrep == 1 and not args.no_cpu_baseline:
             prof = Prof(synprof.load(r0.prof_path))
@@ -841,6 +842,7 @@ def native(args):
                    f"per tenant, {args.requests} requests/tenant/step, seeds 1-3, box-wide trace routed by the "
                    "native dispatcher (bl_dispatch)", "squad_max": r0.squad_max,
                    "split_pct": args.split_pct, "ablate": args.ablate, "squad_max_solo": args.squad_max_solo, "barrier": args.barrier,
+                   "seed_all": args.seed_all,
                    "parallelism": f"replicas x{n_box} (no collective; "
                                   f"{'one process per GPU, gloo host barrier' if world > 1 else 'one process'})",
                    "quotas": [m.quota for m in r0.tms],
